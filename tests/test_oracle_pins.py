@@ -1,0 +1,327 @@
+"""Pins for the fp64 oracle, run on CPU (-m "not gpu").
+
+Each test checks the oracle against something other than itself: a closed form,
+a hand-computed value (tests/golden), or an independent library routine
+(torch.nn.functional.conv2d / grid_sample, torchvision.ops.deform_conv2d), in fp64.
+Each is chosen so that a plausible slip in the oracle (dropped tap, swapped dy/dx,
+transposed (i,j), wrong group index, off-by-one border, truncation instead of floor,
+mask applied to the wrong tap) fails at least one of them.
+"""
+import os
+
+import numpy as np
+import pytest
+import torch
+import torch.nn.functional as F
+
+from defcon_workloads import configs, inputs
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+rng = np.random.default_rng(12345)
+
+
+def nchw(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float64)).permute(0, 3, 1, 2)
+
+
+def oihw(w):
+    return torch.from_numpy(np.ascontiguousarray(w, np.float64)).permute(0, 3, 1, 2)
+
+
+def nhwc(t):
+    return t.permute(0, 2, 3, 1).contiguous().numpy()
+
+
+def rand_layer(N=2, H=7, W=9, Cin=8, Cout=5, K=3, G=1, stride=1, pad=1, dil=1, seed=0):
+    r = np.random.default_rng(seed)
+    Ho = configs.out_size(H, K, stride, pad, dil)
+    Wo = configs.out_size(W, K, stride, pad, dil)
+    x = r.standard_normal((N, H, W, Cin))
+    w = r.standard_normal((Cout, K, K, Cin))
+    b = r.standard_normal(Cout)
+    off = 1.5 * r.standard_normal((N, Ho, Wo, G, K * K, 2))
+    m = r.random((N, Ho, Wo, G, K * K))
+    return x, w, b, off, m, Ho, Wo
+
+
+# ---------------------------------------------------------------- P1: Eq.1 special case
+@pytest.mark.parametrize("stride,H,W", [(1, 7, 9), (2, 9, 8), (2, 35, 35)])
+@pytest.mark.parametrize("dil", [1, 2])
+def test_p1_zero_offsets_equal_regular_conv(oracle_mod, stride, H, W, dil):
+    """Zero offsets, m = 1: Eq.2 reduces to Eq.1 == F.conv2d in fp64."""
+    x, w, b, _, _, Ho, Wo = rand_layer(H=H, W=W, stride=stride, dil=dil, pad=dil, Cin=6, Cout=4)
+    off = np.zeros((x.shape[0], Ho, Wo, 1, 9, 2))
+    y = oracle_mod.dcn_forward(x, off, w, b, stride=stride, pad=dil, dil=dil)
+    ref = nhwc(F.conv2d(nchw(x), oihw(w), torch.from_numpy(b), stride=stride, padding=dil,
+                        dilation=dil))
+    assert y.shape == ref.shape
+    np.testing.assert_allclose(y, ref, rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- P2: integer offsets
+def _shift(xt, dy, dx):
+    """x'(q) = x(q + (dy, dx)) with zeros outside (NCHW)."""
+    N, C, H, W = xt.shape
+    out = torch.zeros_like(xt)
+    ys, yd = (slice(dy, H), slice(0, H - dy)) if dy >= 0 else (slice(0, H + dy), slice(-dy, H))
+    xs, xd = (slice(dx, W), slice(0, W - dx)) if dx >= 0 else (slice(0, W + dx), slice(-dx, W))
+    out[:, :, yd, xd] = xt[:, :, ys, xs]
+    return out
+
+
+def test_p2_integer_offsets_are_shifted_taps(oracle_mod):
+    """Per-tap integer offsets (distinct dy != dx per tap) give exactly shifted taps:
+    y = b + sum_k conv_k(shift(x, dy_k, dx_k)) with the single-tap kernel k.  A swapped
+    dy/dx, transposed (i,j) or misplaced tap index changes the result."""
+    x, w, b, _, _, Ho, Wo = rand_layer(H=8, W=10, Cin=4, Cout=3, seed=3)
+    N = x.shape[0]
+    taps = [(1, 0), (0, -2), (2, 1), (-1, 3), (0, 0), (-3, -1), (1, 2), (2, -2), (-2, 0)]
+    off = np.zeros((N, Ho, Wo, 1, 9, 2))
+    for k, (dy, dx) in enumerate(taps):
+        off[..., 0, k, 0] = dy
+        off[..., 0, k, 1] = dx
+    y = oracle_mod.dcn_forward(x, off, w, b)
+    P = 5   # shift on a zero-extended domain so that padding taps can land inside the image
+    xt = F.pad(nchw(x), (P, P, P, P))
+    H, W = x.shape[1:3]
+    ref = torch.zeros(N, 3, Ho, Wo, dtype=torch.float64) + torch.from_numpy(b)[None, :, None, None]
+    for k, (dy, dx) in enumerate(taps):
+        wk = torch.zeros(3, 4, 3, 3, dtype=torch.float64)
+        i, j = divmod(k, 3)
+        wk[:, :, i, j] = oihw(w)[:, :, i, j]
+        xs = _shift(xt, dy, dx)[:, :, P - 1:P + H + 1, P - 1:P + W + 1]
+        ref += F.conv2d(xs, wk)
+    np.testing.assert_allclose(y, nhwc(ref), rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- P3: half-pixel closed form
+def test_p3_half_pixel_equals_box_average(oracle_mod):
+    """dp = (0.5, 0.5) on every tap: x(q + 0.5) is the mean of the 2x2 block at q
+    (zeros outside), so y = conv2d of the 2x2 box average (avg_pool2d) of padded x."""
+    x, w, b, _, _, Ho, Wo = rand_layer(H=7, W=6, Cin=3, Cout=2, seed=4)
+    off = np.full((x.shape[0], Ho, Wo, 1, 9, 2), 0.5)
+    y = oracle_mod.dcn_forward(x, off, w, b)
+    xp = F.pad(nchw(x), (2, 2, 2, 2))
+    xa = F.avg_pool2d(xp, 2, stride=1)        # xa[t] = x~(t - 2 + 0.5)
+    # y(ho) = sum_i w_i x~(ho - 1 + i + 0.5) = sum_i w_i xa[ho + i + 1]
+    ref = F.conv2d(xa[:, :, 1:, 1:], oihw(w), torch.from_numpy(b))
+    ref = ref[:, :, :Ho, :Wo]
+    np.testing.assert_allclose(y, nhwc(ref), rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- P4: far out of bounds
+def test_p4_far_oob_gives_bias(oracle_mod):
+    x, w, b, _, m, Ho, Wo = rand_layer(H=6, W=5, seed=5)
+    s = np.where(rng.random((x.shape[0], Ho, Wo, 1, 9, 2)) < 0.5, -1, 1)
+    off = s * (max(6, 5) + 1 + rng.random(s.shape) * 3)
+    y = oracle_mod.dcn_forward(x, off, w, b, mask=m)
+    assert np.array_equal(y, np.broadcast_to(b, y.shape))
+
+
+# ---------------------------------------------------------------- P5: mask
+def test_p5_mask_one_zero_linear(oracle_mod):
+    x, w, b, off, m, Ho, Wo = rand_layer(seed=6, G=2)
+    v1 = oracle_mod.dcn_forward(x, off, w, b, G=2)
+    ones = oracle_mod.dcn_forward(x, off, w, b, mask=np.ones_like(m), G=2)
+    assert np.array_equal(v1, ones)
+    zeros = oracle_mod.dcn_forward(x, off, w, b, mask=np.zeros_like(m), G=2)
+    assert np.array_equal(zeros, np.broadcast_to(b, zeros.shape))
+    m2 = rng.random(m.shape)
+    ya = oracle_mod.dcn_forward(x, off, w, b, mask=m, G=2) - b
+    yb = oracle_mod.dcn_forward(x, off, w, b, mask=m2, G=2) - b
+    yab = oracle_mod.dcn_forward(x, off, w, b, mask=m + 0.5 * m2, G=2) - b
+    np.testing.assert_allclose(yab, ya + 0.5 * yb, rtol=0, atol=1e-11)
+
+
+def test_p5_mask_is_per_tap(oracle_mod):
+    """Masking only tap k equals the single-tap conv for that tap (k = i*Kw + j)."""
+    x, w, b, _, _, Ho, Wo = rand_layer(H=6, W=7, Cin=3, Cout=2, seed=7)
+    N = x.shape[0]
+    off = np.zeros((N, Ho, Wo, 1, 9, 2))
+    for k in range(9):
+        m = np.zeros((N, Ho, Wo, 1, 9))
+        m[..., 0, k] = 1.0
+        y = oracle_mod.dcn_forward(x, off, w, b, mask=m)
+        wk = torch.zeros(2, 3, 3, 3, dtype=torch.float64)
+        i, j = divmod(k, 3)
+        wk[:, :, i, j] = oihw(w)[:, :, i, j]
+        ref = F.conv2d(nchw(x), wk, torch.from_numpy(b), padding=1)
+        np.testing.assert_allclose(y, nhwc(ref), rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- P6: hand values
+def test_p6_hand_computed_bilinear(oracle_mod):
+    rows = np.loadtxt(os.path.join(HERE, "golden", "bilinear_2x2.txt"), comments="#")
+    x = np.array([[1.0, 2.0], [3.0, 4.0]]).reshape(1, 2, 2, 1)
+    w = np.ones((1, 1, 1, 1))
+    for dy, dx, expect in rows:
+        off = np.zeros((1, 2, 2, 1, 1, 2))
+        off[..., 0] = dy
+        off[..., 1] = dx
+        y = oracle_mod.dcn_forward(x, off, w, None, pad=0)
+        assert abs(y[0, 0, 0, 0] - expect) < 1e-12, (dy, dx, y[0, 0, 0, 0], expect)
+        assert abs(oracle_mod.bilinear(x[0, :, :, 0], dy, dx) - expect) < 1e-12
+
+
+# ---------------------------------------------------------------- P7: library routine
+def test_p7_k1_equals_grid_sample(oracle_mod):
+    """K=1 DCN == grid_sample(bilinear, zeros, align_corners=True) then a 1x1 conv."""
+    N, H, W, C, Co = 2, 9, 11, 5, 4
+    r = np.random.default_rng(8)
+    x = r.standard_normal((N, H, W, C))
+    w = r.standard_normal((Co, 1, 1, C))
+    b = r.standard_normal(Co)
+    off = 3.0 * r.standard_normal((N, H, W, 1, 1, 2))
+    y = oracle_mod.dcn_forward(x, off, w, b, pad=0)
+    py = np.arange(H)[None, :, None] + off[..., 0, 0, 0]
+    px = np.arange(W)[None, None, :] + off[..., 0, 0, 1]
+    grid = np.stack([2 * px / (W - 1) - 1, 2 * py / (H - 1) - 1], axis=-1)
+    s = F.grid_sample(nchw(x), torch.from_numpy(grid), mode="bilinear", padding_mode="zeros",
+                      align_corners=True)
+    ref = F.conv2d(s, oihw(w), torch.from_numpy(b))
+    np.testing.assert_allclose(y, nhwc(ref), rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- P8: groups
+def test_p8_groups_sum_of_blocks(oracle_mod):
+    """A G-group DCN equals the sum of per-block G=1 DCNs (R5: contiguous blocks)."""
+    G, Cin = 4, 8
+    x, w, b, off, m, Ho, Wo = rand_layer(Cin=Cin, G=G, seed=9)
+    y = oracle_mod.dcn_forward(x, off, w, b, mask=m, G=G)
+    Cg = Cin // G
+    acc = np.broadcast_to(b, y.shape).copy()
+    for g in range(G):
+        sl = slice(g * Cg, (g + 1) * Cg)
+        acc += oracle_mod.dcn_forward(x[..., sl], off[:, :, :, g:g + 1], w[..., sl], None,
+                                      mask=m[:, :, :, g:g + 1])
+    np.testing.assert_allclose(y, acc, rtol=0, atol=1e-11)
+
+
+# ---------------------------------------------------------------- P9: torchvision
+@pytest.mark.parametrize("G,stride,dil,mod", [(1, 1, 1, True), (2, 2, 1, True), (4, 1, 2, False),
+                                               (1, 2, 2, True)])
+def test_p9_matches_torchvision(oracle_mod, G, stride, dil, mod):
+    tv = pytest.importorskip("torchvision.ops")
+    x, w, b, off, m, Ho, Wo = rand_layer(N=2, H=11, W=9, Cin=8, Cout=6, G=G, stride=stride,
+                                         dil=dil, pad=dil, seed=10 + G)
+    off = off * 2.0
+    y = oracle_mod.dcn_forward(x, off, w, b, mask=m if mod else None, stride=stride, pad=dil,
+                               dil=dil, G=G)
+    N = x.shape[0]
+    off_t = torch.from_numpy(off.reshape(N, Ho, Wo, G * 9 * 2)).permute(0, 3, 1, 2)
+    m_t = torch.from_numpy(m.reshape(N, Ho, Wo, G * 9)).permute(0, 3, 1, 2) if mod else None
+    ref = tv.deform_conv2d(nchw(x), off_t, oihw(w), torch.from_numpy(b), stride=stride,
+                           padding=dil, dilation=dil, mask=m_t)
+    np.testing.assert_allclose(y, nhwc(ref), rtol=0, atol=1e-10)
+
+
+def test_pixels_equals_grid(oracle_mod):
+    x, w, b, off, m, Ho, Wo = rand_layer(seed=20, G=2)
+    y = oracle_mod.dcn_forward(x, off, w, b, mask=m, G=2)
+    idx = np.array([0, 5, 17, x.shape[0] * Ho * Wo - 1])
+    yp = oracle_mod.dcn_pixels(x, off, w, idx, b, mask=m, G=2)
+    assert np.array_equal(yp, y.reshape(-1, y.shape[-1])[idx])
+
+
+# ---------------------------------------------------------------- P10: offset branch
+@pytest.mark.parametrize("G,with_mask,stride", [(1, True, 1), (4, True, 2), (2, False, 1)])
+def test_p10_offset_branch_matches_torch(oracle_mod, G, with_mask, stride):
+    r = np.random.default_rng(30 + G)
+    N, H, W, C, K = 2, 9, 8, 6, 3
+    x = r.standard_normal((N, H, W, C))
+    dw = r.standard_normal((C, 3, 3))
+    sc, sh = r.uniform(0.5, 1.5, C), 0.3 * r.standard_normal(C)
+    OC = G * K * K * (3 if with_mask else 2)
+    w2, b2 = r.standard_normal((OC, C)), r.standard_normal(OC)
+    off, msk = oracle_mod.offset_branch(x, dw, sc, sh, w2, b2, K=K, G=G, with_mask=with_mask,
+                                        stride=stride)
+    t = F.conv2d(nchw(x), torch.from_numpy(dw)[:, None], stride=stride, padding=1, groups=C)
+    t = torch.relu(t * torch.from_numpy(sc)[None, :, None, None]
+                   + torch.from_numpy(sh)[None, :, None, None])
+    u = F.conv2d(t, torch.from_numpy(w2)[:, :, None, None], torch.from_numpy(b2))
+    u = nhwc(u)
+    n_off = 2 * G * K * K
+    np.testing.assert_allclose(off.reshape(*off.shape[:3], -1), u[..., :n_off], rtol=0, atol=1e-12)
+    if with_mask:
+        np.testing.assert_allclose(msk.reshape(*msk.shape[:3], -1),
+                                   torch.sigmoid(torch.from_numpy(u[..., n_off:])).numpy(),
+                                   rtol=0, atol=1e-14)
+    else:
+        assert msk is None
+
+
+def test_p10_zero_w2_gives_bias(oracle_mod):
+    r = np.random.default_rng(40)
+    x = r.standard_normal((1, 5, 5, 4))
+    OC = 27
+    b2 = r.standard_normal(OC)
+    off, msk = oracle_mod.offset_branch(x, r.standard_normal((4, 3, 3)), np.ones(4), np.zeros(4),
+                                        np.zeros((OC, 4)), b2)
+    assert np.array_equal(off[0, 2, 3].reshape(-1), b2[:18])
+    np.testing.assert_allclose(msk[0, 1, 1].reshape(-1), 1 / (1 + np.exp(-b2[18:])), atol=1e-15)
+
+
+# ---------------------------------------------------------------- P11: continuity
+def test_p11_continuity(oracle_mod):
+    """Eq.3 is continuous: crossing an integer grid line changes y by O(eps)."""
+    x, w, b, off, m, Ho, Wo = rand_layer(seed=50)
+    off = np.round(off)
+    ya = oracle_mod.dcn_forward(x, off - 1e-9, w, b, mask=m)
+    yb = oracle_mod.dcn_forward(x, off + 1e-9, w, b, mask=m)
+    assert np.max(np.abs(ya - yb)) < 1e-6
+
+
+# ---------------------------------------------------------------- P13: texture model
+def test_p13_texq_exact_on_256th_grid(oracle_mod):
+    """With fractions already multiples of 1/256 the quantised filter is exact."""
+    x, w, b, off, m, Ho, Wo = rand_layer(seed=60)
+    off = np.round(off * 256) / 256
+    ye = oracle_mod.dcn_forward(x, off, w, b, mask=m)
+    for q in ("round", "trunc"):
+        yq = oracle_mod.dcn_forward_texq(x, off, w, b, mask=m, quant=q)
+        np.testing.assert_allclose(yq, ye, rtol=0, atol=1e-12)
+
+
+def test_p13_texq_error_bound(oracle_mod):
+    """Per-sample |quantised - exact| <= (|da_y| + |da_x|) * 2 max|x| with |da| <= 1/512
+    (round) or < 1/256 (trunc); checked with K=1, w=1 so y is a single sample."""
+    r = np.random.default_rng(61)
+    x = r.standard_normal((1, 8, 8, 1))
+    off = 3 * r.standard_normal((1, 8, 8, 1, 1, 2))
+    w = np.ones((1, 1, 1, 1))
+    ye = oracle_mod.dcn_forward(x, off, w, None, pad=0)
+    for q, da in (("round", 1 / 512), ("trunc", 1 / 256)):
+        yq = oracle_mod.dcn_forward_texq(x, off, w, None, pad=0, quant=q)
+        bound = 2 * da * 2 * np.max(np.abs(x)) + 1e-12
+        assert np.max(np.abs(yq - ye)) <= bound
+        assert np.max(np.abs(yq - ye)) > 0
+
+
+# ---------------------------------------------------------------- P14: FLOP model
+def test_p14_eq9_mac_saving():
+    """Eq.9 prints 83.3% for k = 3."""
+    assert round(100 * configs.lightweight_mac_saving(3), 1) == 83.3
+    c = configs.C4.replace(modulated=False)
+    regular = c.M * c.Cin * 9 * 2 * 9
+    assert abs(1 - configs.offset_branch_macs(c) / regular - 0.8333333) < 1e-6
+
+
+def test_flop_model_values():
+    """11.23 / 23.12 / 48.92 GFLOP for C3 / C4 / C5."""
+    for c, gf in ((configs.C3, 11.23), (configs.C4, 23.12), (configs.C5, 48.92)):
+        assert round(configs.contraction_flops(c) / 1e9, 2) == gf
+    assert len(configs.stack_layers()) == 11
+
+
+def test_out_size_matches(oracle_mod):
+    for args in [(35, 3, 2, 1, 1), (69, 3, 1, 1, 1), (2, 3, 2, 0, 1), (1, 3, 1, 0, 1), (18, 3, 1, 1, 2)]:
+        assert oracle_mod.out_size(*args) == configs.out_size(*args)
+
+
+def test_inputs_are_seeded_per_image():
+    c = configs.C4.replace(N=3, H=5, W=5, Cin=8, Cout=8)
+    full = inputs.gen_x(c)
+    part = inputs.gen_x(c, images=[2])
+    assert np.array_equal(full[2:3], part)
+    xb = inputs.gen_x(c)
+    assert np.array_equal(inputs.round_to(xb, "bf16"), xb)
