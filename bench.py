@@ -1,0 +1,459 @@
+#!/usr/bin/env python3
+"""DEFCON hot-path benchmark on B200 (contract: one JSON line from rank 0).
+
+Workload (BASELINE.json configs[2], the north-star target): YOLACT++ ResNet-101 C4 DCNv2
+3x3 layer, N=16 images per GPU, C=256, 35x35, offset_groups=1, bf16 storage, fed by the
+paper's lightweight depthwise offset branch.  One "step" = one pass of the
+whole hot path over one batch: defcon_offset_dw_conv (step 1) + defcon_dcn_forward (step 2).
+
+metric: contraction TFLOP/s (2*M*Cout*K^2*Cin per layer), higher is better;
+ms_per_step gives the layer latency.  value = FLOPs of all ranks / max-over-ranks time.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+Multi-GPU: launched by torchrun (one rank per GPU, NCCL, weak scaling by image).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from defcon_workloads import configs, inputs  # noqa: E402
+
+WORKLOAD = configs.C4
+L2_BYTES = 126 * 2**20
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary.json")
+
+
+def metric_name():
+    return "DCNv2 layer TFLOP/s (contraction) at YOLACT++ C4 shape, incl. offset branch"
+
+
+def workload_config(c, world, extra=None):
+    d = {
+        "workload": f"{c.name}: N={c.N}/GPU Cin=Cout={c.Cin} {c.H}x{c.W} K={c.K} stride={c.stride} "
+                    f"G={c.G} DCNv2 {c.dtype} + lightweight offset branch (dw3x3+BN+ReLU+1x1)",
+        "global_batch": c.N * world,
+        "parallelism": f"dp{world} (images sharded, no data-path collective)",
+    }
+    if extra:
+        d.update(extra)
+    return d
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_PATH) as f:
+            p = json.load(f)
+        return p, "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+# ------------------------------------------------------------------ clocks sampler
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+        self.t = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append((time.time(), line.strip()))
+
+    def stop(self):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        if self.t is not None:
+            self.t.join(timeout=2)
+
+    def summary(self, t0, t1):
+        rows = [l for (t, l) in self.lines if t0 - 0.06 <= t <= t1 + 0.06] or [l for _, l in self.lines]
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            parts = [p.strip() for p in r.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ GPU arm
+class Layer:
+    """Device-resident inputs/outputs of one buffer set (one batch of the workload)."""
+
+    def __init__(self, c, images, dev, branch_dev, weight, bias):
+        dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
+        self.x = torch.from_numpy(inputs.gen_x(c, images)).to(dev, dt)
+        KK = c.K * c.K
+        self.off = torch.empty((c.N, c.Ho, c.Wo, c.G, KK, 2), device=dev, dtype=torch.float32)
+        self.msk = torch.empty((c.N, c.Ho, c.Wo, c.G, KK), device=dev, dtype=torch.float32)
+        self.y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
+        self.branch = branch_dev
+        self.weight = weight
+        self.bias = bias
+
+    def nbytes(self):
+        return sum(t.numel() * t.element_size() for t in (self.x, self.off, self.msk, self.y,
+                                                           self.weight))
+
+
+def step1(d, c, L):
+    B = L.branch
+    d.defcon_offset_dw_conv(L.x, B["dw_w"], B["dw_scale"], B["dw_shift"], B["pw_w"], B["pw_b"],
+                            K=c.K, stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
+                            with_mask=c.modulated, offset=L.off, mask=L.msk)
+
+
+def step2(d, c, L):
+    d.defcon_dcn_forward(L.x, L.off, L.msk, L.weight, L.bias, stride=c.stride, pad=c.pad,
+                         dil=c.dil, offset_groups=c.G, y=L.y)
+
+
+def capture(fn, stream):
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=stream):
+        fn()
+    return g
+
+
+def gpu_arm(args, rank, world, local_rank, dist):
+    import paper_conf_ipps_jayaweeralwrk24_b200 as d
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    d.load_library()
+    c = WORKLOAD
+    # per-rank images: weak scaling, each rank regenerates exactly its own shard
+    images = list(range(rank * c.N, (rank + 1) * c.N))
+    P = inputs.gen_offset_branch(c)
+    w, b = inputs.gen_weight(c)
+    dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
+
+    # Rotate buffer sets so the sets touched between two visits exceed L2 (cold-L2 timing).
+    probe_bytes = (c.N * c.H * c.W * c.Cin * 2 + c.M * c.Cout * 2 + c.M * 27 * 4 +
+                   c.Cout * 9 * c.Cin * 2)
+    R = max(2, int(np.ceil(1.5 * L2_BYTES / probe_bytes)))
+    sets = []
+    for r in range(R):
+        Pd = {k: torch.from_numpy(v).to(dev) for k, v in P.items()}
+        sets.append(Layer(c, images, dev, Pd, torch.from_numpy(w).to(dev, dt),
+                          torch.from_numpy(b).to(dev)))
+    rot_bytes = sum(L.nbytes() for L in sets)
+
+    stream = torch.cuda.Stream(device=dev)
+    with torch.cuda.stream(stream):
+        for L in sets:          # eager warm-up outside capture (module load, attributes)
+            step1(d, c, L)
+            step2(d, c, L)
+    torch.cuda.synchronize()
+    g_step = [capture(lambda L=L: (step1(d, c, L), step2(d, c, L)), stream) for L in sets]
+    g_dcn = [capture(lambda L=L: step2(d, c, L), stream) for L in sets]
+    g_br = [capture(lambda L=L: step1(d, c, L), stream) for L in sets]
+    torch.cuda.synchronize()
+
+    def run(graphs, n):
+        for i in range(n):
+            graphs[i % R].replay()
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+
+    clk = ClockSampler(local_rank)
+    clk.start()
+    time.sleep(0.3)
+    with torch.cuda.stream(stream):
+        run(g_step, args.warmup)
+    torch.cuda.synchronize()
+
+    # ---------------- timed region: exactly K steps
+    barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t_wall0 = time.time()
+    with torch.cuda.stream(stream):
+        e0.record(stream)
+        run(g_step, args.steps)
+        e1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    t_wall1 = time.time()
+    ms_total = e0.elapsed_time(e1)
+    # keep the GPU busy for clock sampling when the timed region was very short
+    if t_wall1 - t_wall0 < 0.5:
+        t_ext = time.time()
+        with torch.cuda.stream(stream):
+            while time.time() - t_ext < 0.6:
+                run(g_step, 200)
+                torch.cuda.synchronize()
+        t_wall1 = time.time()
+
+    # ---------------- per-kernel timing (same rotation), for the roofline
+    def time_graphs(graphs, n):
+        a, bq = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            run(graphs, 3 * R)
+            a.record(stream)
+            run(graphs, n)
+            bq.record(stream)
+        torch.cuda.synchronize()
+        return a.elapsed_time(bq) / n
+
+    n_k = max(args.steps, 200)
+    ms_dcn = time_graphs(g_dcn, n_k)
+    ms_branch = time_graphs(g_br, n_k)
+    clk.stop()
+    clocks = clk.summary(t_wall0, t_wall1)
+
+    # ---------------- end to end through the C ABI with pinned host buffers
+    ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, K=c.K,
+                                                   stride=c.stride, pad=c.pad, dil=c.dil,
+                                                   offset_groups=c.G, dtype=dt,
+                                                   modulated=c.modulated),
+                     dtype=torch.uint8, device=dev)
+    xh = sets[0].x.cpu().pin_memory()
+    yh = torch.empty(tuple(sets[0].y.shape), dtype=dt).pin_memory()
+    L0 = sets[0]
+    e2e_steps = max(3, min(args.steps, 50))
+    with torch.cuda.stream(stream):
+        for _ in range(2):
+            d.defcon_layer_forward_host(xh, L0.branch, L0.weight, L0.bias, yh, ws, K=c.K,
+                                        stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
+                                        modulated=c.modulated, stream=stream)
+        barrier()
+        a, bq = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(e2e_steps):
+            d.defcon_layer_forward_host(xh, L0.branch, L0.weight, L0.bias, yh, ws, K=c.K,
+                                        stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
+                                        modulated=c.modulated, stream=stream)
+        bq.record(stream)
+    torch.cuda.synchronize()
+    ms_e2e = a.elapsed_time(bq) / e2e_steps
+
+    # ---------------- max over ranks
+    vals = torch.tensor([ms_total, ms_e2e, ms_dcn, ms_branch], dtype=torch.float64, device=dev)
+    if dist is not None:
+        dist.all_reduce(vals, op=dist.ReduceOp.MAX)
+    ms_total, ms_e2e, ms_dcn, ms_branch = [float(v) for v in vals.cpu()]
+
+    flops = configs.contraction_flops(c)
+    ms_step = ms_total / args.steps
+    value = world * flops * args.steps / (ms_total * 1e-3) / 1e12
+    peaks, peak_src = load_peaks()
+    achieved = flops / (ms_dcn * 1e-3) / 1e12
+    traffic = None
+    try:
+        with open(NCU_SUMMARY) as f:
+            traffic = json.load(f).get("dcn_dram_bytes_per_launch")
+    except Exception:
+        pass
+    line = {
+        "metric": metric_name(),
+        "value": round(value, 3),
+        "unit": "TFLOP/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(ms_step, 5),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "bf16",
+        "data": "synthetic (seeded; x=ReLU(N(0,1)) bf16, offsets from the dw offset branch, "
+                "random-init weights)",
+        "config": workload_config(c, world, {
+            "l2": f"rotating {R} buffer sets ({rot_bytes / 2**20:.0f} MiB > 126 MiB L2), CUDA graphs",
+            "us_per_layer": round(ms_step * 1e3, 2),
+            "us_dcn_kernel": round(ms_dcn * 1e3, 2),
+            "us_offset_branch_kernel": round(ms_branch * 1e3, 2),
+        }),
+        "roofline": {
+            "kernel": "dcn_fwd_bf16_tc_kernel (fused gather + tcgen05 implicit GEMM)",
+            "bound": "tensor",
+            "achieved": round(achieved, 2),
+            "peak": peaks["bf16_tflops"],
+            "peak_source": f"{peak_src} bf16 burst (MEASURED_PEAKS.json)" if peak_src == "measured"
+                           else "fallback bf16 burst (B200_PROFILING.md)",
+            "unit": "TFLOP/s",
+            "frac": round(achieved / peaks["bf16_tflops"], 4),
+            "traffic": traffic,
+        },
+        "clocks": clocks,
+        "e2e": {
+            "value": round(world * flops / (ms_e2e * 1e-3) / 1e12, 3),
+            "unit": "TFLOP/s",
+            "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
+            "d2h_bytes_per_step": int(yh.numel() * yh.element_size()),
+            "ms_per_step": round(ms_e2e, 4),
+            "api": "defcon_layer_forward_host (C ABI, pinned host x -> y)",
+        },
+        "gpu_launches": 2 * args.steps,
+    }
+    return line
+
+
+# ------------------------------------------------------------------ oracle (CPU) legs
+def oracle_sample(c, target_s):
+    """Time the oracle as it stands on a bounded sample of the workload: the offset branch
+    of image 0 plus the DCN at `n_pix` output pixels; returns (TFLOP/s, seconds, sample)."""
+    import oracle
+    oracle.build()
+    x = inputs.gen_x(c, images=[0])
+    P = inputs.gen_offset_branch(c)
+    w, b = inputs.gen_weight(c)
+    c1 = c.replace(N=1)
+
+    def once(n_pix):
+        t0 = time.perf_counter()
+        off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
+                                        P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated,
+                                        stride=c.stride, pad=c.pad, dil=c.dil)
+        idx = np.arange(n_pix) % c1.M
+        oracle.dcn_pixels(x, off, w, idx, b, mask=msk, stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+        return time.perf_counter() - t0
+
+    t_cal = once(64)
+    n_pix = int(np.clip(64 * target_s / max(t_cal, 1e-3), 64, 4 * c1.M))
+    dt = once(n_pix)
+    flops = 2 * n_pix * c.Cout * c.K * c.K * c.Cin
+    sample = (f"{c.name}: offset branch of 1 image + DCN at {n_pix} output pixels "
+              f"({flops / 1e9:.2f} GFLOP contraction), fp64")
+    return flops / dt / 1e12, dt, sample, n_pix
+
+
+def cpu_baseline(c):
+    import oracle
+    v, dt, sample, _ = oracle_sample(c, target_s=10.0)
+    return {"value": v, "unit": "TFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": sample, "seconds": round(dt, 2)}
+
+
+def reference_arm(args, world):
+    """--impl reference: the fp64 oracle, as it stands, on the host cores (rank 0 only)."""
+    import oracle
+    c = WORKLOAD
+    per_step_s = 6.0
+    _, _, _, n_pix = oracle_sample(c, target_s=per_step_s)
+    x = inputs.gen_x(c, images=[0])
+    P = inputs.gen_offset_branch(c)
+    w, b = inputs.gen_weight(c)
+
+    def step():
+        off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
+                                        P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated)
+        oracle.dcn_pixels(x, off, w, np.arange(n_pix) % c.replace(N=1).M, b, mask=msk, G=c.G)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = time.perf_counter() - t0
+    flops = 2 * n_pix * c.Cout * c.K * c.K * c.Cin
+    value = flops * args.steps / dt / 1e12
+    sample = (f"{c.name}: per step the offset branch of 1 image + DCN at {n_pix} output pixels, "
+              f"fp64 C oracle with OpenMP")
+    return {
+        "impl": "reference",
+        "metric": metric_name(),
+        "value": value,
+        "unit": "TFLOP/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": dt / args.steps * 1e3,
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f64",
+        "data": "synthetic (seeded)",
+        "config": workload_config(c, world, {"sample": sample}),
+        "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": oracle.num_threads(),
+                         "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=2000)
+    ap.add_argument("--warmup", type=int, default=50)
+    ap.add_argument("--impl", default="defcon", choices=["defcon", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        if rank == 0:
+            print(json.dumps(reference_arm(args, world)), flush=True)
+        return
+
+    dist = None
+    if world > 1:
+        import torch.distributed as tdist
+        torch.cuda.set_device(local_rank)
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        dist = tdist
+    line = gpu_arm(args, rank, world, local_rank, dist)
+    if rank == 0:
+        if not args.no_cpu_baseline and world == 1:
+            line["cpu_baseline"] = cpu_baseline(WORKLOAD)
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

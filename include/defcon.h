@@ -1,0 +1,193 @@
+/*
+ * defcon.h -- C ABI of libdefcon.so, the B200 (sm_100a) implementation of the
+ * DEFCON inference hot path (Jayaweera et al., IPDPSW 2024; /root/reference/PAPER.md).
+ *
+ * The path ("two-step" deformable convolution):
+ *   step 1  defcon_offset_dw_conv  -- the paper's lightweight offset branch
+ *           (P:170 W1 depthwise 3x3 -> P:180 BN + ReLU -> W2 1x1), producing the
+ *           offsets (and the DCNv2 modulation mask, reading R6/R11 in DESIGN.md).
+ *   step 2  defcon_dcn_forward     -- the deformable convolution, Eq.2 with
+ *           the bilinear kernel Eq.3, zero outside the image,
+ *           offset groups, optional DCNv2 mask.
+ *
+ * Conventions (all entry points):
+ *  - Every tensor pointer is a DEVICE pointer owned by the caller unless the
+ *    parameter name ends in _host (pinned host memory, also caller-owned).
+ *    The library never allocates on the call path; its only owned resources are
+ *    texture plans (defcon_tex_plan_create / _destroy).
+ *  - Tensors are dense, row-major, channel-last (NHWC), with the layouts given per
+ *    argument.  Every tensor pointer must be 16-byte aligned (DEFCON_ERR_MISALIGNED).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    Calls are asynchronous on that stream; no host synchronisation happens,
+ *    except in defcon_layer_forward_host (see there).
+ *  - Errors are returned as status codes, never as aborts or exceptions.  All
+ *    argument checks happen before any launch; a failed launch returns
+ *    DEFCON_ERR_CUDA.  defcon_last_error_detail() gives a thread-local message.
+ *    Faults inside a kernel surface at the caller's next synchronisation.
+ *  - There is no CPU fallback and no alternative backend: if the device cannot
+ *    run the sm_100a kernels the call returns DEFCON_ERR_CUDA.
+ *  - Output size: Ho = floor((H + 2*pad_h - dil_h*(Kh-1) - 1) / stride_h) + 1
+ *    ("computed similarly to a regular convolution"), likewise Wo.
+ */
+#ifndef DEFCON_H_
+#define DEFCON_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define DEFCON_ABI_VERSION 1
+
+typedef enum {
+    DEFCON_OK = 0,
+    DEFCON_ERR_INVALID_ARG = 1,  /* shape / enum / pointer argument invalid        */
+    DEFCON_ERR_UNSUPPORTED = 2,  /* valid, but this build has no kernel for it     */
+    DEFCON_ERR_MISALIGNED = 3,   /* a tensor pointer is not 16-byte aligned        */
+    DEFCON_ERR_CUDA = 4,         /* a CUDA runtime call or kernel launch failed    */
+    DEFCON_ERR_LIMIT = 5         /* exceeds an index / texture / workspace limit   */
+} defcon_status_t;
+
+typedef enum {
+    DEFCON_F32 = 0,   /* x, weight, y stored as float32                         */
+    DEFCON_BF16 = 1   /* x, weight, y stored as bfloat16 (fp32 accumulation)    */
+} defcon_dtype_t;
+
+typedef enum {
+    DEFCON_SAMPLER_LDG = 0,  /* software bilinear: vectorised NHWC gathers, fp32 weights */
+    DEFCON_SAMPLER_TEX = 1   /* hardware bilinear: tex2DLayered, border (zero) addressing,
+                                the paper's texel-based optimisation         */
+} defcon_sampler_t;
+
+typedef enum {
+    DEFCON_FP32_3XTF32 = 0,  /* fp32 path on the tensor cores, 3 x TF32 split products  */
+    DEFCON_FP32_SIMT = 1     /* fp32 path on CUDA cores (FFMA), the simple anchor        */
+} defcon_fp32_mode_t;
+
+/* Regular-conv geometry shared by both steps (reading R3) and the number of
+ * offset (deformable) groups G: input channels [g*Cin/G, (g+1)*Cin/G) share
+ * offset field g (reading R5). */
+typedef struct {
+    int stride_h, stride_w;
+    int pad_h, pad_w;
+    int dil_h, dil_w;
+    int offset_groups;
+} defcon_conv_t;
+
+/* Opaque texture plan: owns one layered cudaArray + texture object per image. */
+typedef struct defcon_tex_plan_s* defcon_tex_plan_t;
+
+/*
+ * Step 1 -- lightweight offset branch (Eq.9 P:172 for its cost).
+ *   t[c]  = max(0, dw_scale[c] * sum_{a,b<3} dw_w[c][a][b] * x[n][ho*s-p+a*d][wo*s-p+b*d][c]
+ *                 + dw_shift[c])                  (zero padding; BN folded, R10)
+ *   u[o]  = pw_b[o] + sum_c pw_w[o][c] * t[c]     (o < OC)
+ *   offset[n][ho][wo][g][k][0..1] = u[g*2*K*K + 2*k + {0: dy, 1: dx}]          (R4)
+ *   mask  [n][ho][wo][g][k]       = sigmoid(u[2*G*K*K + g*K*K + k])           (R6, R11)
+ * Arguments
+ *   x        [N][H][W][C], dtype x_dtype
+ *   dw_w     [C][3][3] fp32;  dw_scale, dw_shift [C] fp32 (BN folded with the conv bias)
+ *   pw_w     [OC][C] fp32, OC = G*K*K*(mask ? 3 : 2);  pw_b [OC] fp32 or NULL (= 0)
+ *   K        kernel size of the deformable conv that consumes the offsets (taps K*K)
+ *   cv       stride/pad/dil of the depthwise 3x3 conv (its output grid must be the
+ *            DCN's Ho x Wo, R10) and G = cv.offset_groups
+ *   offset   [N][Ho][Wo][G][K*K][2] fp32 (written)
+ *   mask     [N][Ho][Wo][G][K*K] fp32 (written) or NULL (DCNv1: no mask rows)
+ * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G <= 0; LIMIT if
+ *   OC > 1024 or C > 4096; MISALIGNED for unaligned pointers.
+ */
+int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype,
+                          const float* dw_w, const float* dw_scale, const float* dw_shift,
+                          const float* pw_w, const float* pw_b, int K, defcon_conv_t cv,
+                          float* offset, float* mask, void* stream);
+
+/*
+ * Step 2 -- deformable convolution forward, Eq.2 + Eq.3:
+ *   y[n][ho][wo][co] = bias[co] + sum_{i<Kh, j<Kw, ci<Cin} weight[co][i][j][ci]
+ *                      * m[n][ho][wo][g][k] * X(n, ci, p_y, p_x)
+ *   k = i*Kw + j, g = ci / (Cin/G),
+ *   p_y = ho*stride_h - pad_h + i*dil_h + offset[n][ho][wo][g][k][0]
+ *   p_x = wo*stride_w - pad_w + j*dil_w + offset[n][ho][wo][g][k][1]
+ *   X = bilinear interpolation of channel ci of image n at (p_y, p_x), with the four
+ *       neighbours floor(p)+{0,1}; neighbours outside [0,H)x[0,W) contribute 0
+ *   m = mask, or 1 when mask == NULL (DCNv1)
+ * Arguments
+ *   x        [N][H][W][Cin], dtype `dtype`
+ *   offset   [N][Ho][Wo][G][Kh*Kw][2] fp32 (dy, dx);  mask [N][Ho][Wo][G][Kh*Kw] fp32 or NULL
+ *   weight   [Cout][Kh][Kw][Cin], dtype `dtype`;  bias [Cout] fp32 or NULL (= 0)
+ *   sampler  DEFCON_SAMPLER_LDG (any dtype) or DEFCON_SAMPLER_TEX (requires tex_plan made
+ *            for the same N, H, W, Cin, dtype; the plan's array is (re)filled from x on
+ *            `stream` by this call)
+ *   fp32_mode  used only when dtype == DEFCON_F32
+ *   y        [N][Ho][Wo][Cout], dtype `dtype` (written)
+ *   workspace / workspace_bytes: device scratch of at least defcon_dcn_workspace_size()
+ *            bytes (may be NULL when that size is 0)
+ * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G not dividing Cin, bad enums,
+ *   NULL required pointers; UNSUPPORTED for (Cin/G) % 8 != 0 (bf16) or % 4 != 0 (fp32),
+ *   or a Cout not multiple of 16 on the tensor-core paths; LIMIT when N*H*W*Cin >= 2^31
+ *   or the workspace is too small; MISALIGNED for unaligned pointers.
+ */
+int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin,
+                       const float* offset, const float* mask,
+                       const void* weight, const float* bias, int Cout, int Kh, int Kw,
+                       defcon_conv_t cv, int dtype, int sampler, int fp32_mode,
+                       void* y, void* workspace, size_t workspace_bytes,
+                       defcon_tex_plan_t tex_plan, void* stream);
+
+/* Device workspace defcon_dcn_forward needs for these arguments (0 if none). */
+int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
+                              defcon_conv_t cv, int dtype, int sampler, int fp32_mode,
+                              size_t* bytes);
+
+/*
+ * Whole layer with HOST buffers (the end-to-end entry point): copies x_host (pinned)
+ * to the device, runs step 1 and step 2 on `stream`, copies y back to y_host and
+ * synchronises `stream` before returning.  Parameters dw_* / pw_* / weight / bias are
+ * device pointers (resident model weights), as in the two calls above.
+ * dev_workspace must hold defcon_layer_workspace_size() bytes (x, offsets, mask, y and
+ * the step-2 workspace are carved out of it).  modulated != 0 selects DCNv2.
+ */
+int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, int dtype,
+                              const float* dw_w, const float* dw_scale, const float* dw_shift,
+                              const float* pw_w, const float* pw_b,
+                              const void* weight, const float* bias, int Cout, int K,
+                              defcon_conv_t cv, int modulated, int sampler, int fp32_mode,
+                              void* y_host, void* dev_workspace, size_t dev_workspace_bytes,
+                              void* stream);
+
+int defcon_layer_workspace_size(int N, int H, int W, int Cin, int dtype, int Cout, int K,
+                                defcon_conv_t cv, int modulated, int sampler, int fp32_mode,
+                                size_t* bytes);
+
+/*
+ * Texture plan for DEFCON_SAMPLER_TEX: one 2-D layered cudaArray per image
+ * (one layer per 4 channels, half4 texels for bf16 input and float4 texels for fp32;
+ * H x W texels per layer) with a texture object using border (zero) addressing,
+ * linear filtering and unnormalised coordinates.  One object per image keeps the
+ * layer count at Cin/4 per object, inside the 2048-layer limit the paper notes.
+ * Errors: INVALID_ARG for bad sizes, UNSUPPORTED for Cin % 4 != 0, LIMIT for
+ * Cin/4 > device max layers or H, W above the layered-texture limits, CUDA on
+ * allocation failure.  destroy(NULL) is a no-op returning DEFCON_OK.
+ */
+int defcon_tex_plan_create(int N, int H, int W, int Cin, int dtype, defcon_tex_plan_t* plan);
+int defcon_tex_plan_destroy(defcon_tex_plan_t plan);
+
+/*
+ * Texture-filter probe (measures the reading R14 on the device): samples a single
+ * 2 x 2 float texel layer [[0, 0], [0, 1]] (border addressing, linear filter) at
+ * the n coordinates (px[i], py[i]) given in texel units (no +0.5 applied), writing
+ * the filtered values to out[i].  px, py, out are device fp32 arrays of length n.
+ */
+int defcon_tex_filter_probe(const float* px, const float* py, float* out, int n, void* stream);
+
+const char* defcon_status_string(int status);
+const char* defcon_last_error_detail(void);   /* thread-local, "" if none */
+int defcon_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* DEFCON_H_ */

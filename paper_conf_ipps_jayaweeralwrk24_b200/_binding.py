@@ -1,0 +1,281 @@
+"""Thin ctypes binding over libdefcon.so (include/defcon.h): same entry-point names,
+argument marshalling only.  Every step of the hot path runs in the library's CUDA
+kernels; there is no CPU fallback -- if the library is missing or the device cannot
+run it, these functions raise.
+
+Tensors are torch CUDA tensors (torch is used for device memory and streams only).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libdefcon.so")
+
+DEFCON_OK, DEFCON_ERR_INVALID_ARG, DEFCON_ERR_UNSUPPORTED, DEFCON_ERR_MISALIGNED, \
+    DEFCON_ERR_CUDA, DEFCON_ERR_LIMIT = range(6)
+DEFCON_F32, DEFCON_BF16 = 0, 1
+DEFCON_SAMPLER_LDG, DEFCON_SAMPLER_TEX = 0, 1
+DEFCON_FP32_3XTF32, DEFCON_FP32_SIMT = 0, 1
+
+# Every symbol include/defcon.h declares (checked by tests/test_abi.py).
+EXPORTED = (
+    "defcon_offset_dw_conv", "defcon_dcn_forward", "defcon_dcn_workspace_size",
+    "defcon_layer_forward_host", "defcon_layer_workspace_size", "defcon_tex_plan_create",
+    "defcon_tex_plan_destroy", "defcon_tex_filter_probe", "defcon_status_string",
+    "defcon_last_error_detail", "defcon_abi_version",
+)
+
+_DTYPES = {torch.float32: DEFCON_F32, torch.bfloat16: DEFCON_BF16}
+_SAMPLERS = {"ldg": DEFCON_SAMPLER_LDG, "tex": DEFCON_SAMPLER_TEX}
+_FP32_MODES = {"3xtf32": DEFCON_FP32_3XTF32, "simt": DEFCON_FP32_SIMT}
+
+
+class DefconError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        self.status = status
+        super().__init__(f"{where}: {_status_name(status)} ({detail})")
+
+
+class defcon_conv_t(ctypes.Structure):
+    _fields_ = [("stride_h", ctypes.c_int), ("stride_w", ctypes.c_int),
+                ("pad_h", ctypes.c_int), ("pad_w", ctypes.c_int),
+                ("dil_h", ctypes.c_int), ("dil_w", ctypes.c_int),
+                ("offset_groups", ctypes.c_int)]
+
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Load libdefcon.so; raises if it has not been built (no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise RuntimeError(f"{path} not built: run `python -m paper_conf_ipps_jayaweeralwrk24_b200.build`"
+                           " (or __graft_entry__.build())")
+    lib = ctypes.CDLL(path)
+    vp, fp, i, sz = ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_size_t
+    conv = defcon_conv_t
+    lib.defcon_offset_dw_conv.argtypes = [vp, i, i, i, i, i, fp, fp, fp, fp, fp, i, conv, fp, fp, vp]
+    lib.defcon_dcn_forward.argtypes = [vp, i, i, i, i, fp, fp, vp, fp, i, i, i, conv, i, i, i, vp, vp,
+                                       sz, vp, vp]
+    lib.defcon_dcn_workspace_size.argtypes = [i, i, i, i, i, i, i, conv, i, i, i,
+                                              ctypes.POINTER(sz)]
+    lib.defcon_layer_forward_host.argtypes = [vp, i, i, i, i, i, fp, fp, fp, fp, fp, vp, fp, i, i,
+                                              conv, i, i, i, vp, vp, sz, vp]
+    lib.defcon_layer_workspace_size.argtypes = [i, i, i, i, i, i, i, conv, i, i, i,
+                                                ctypes.POINTER(sz)]
+    lib.defcon_tex_plan_create.argtypes = [i, i, i, i, i, ctypes.POINTER(vp)]
+    lib.defcon_tex_plan_destroy.argtypes = [vp]
+    lib.defcon_tex_filter_probe.argtypes = [fp, fp, fp, i, vp]
+    lib.defcon_status_string.argtypes = [i]
+    lib.defcon_status_string.restype = ctypes.c_char_p
+    lib.defcon_last_error_detail.restype = ctypes.c_char_p
+    for name in EXPORTED:
+        if name not in ("defcon_status_string", "defcon_last_error_detail"):
+            getattr(lib, name).restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+def _status_name(status: int) -> str:
+    try:
+        return load_library().defcon_status_string(status).decode()
+    except Exception:
+        return str(status)
+
+
+def _check(rc: int, where: str):
+    if rc != DEFCON_OK:
+        raise DefconError(rc, where, load_library().defcon_last_error_detail().decode())
+
+
+def _conv(stride, pad, dil, groups) -> defcon_conv_t:
+    s = (stride, stride) if isinstance(stride, int) else tuple(stride)
+    p = (pad, pad) if isinstance(pad, int) else tuple(pad)
+    d = (dil, dil) if isinstance(dil, int) else tuple(dil)
+    return defcon_conv_t(s[0], s[1], p[0], p[1], d[0], d[1], int(groups))
+
+
+def _out(n, k, s, p, d):
+    span = n + 2 * p - d * (k - 1) - 1
+    return 0 if span < 0 else span // s + 1
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _dev_tensor(t, name, dtype=None, shape=None, allow_none=False):
+    if t is None:
+        if allow_none:
+            return
+        raise ValueError(f"{name} is required")
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if dtype is not None and t.dtype != dtype:
+        raise ValueError(f"{name} must be {dtype}, got {t.dtype}")
+    if shape is not None and tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name} shape {tuple(t.shape)} != {tuple(shape)}")
+
+
+def _stream_handle(stream):
+    s = torch.cuda.current_stream() if stream is None else stream
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, stride=1, pad=1,
+                          dil=1, offset_groups=1, with_mask=True, offset=None, mask=None,
+                          stream=None):
+    """Step 1: lightweight offset branch.  Returns (offset, mask|None)."""
+    lib = load_library()
+    _dev_tensor(x, "x")
+    if x.dtype not in _DTYPES:
+        raise ValueError("x must be float32 or bfloat16")
+    N, H, W, C = x.shape
+    cv = _conv(stride, pad, dil, offset_groups)
+    Ho, Wo = _out(H, 3, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, 3, cv.stride_w, cv.pad_w, cv.dil_w)
+    G, KK = int(offset_groups), K * K
+    OC = G * KK * (3 if with_mask else 2)
+    _dev_tensor(dw_w, "dw_w", torch.float32, (C, 3, 3))
+    _dev_tensor(dw_scale, "dw_scale", torch.float32, (C,))
+    _dev_tensor(dw_shift, "dw_shift", torch.float32, (C,))
+    _dev_tensor(pw_w, "pw_w", torch.float32, (OC, C))
+    _dev_tensor(pw_b, "pw_b", torch.float32, (OC,), allow_none=True)
+    if offset is None:
+        offset = torch.empty((N, Ho, Wo, G, KK, 2), device=x.device, dtype=torch.float32)
+    _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, KK, 2))
+    if with_mask:
+        if mask is None:
+            mask = torch.empty((N, Ho, Wo, G, KK), device=x.device, dtype=torch.float32)
+        _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, KK))
+    else:
+        mask = None
+    rc = lib.defcon_offset_dw_conv(_ptr(x), N, H, W, C, _DTYPES[x.dtype], _ptr(dw_w), _ptr(dw_scale),
+                                   _ptr(dw_shift), _ptr(pw_w), _ptr(pw_b), K, cv, _ptr(offset),
+                                   _ptr(mask), _stream_handle(stream))
+    _check(rc, "defcon_offset_dw_conv")
+    return offset, mask
+
+
+def defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw, stride=1, pad=1, dil=1, offset_groups=1,
+                              dtype=torch.bfloat16, sampler="ldg", fp32_mode="simt") -> int:
+    lib = load_library()
+    out = ctypes.c_size_t(0)
+    rc = lib.defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw,
+                                       _conv(stride, pad, dil, offset_groups), _DTYPES[dtype],
+                                       _SAMPLERS[sampler], _FP32_MODES[fp32_mode], ctypes.byref(out))
+    _check(rc, "defcon_dcn_workspace_size")
+    return int(out.value)
+
+
+def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=1, offset_groups=1,
+                       sampler="ldg", fp32_mode="simt", y=None, workspace=None, tex_plan=None,
+                       stream=None):
+    """Step 2 (Eq.2 P:58 + Eq.3): deformable conv forward, NHWC.  Returns y."""
+    lib = load_library()
+    _dev_tensor(x, "x")
+    if x.dtype not in _DTYPES:
+        raise ValueError("x must be float32 or bfloat16")
+    N, H, W, Cin = x.shape
+    _dev_tensor(weight, "weight", x.dtype)
+    Cout, Kh, Kw, Cw = weight.shape
+    if Cw != Cin:
+        raise ValueError("weight Cin mismatch")
+    cv = _conv(stride, pad, dil, offset_groups)
+    Ho, Wo = _out(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w)
+    G = int(offset_groups)
+    _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
+    _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
+    _dev_tensor(bias, "bias", torch.float32, (Cout,), allow_none=True)
+    if y is None:
+        y = torch.empty((N, Ho, Wo, Cout), device=x.device, dtype=x.dtype)
+    _dev_tensor(y, "y", x.dtype, (N, Ho, Wo, Cout))
+    ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
+    plan = None if tex_plan is None else tex_plan.handle
+    rc = lib.defcon_dcn_forward(_ptr(x), N, H, W, Cin, _ptr(offset), _ptr(mask), _ptr(weight),
+                                _ptr(bias), Cout, Kh, Kw, cv, _DTYPES[x.dtype], _SAMPLERS[sampler],
+                                _FP32_MODES[fp32_mode], _ptr(y), _ptr(workspace), ws_bytes, plan,
+                                _stream_handle(stream))
+    _check(rc, "defcon_dcn_forward")
+    return y
+
+
+def defcon_layer_workspace_size(N, H, W, Cin, Cout, K=3, stride=1, pad=1, dil=1, offset_groups=1,
+                                dtype=torch.bfloat16, modulated=True, sampler="ldg",
+                                fp32_mode="simt") -> int:
+    lib = load_library()
+    out = ctypes.c_size_t(0)
+    rc = lib.defcon_layer_workspace_size(N, H, W, Cin, _DTYPES[dtype], Cout, K,
+                                         _conv(stride, pad, dil, offset_groups), int(modulated),
+                                         _SAMPLERS[sampler], _FP32_MODES[fp32_mode],
+                                         ctypes.byref(out))
+    _check(rc, "defcon_layer_workspace_size")
+    return int(out.value)
+
+
+def defcon_layer_forward_host(x_host, branch, weight, bias, y_host, dev_workspace, K=3, stride=1,
+                              pad=1, dil=1, offset_groups=1, modulated=True, sampler="ldg",
+                              fp32_mode="simt", stream=None):
+    """Whole layer from pinned host x to pinned host y (H2D, step 1, step 2, D2H, sync).
+
+    branch: dict of device tensors dw_w, dw_scale, dw_shift, pw_w, pw_b (resident weights).
+    """
+    lib = load_library()
+    if x_host.is_cuda or y_host.is_cuda:
+        raise ValueError("x_host / y_host must be host tensors (pinned)")
+    N, H, W, Cin = x_host.shape
+    Cout = weight.shape[0]
+    rc = lib.defcon_layer_forward_host(
+        _ptr(x_host), N, H, W, Cin, _DTYPES[x_host.dtype], _ptr(branch["dw_w"]),
+        _ptr(branch["dw_scale"]), _ptr(branch["dw_shift"]), _ptr(branch["pw_w"]),
+        _ptr(branch.get("pw_b")), _ptr(weight), _ptr(bias), Cout, K,
+        _conv(stride, pad, dil, offset_groups), int(modulated), _SAMPLERS[sampler],
+        _FP32_MODES[fp32_mode], _ptr(y_host), _ptr(dev_workspace),
+        dev_workspace.numel() * dev_workspace.element_size(), _stream_handle(stream))
+    _check(rc, "defcon_layer_forward_host")
+    return y_host
+
+
+class TexPlan:
+    """Owns a libdefcon texture plan (layered cudaArray + texture object per image)."""
+
+    def __init__(self, N, H, W, Cin, dtype=torch.bfloat16):
+        lib = load_library()
+        h = ctypes.c_void_p()
+        _check(lib.defcon_tex_plan_create(N, H, W, Cin, _DTYPES[dtype], ctypes.byref(h)),
+               "defcon_tex_plan_create")
+        self.handle = h
+
+    def close(self):
+        if self.handle is not None and self.handle.value:
+            load_library().defcon_tex_plan_destroy(self.handle)
+        self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def defcon_tex_filter_probe(px, py, out=None, stream=None):
+    lib = load_library()
+    _dev_tensor(px, "px", torch.float32)
+    _dev_tensor(py, "py", torch.float32, tuple(px.shape))
+    if out is None:
+        out = torch.empty_like(px)
+    rc = lib.defcon_tex_filter_probe(_ptr(px), _ptr(py), _ptr(out), px.numel(), _stream_handle(stream))
+    _check(rc, "defcon_tex_filter_probe")
+    return out
+
+
+def defcon_abi_version() -> int:
+    return int(load_library().defcon_abi_version())

@@ -1,0 +1,306 @@
+// api.cu -- the extern "C" boundary of libdefcon.so (declared in include/defcon.h):
+// argument validation, kernel selection and launch, workspace sizing and the
+// host-buffer end-to-end entry point.  No allocation on the call path, no host sync
+// (except defcon_layer_forward_host), no CPU fallback.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+
+#include "../../include/defcon.h"
+#include "common.cuh"
+#include "kernels.h"
+
+namespace defcon {
+
+static thread_local char g_detail[512] = "";
+
+static int fail(int status, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_detail, sizeof(g_detail), fmt, ap);
+    va_end(ap);
+    return status;
+}
+
+static int cuda_fail(cudaError_t e, const char* what) {
+    return fail(DEFCON_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+static int out_size(int in, int k, int stride, int pad, int dil) {
+    const long span = (long)in + 2L * pad - (long)dil * (k - 1) - 1;
+    if (span < 0 || stride <= 0) return 0;
+    return (int)(span / stride + 1);
+}
+
+PFN_encodeTiled get_encode_tiled() {
+    static PFN_encodeTiled fn = nullptr;
+    static bool tried = false;
+    if (!tried) {
+        tried = true;
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
+                cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_encodeTiled>(p);
+    }
+    return fn;
+}
+
+// Shared validation of the conv geometry.
+static int check_conv(const defcon_conv_t& cv) {
+    if (cv.stride_h <= 0 || cv.stride_w <= 0 || cv.dil_h <= 0 || cv.dil_w <= 0)
+        return fail(DEFCON_ERR_INVALID_ARG, "stride and dilation must be positive");
+    if (cv.pad_h < 0 || cv.pad_w < 0) return fail(DEFCON_ERR_INVALID_ARG, "padding must be >= 0");
+    if (cv.offset_groups <= 0) return fail(DEFCON_ERR_INVALID_ARG, "offset_groups must be > 0");
+    return DEFCON_OK;
+}
+
+static int make_geom(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
+                     const defcon_conv_t& cv, int dtype, DcnGeom* g) {
+    if (N <= 0 || H <= 0 || W <= 0 || Cin <= 0 || Cout <= 0 || Kh <= 0 || Kw <= 0)
+        return fail(DEFCON_ERR_INVALID_ARG, "sizes must be positive");
+    int rc = check_conv(cv);
+    if (rc) return rc;
+    if (dtype != DEFCON_F32 && dtype != DEFCON_BF16) return fail(DEFCON_ERR_INVALID_ARG, "bad dtype");
+    if (Cin % cv.offset_groups != 0)
+        return fail(DEFCON_ERR_INVALID_ARG, "offset_groups (%d) must divide Cin (%d)", cv.offset_groups, Cin);
+    g->N = N; g->H = H; g->W = W; g->Cin = Cin; g->Cout = Cout; g->Kh = Kh; g->Kw = Kw;
+    g->Ho = out_size(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h);
+    g->Wo = out_size(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w);
+    if (g->Ho <= 0 || g->Wo <= 0) return fail(DEFCON_ERR_INVALID_ARG, "output grid is empty");
+    g->sh = cv.stride_h; g->sw = cv.stride_w; g->ph = cv.pad_h; g->pw = cv.pad_w;
+    g->dh = cv.dil_h; g->dw = cv.dil_w;
+    g->G = cv.offset_groups;
+    g->Cg = Cin / cv.offset_groups;
+    g->KK = Kh * Kw;
+    const long M = (long)N * g->Ho * g->Wo;
+    if ((long)N * H * W * Cin >= (1L << 31) || M * Cout >= (1L << 31) ||
+        M * g->G * g->KK * 2 >= (1L << 31) || (long)Cout * g->KK * Cin >= (1L << 31))
+        return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
+    g->M = (int)M;
+    const int vec = dtype == DEFCON_BF16 ? 8 : 4;
+    if (g->Cg % vec != 0)
+        return fail(DEFCON_ERR_UNSUPPORTED, "Cin/G = %d must be a multiple of %d for this dtype",
+                    g->Cg, vec);
+    return DEFCON_OK;
+}
+
+enum class Path { SIMT_F32, SIMT_BF16, TC_BF16 };
+
+static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, Path* path) {
+    if (sampler != DEFCON_SAMPLER_LDG && sampler != DEFCON_SAMPLER_TEX)
+        return fail(DEFCON_ERR_INVALID_ARG, "bad sampler");
+    if (fp32_mode != DEFCON_FP32_3XTF32 && fp32_mode != DEFCON_FP32_SIMT)
+        return fail(DEFCON_ERR_INVALID_ARG, "bad fp32_mode");
+    if (sampler == DEFCON_SAMPLER_TEX)
+        return fail(DEFCON_ERR_UNSUPPORTED, "texture sampler not built in this version");
+    if (dtype == DEFCON_BF16) {
+        *path = dcn_tc_bf16_supported(g) ? Path::TC_BF16 : Path::SIMT_BF16;
+    } else {
+        if (fp32_mode == DEFCON_FP32_3XTF32)
+            return fail(DEFCON_ERR_UNSUPPORTED, "3xTF32 fp32 path not built in this version");
+        *path = Path::SIMT_F32;
+    }
+    return DEFCON_OK;
+}
+
+}  // namespace defcon
+
+using namespace defcon;
+
+extern "C" {
+
+const char* defcon_status_string(int status) {
+    switch (status) {
+        case DEFCON_OK: return "DEFCON_OK";
+        case DEFCON_ERR_INVALID_ARG: return "DEFCON_ERR_INVALID_ARG";
+        case DEFCON_ERR_UNSUPPORTED: return "DEFCON_ERR_UNSUPPORTED";
+        case DEFCON_ERR_MISALIGNED: return "DEFCON_ERR_MISALIGNED";
+        case DEFCON_ERR_CUDA: return "DEFCON_ERR_CUDA";
+        case DEFCON_ERR_LIMIT: return "DEFCON_ERR_LIMIT";
+        default: return "DEFCON_ERR_UNKNOWN";
+    }
+}
+
+const char* defcon_last_error_detail(void) { return g_detail; }
+
+int defcon_abi_version(void) { return DEFCON_ABI_VERSION; }
+
+int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype,
+                          const float* dw_w, const float* dw_scale, const float* dw_shift,
+                          const float* pw_w, const float* pw_b, int K, defcon_conv_t cv,
+                          float* offset, float* mask, void* stream) {
+    g_detail[0] = 0;
+    if (N <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0)
+        return fail(DEFCON_ERR_INVALID_ARG, "sizes must be positive");
+    int rc = check_conv(cv);
+    if (rc) return rc;
+    if (x_dtype != DEFCON_F32 && x_dtype != DEFCON_BF16) return fail(DEFCON_ERR_INVALID_ARG, "bad dtype");
+    if (!x || !dw_w || !dw_scale || !dw_shift || !pw_w || !offset)
+        return fail(DEFCON_ERR_INVALID_ARG, "NULL tensor pointer");
+    const void* ptrs[] = {x, dw_w, dw_scale, dw_shift, pw_w, pw_b, offset, mask};
+    for (const void* p : ptrs)
+        if (p && !aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "tensor pointer not 16-byte aligned");
+    const int Ho = out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h);
+    const int Wo = out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w);
+    if (Ho <= 0 || Wo <= 0) return fail(DEFCON_ERR_INVALID_ARG, "output grid is empty");
+    const int G = cv.offset_groups;
+    const int OC = G * K * K * (mask ? 3 : 2);
+    if (OC > 512) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 512", OC);
+    if ((long)N * H * W * C >= (1L << 31) || (long)N * Ho * Wo * OC >= (1L << 31))
+        return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
+    cudaError_t e = launch_offset_branch(x, x_dtype == DEFCON_BF16, N, H, W, C, dw_w, dw_scale,
+                                         dw_shift, pw_w, pw_b, K, G, mask != nullptr, cv.stride_h,
+                                         cv.stride_w, cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, Ho, Wo,
+                                         offset, mask, static_cast<cudaStream_t>(stream));
+    if (e == cudaErrorInvalidValue)
+        return fail(DEFCON_ERR_LIMIT, "offset branch: C = %d needs more shared memory than available", C);
+    if (e != cudaSuccess) return cuda_fail(e, "offset_branch launch");
+    return DEFCON_OK;
+}
+
+int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
+                              defcon_conv_t cv, int dtype, int sampler, int fp32_mode,
+                              size_t* bytes) {
+    g_detail[0] = 0;
+    if (!bytes) return fail(DEFCON_ERR_INVALID_ARG, "bytes is NULL");
+    DcnGeom g;
+    int rc = make_geom(N, H, W, Cin, Cout, Kh, Kw, cv, dtype, &g);
+    if (rc) return rc;
+    Path path;
+    rc = select_path(g, dtype, sampler, fp32_mode, &path);
+    if (rc) return rc;
+    *bytes = 0;
+    return DEFCON_OK;
+}
+
+int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float* offset,
+                       const float* mask, const void* weight, const float* bias, int Cout, int Kh,
+                       int Kw, defcon_conv_t cv, int dtype, int sampler, int fp32_mode, void* y,
+                       void* workspace, size_t workspace_bytes, defcon_tex_plan_t tex_plan,
+                       void* stream) {
+    g_detail[0] = 0;
+    DcnGeom g;
+    int rc = make_geom(N, H, W, Cin, Cout, Kh, Kw, cv, dtype, &g);
+    if (rc) return rc;
+    if (!x || !offset || !weight || !y) return fail(DEFCON_ERR_INVALID_ARG, "NULL tensor pointer");
+    const void* ptrs[] = {x, offset, mask, weight, bias, y, workspace};
+    for (const void* p : ptrs)
+        if (p && !aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "tensor pointer not 16-byte aligned");
+    Path path;
+    rc = select_path(g, dtype, sampler, fp32_mode, &path);
+    if (rc) return rc;
+    (void)tex_plan;
+    (void)workspace_bytes;
+    DcnPtrs p{x, offset, mask, weight, bias, y};
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaError_t e;
+    const char* detail = "dcn launch";
+    switch (path) {
+        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, st, &detail); break;
+        case Path::SIMT_BF16: e = launch_dcn_simt(g, p, true, st); break;
+        default: e = launch_dcn_simt(g, p, false, st); break;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, detail);
+    return DEFCON_OK;
+}
+
+// ---------------------------------------------------------------- end-to-end host entry
+static size_t align_up(size_t v) { return (v + 255) & ~size_t(255); }
+
+struct LayerCarve {
+    size_t x, off, msk, y, ws, total;
+};
+
+static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
+                       const defcon_conv_t& cv, int modulated, int sampler, int fp32_mode,
+                       DcnGeom* g, LayerCarve* c) {
+    int rc = make_geom(N, H, W, Cin, Cout, K, K, cv, dtype, g);
+    if (rc) return rc;
+    Path path;
+    rc = select_path(*g, dtype, sampler, fp32_mode, &path);
+    if (rc) return rc;
+    const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
+    c->x = align_up((size_t)N * H * W * Cin * es);
+    c->off = align_up((size_t)g->M * g->G * g->KK * 2 * sizeof(float));
+    c->msk = modulated ? align_up((size_t)g->M * g->G * g->KK * sizeof(float)) : 0;
+    c->y = align_up((size_t)g->M * Cout * es);
+    c->ws = 0;
+    c->total = c->x + c->off + c->msk + c->y + c->ws;
+    return DEFCON_OK;
+}
+
+int defcon_layer_workspace_size(int N, int H, int W, int Cin, int dtype, int Cout, int K,
+                                defcon_conv_t cv, int modulated, int sampler, int fp32_mode,
+                                size_t* bytes) {
+    g_detail[0] = 0;
+    if (!bytes) return fail(DEFCON_ERR_INVALID_ARG, "bytes is NULL");
+    DcnGeom g;
+    LayerCarve c;
+    int rc = layer_carve(N, H, W, Cin, dtype, Cout, K, cv, modulated, sampler, fp32_mode, &g, &c);
+    if (rc) return rc;
+    *bytes = c.total;
+    return DEFCON_OK;
+}
+
+int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, int dtype,
+                              const float* dw_w, const float* dw_scale, const float* dw_shift,
+                              const float* pw_w, const float* pw_b, const void* weight,
+                              const float* bias, int Cout, int K, defcon_conv_t cv, int modulated,
+                              int sampler, int fp32_mode, void* y_host, void* dev_workspace,
+                              size_t dev_workspace_bytes, void* stream) {
+    g_detail[0] = 0;
+    if (!x_host || !y_host || !dev_workspace) return fail(DEFCON_ERR_INVALID_ARG, "NULL pointer");
+    DcnGeom g;
+    LayerCarve c;
+    int rc = layer_carve(N, H, W, Cin, dtype, Cout, K, cv, modulated, sampler, fp32_mode, &g, &c);
+    if (rc) return rc;
+    if (dev_workspace_bytes < c.total)
+        return fail(DEFCON_ERR_LIMIT, "device workspace %zu < required %zu", dev_workspace_bytes, c.total);
+    uint8_t* base = static_cast<uint8_t*>(dev_workspace);
+    void* xd = base;
+    float* offd = reinterpret_cast<float*>(base + c.x);
+    float* mskd = modulated ? reinterpret_cast<float*>(base + c.x + c.off) : nullptr;
+    void* yd = base + c.x + c.off + c.msk;
+    void* wsd = c.ws ? base + c.x + c.off + c.msk + c.y : nullptr;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
+    cudaError_t e = cudaMemcpyAsync(xd, x_host, (size_t)N * H * W * Cin * es, cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return cuda_fail(e, "H2D copy of x");
+    rc = defcon_offset_dw_conv(xd, N, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
+                               offd, mskd, stream);
+    if (rc) return rc;
+    if (out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h) != g.Ho ||
+        out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w) != g.Wo)
+        return fail(DEFCON_ERR_INVALID_ARG, "offset-branch grid differs from the DCN grid");
+    rc = defcon_dcn_forward(xd, N, H, W, Cin, offd, mskd, weight, bias, Cout, K, K, cv, dtype,
+                            sampler, fp32_mode, yd, wsd, c.ws, nullptr, stream);
+    if (rc) return rc;
+    e = cudaMemcpyAsync(y_host, yd, (size_t)g.M * Cout * es, cudaMemcpyDeviceToHost, st);
+    if (e != cudaSuccess) return cuda_fail(e, "D2H copy of y");
+    e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_fail(e, "stream synchronize");
+    return DEFCON_OK;
+}
+
+int defcon_tex_plan_create(int N, int H, int W, int Cin, int dtype, defcon_tex_plan_t* plan) {
+    g_detail[0] = 0;
+    (void)N; (void)H; (void)W; (void)Cin; (void)dtype;
+    if (plan) *plan = nullptr;
+    return fail(DEFCON_ERR_UNSUPPORTED, "texture sampler not built in this version");
+}
+
+int defcon_tex_plan_destroy(defcon_tex_plan_t plan) {
+    (void)plan;
+    return DEFCON_OK;
+}
+
+int defcon_tex_filter_probe(const float* px, const float* py, float* out, int n, void* stream) {
+    (void)px; (void)py; (void)out; (void)n; (void)stream;
+    return fail(DEFCON_ERR_UNSUPPORTED, "texture sampler not built in this version");
+}
+
+}  // extern "C"

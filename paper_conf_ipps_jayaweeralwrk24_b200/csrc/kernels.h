@@ -1,0 +1,52 @@
+// kernels.h -- internal host-side launch interface between api.cu and the
+// kernel translation units.  Not part of the public C ABI (include/defcon.h).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+namespace defcon {
+
+// Geometry of one deformable-conv launch (all validated by api.cu).
+struct DcnGeom {
+    int N, H, W, Cin, Cout, Kh, Kw, Ho, Wo;
+    int sh, sw, ph, pw, dh, dw;
+    int G, Cg;   // offset groups, channels per group
+    int M;       // N * Ho * Wo output pixels
+    int KK;      // Kh * Kw taps
+};
+
+struct DcnPtrs {
+    const void* x;
+    const float* offset;
+    const float* mask;   // nullptr => DCNv1
+    const void* weight;
+    const float* bias;   // nullptr => 0
+    void* y;
+};
+
+// ---- step 1: lightweight offset branch (offset_branch.cu)
+cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W, int C,
+                                 const float* dw_w, const float* dw_scale, const float* dw_shift,
+                                 const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
+                                 int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
+                                 float* offset, float* mask, cudaStream_t stream);
+
+// ---- step 2, CUDA-core anchor (dcn_simt.cu): fp32 math for fp32 or bf16 storage
+cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaStream_t stream);
+
+// ---- step 2, fused gather + tcgen05 implicit GEMM, bf16 (dcn_tc_bf16.cu)
+bool dcn_tc_bf16_supported(const DcnGeom& g);
+cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, cudaStream_t stream,
+                               const char** detail);
+
+// ---- driver entry point for cuTensorMapEncodeTiled (api.cu)
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                    const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                    const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                    CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+PFN_encodeTiled get_encode_tiled();
+
+}  // namespace defcon

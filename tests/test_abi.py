@@ -1,0 +1,126 @@
+"""C-ABI contract tests that need no GPU (tier T1).
+
+The library is built (nvcc cross-compiles sm_100a here) and loaded; every symbol
+include/defcon.h declares must be exported, and invalid arguments must come back as
+the documented status codes *before* any CUDA call (fake device pointers are fine).
+"""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_ipps_jayaweeralwrk24_b200 import build, _binding
+    build.build()
+    return _binding.load_library()
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "defcon.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(defcon_[a-z0-9_]+)\s*\(", txt)))
+
+
+def test_header_symbols_exported(lib):
+    from paper_conf_ipps_jayaweeralwrk24_b200 import _binding
+    syms = header_symbols()
+    assert len(syms) >= 11
+    for s in syms:
+        assert hasattr(lib, s), s
+    assert sorted(_binding.EXPORTED) == syms
+
+
+def test_status_strings(lib):
+    assert lib.defcon_abi_version() == 1
+    assert lib.defcon_status_string(0) == b"DEFCON_OK"
+    assert lib.defcon_status_string(5) == b"DEFCON_ERR_LIMIT"
+
+
+def _conv(**kw):
+    from paper_conf_ipps_jayaweeralwrk24_b200._binding import defcon_conv_t
+    d = dict(stride_h=1, stride_w=1, pad_h=1, pad_w=1, dil_h=1, dil_w=1, offset_groups=1)
+    d.update(kw)
+    return defcon_conv_t(**d)
+
+
+FAKE = 0x7F0000000000   # 16-byte aligned fake device address; never dereferenced
+
+
+def _fwd(lib, x=FAKE, N=2, H=8, W=8, Cin=64, off=FAKE, mask=FAKE, w=FAKE, b=FAKE, Cout=64, K=3,
+         cv=None, dtype=1, sampler=0, fp32_mode=1, y=FAKE):
+    cv = cv or _conv()
+    V = ctypes.c_void_p
+    return lib.defcon_dcn_forward(V(x), N, H, W, Cin, V(off), V(mask), V(w), V(b), Cout, K, K, cv,
+                                  dtype, sampler, fp32_mode, V(y), None, 0, None, None)
+
+
+@pytest.mark.parametrize("kw,status", [
+    (dict(N=0), 1), (dict(H=-1), 1), (dict(Cout=0), 1),
+    (dict(cv="g3"), 1),                   # G does not divide Cin
+    (dict(cv="s0"), 1),                   # zero stride
+    (dict(cv="tiny"), 1),                 # empty output grid (H=1, pad 0, K=3)
+    (dict(dtype=7), 1), (dict(sampler=9), 1), (dict(fp32_mode=4), 1),
+    (dict(x=0), 1), (dict(off=0), 1), (dict(y=0), 1),
+    (dict(x=FAKE + 8), 3), (dict(mask=FAKE + 4), 3), (dict(w=FAKE + 2), 3),
+    (dict(cv="g16_bf16"), 2),             # Cin/G = 4, not a multiple of 8 for bf16
+])
+def test_dcn_forward_validation(lib, kw, status):
+    cvs = {"g3": _conv(offset_groups=3), "s0": _conv(stride_h=0),
+           "tiny": _conv(pad_h=0, pad_w=0), "g16_bf16": _conv(offset_groups=16)}
+    if kw.get("cv") in cvs:
+        name = kw.pop("cv")
+        kw["cv"] = cvs[name]
+        if name == "tiny":
+            kw.update(H=1, W=1)
+    assert _fwd(lib, **kw) == status
+    assert lib.defcon_last_error_detail() != b""
+
+
+def test_dcn_forward_limit(lib):
+    # N*H*W*Cin >= 2^31 is rejected before launch
+    assert _fwd(lib, N=4096, H=128, W=128, Cin=64) == 5
+
+
+def test_offset_branch_validation(lib):
+    V = ctypes.c_void_p
+    args = [V(FAKE), 1, 8, 8, 16, 1, V(FAKE), V(FAKE), V(FAKE), V(FAKE), V(FAKE), 3]
+    assert lib.defcon_offset_dw_conv(*args, _conv(), V(0), V(FAKE), None) == 1      # offset NULL
+    assert lib.defcon_offset_dw_conv(*args, _conv(), V(FAKE + 4), V(FAKE), None) == 3
+    assert lib.defcon_offset_dw_conv(*args, _conv(offset_groups=64), V(FAKE), V(FAKE), None) == 5
+    bad = list(args)
+    bad[1] = 0
+    assert lib.defcon_offset_dw_conv(*bad, _conv(), V(FAKE), V(FAKE), None) == 1
+
+
+def test_workspace_size_and_layer_size(lib):
+    out = ctypes.c_size_t(99)
+    assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(), 1, 0, 1, ctypes.byref(out)) == 0
+    assert out.value == 0
+    assert lib.defcon_layer_workspace_size(2, 8, 8, 64, 1, 64, 3, _conv(), 1, 0, 1, ctypes.byref(out)) == 0
+    # x (2*8*8*64*2) + offsets + mask + y, each 256-aligned
+    assert out.value >= 2 * 8 * 8 * 64 * 2 * 2 + 2 * 64 * 9 * 3 * 4
+    assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(offset_groups=3), 1, 0, 1,
+                                         ctypes.byref(out)) == 1
+
+
+def test_binding_rejects_host_tensors():
+    import torch
+    import paper_conf_ipps_jayaweeralwrk24_b200 as d
+    x = torch.zeros(1, 4, 4, 16)
+    with pytest.raises(ValueError):
+        d.defcon_dcn_forward(x, torch.zeros(1, 4, 4, 1, 9, 2), None, torch.zeros(16, 3, 3, 16))
+
+
+def test_product_never_imports_oracle():
+    """The product package must not import, link or call oracle/ (fail loudly instead)."""
+    pkg = os.path.join(ROOT, "paper_conf_ipps_jayaweeralwrk24_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                src = open(os.path.join(dirpath, f)).read()
+                assert "oracle" not in src.lower(), f

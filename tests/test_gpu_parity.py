@@ -1,0 +1,181 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle, element by element.
+
+Tolerances (BASELINE.json north_star; metric = normwise max|g - r| / max|r|, reading R17):
+  fp32 path 1e-4, bf16 tensor-core path 2e-2, texture-filtered path 5e-3.
+Inputs come from defcon_workloads.inputs (seeded, bf16-rounded for bf16 configs), so the
+oracle sees exactly the values the GPU sees.
+"""
+import numpy as np
+import pytest
+import torch
+
+from defcon_workloads import configs, inputs
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"f32": 1e-4, "bf16": 2e-2}
+TDT = {"f32": torch.float32, "bf16": torch.bfloat16}
+
+
+@pytest.fixture(scope="module")
+def dev():
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    from paper_conf_ipps_jayaweeralwrk24_b200 import build
+    build.build()
+    return torch.device("cuda:0")
+
+
+@pytest.fixture(scope="module")
+def d(dev):
+    import paper_conf_ipps_jayaweeralwrk24_b200 as d
+    d.load_library()
+    return d
+
+
+def normwise(g, r):
+    g = np.asarray(g, np.float64)
+    r = np.asarray(r, np.float64)
+    return float(np.max(np.abs(g - r)) / max(np.max(np.abs(r)), 1e-30))
+
+
+def to_dev(a, dtype, dev):
+    return None if a is None else torch.from_numpy(np.ascontiguousarray(a)).to(dev, dtype)
+
+
+def run_dcn(d, dev, c, L, sampler="ldg", fp32_mode="simt"):
+    dt = TDT[c.dtype]
+    y = d.defcon_dcn_forward(to_dev(L["x"], dt, dev), to_dev(L["offset"], torch.float32, dev),
+                             to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], dt, dev),
+                             to_dev(L["bias"], torch.float32, dev), stride=c.stride, pad=c.pad,
+                             dil=c.dil, offset_groups=c.G, sampler=sampler, fp32_mode=fp32_mode)
+    torch.cuda.synchronize()
+    return y.float().cpu().numpy()
+
+
+def small(name, **kw):
+    base = dict(N=2, Cin=128, Cout=128, H=19, W=17, config_id=100)
+    base.update(kw)
+    return configs.LayerConfig(name, **base)
+
+
+# M = 2*19*17 = 646 rows = 5 full 128-row tiles + a ragged tail of 6
+SMALL = [
+    small("bf16_tc_g1_v2"),
+    small("bf16_tc_g2_v1", G=2, modulated=False),
+    small("bf16_tc_s2", stride=2, H=23, W=21),
+    small("bf16_tc_dil2", dil=2, pad=2),
+    small("bf16_tc_cout64", Cout=64),
+    small("bf16_tc_cout256", Cout=256, Cin=64),
+    small("bf16_tc_cout512", Cout=512, Cin=64, H=9, W=11),
+    small("bf16_tc_cout48", Cout=48),               # N tile not full (TMA zero-fill)
+    small("bf16_simt_cg32", Cin=64, G=2),           # Cin/G = 32: CUDA-core fallback
+    small("f32_simt_g1", dtype="f32", Cin=32, Cout=40),
+    small("f32_simt_g4_s2", dtype="f32", Cin=32, Cout=24, G=4, stride=2),
+    configs.TINY,
+]
+
+
+@pytest.mark.parametrize("c", SMALL, ids=lambda c: c.name)
+def test_dcn_small_parity(oracle_mod, d, dev, c):
+    L = inputs.gen_layer(c)
+    y = run_dcn(d, dev, c, L)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
+                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    err = normwise(y, ref)
+    assert err < TOL[c.dtype], err
+    if c.dtype == "f32":
+        assert err < 1e-5
+
+
+@pytest.mark.parametrize("dist", ["zeros", "integer", "half", "far", "border", "local"])
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_dcn_special_offsets(oracle_mod, d, dev, dist, dtype):
+    c = small(f"special_{dist}", dtype=dtype, Cin=64 if dtype == "bf16" else 16, Cout=32, N=1,
+              H=13, W=15)
+    L = inputs.gen_layer(c, off_dist=dist, x_dist="normal")
+    y = run_dcn(d, dev, c, L)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
+    if dist == "far":
+        # every tap samples outside the image: y == bias exactly up to output rounding
+        b = inputs.round_to(np.broadcast_to(L["bias"], y.shape), dtype)
+        assert np.array_equal(y, b)
+    else:
+        assert normwise(y, ref) < TOL[dtype] / (2 if dtype == "bf16" else 1)
+
+
+def test_dcn_deterministic(d, dev):
+    c = small("det")
+    L = inputs.gen_layer(c)
+    y1 = run_dcn(d, dev, c, L)
+    y2 = run_dcn(d, dev, c, L)
+    assert np.array_equal(y1, y2)
+
+
+FULL = [configs.C3, configs.C4, configs.C4_G4, configs.C5, configs.C4_F32, configs.C4_G4_F32]
+
+
+@pytest.mark.parametrize("c", FULL, ids=lambda c: c.name)
+def test_dcn_full_size_sampled(oracle_mod, d, dev, c):
+    """BASELINE.json full sizes in the benchmarked launch configuration; the oracle
+    evaluates a deterministic sample of output pixels (first/last tile rows, ragged tail,
+    random interior) one by one."""
+    L = inputs.gen_layer(c)
+    y = run_dcn(d, dev, c, L).reshape(c.M, c.Cout)
+    r = np.random.default_rng(7)
+    idx = np.unique(np.concatenate([np.arange(0, 130), np.arange(c.M - 130, c.M),
+                                    r.integers(0, c.M, 300)]))
+    ref = oracle_mod.dcn_pixels(L["x"], L["offset"], L["weight"], idx, L["bias"], mask=L["mask"],
+                                stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    assert normwise(y[idx], ref) < TOL[c.dtype]
+
+
+def gen_branch_dev(c, dev):
+    P = inputs.gen_offset_branch(c)
+    return P, {k: to_dev(v, torch.float32, dev) for k, v in P.items()}
+
+
+@pytest.mark.parametrize("c", [configs.C3.replace(N=2), configs.C4_G4.replace(N=2),
+                               small("branch_s2_f32", dtype="f32", stride=2, Cin=48, modulated=False),
+                               configs.C5.replace(N=1)],
+                         ids=lambda c: c.name)
+def test_offset_branch_parity(oracle_mod, d, dev, c):
+    x = inputs.gen_x(c)
+    P, Pd = gen_branch_dev(c, dev)
+    off, msk = d.defcon_offset_dw_conv(to_dev(x, TDT[c.dtype], dev), Pd["dw_w"], Pd["dw_scale"],
+                                       Pd["dw_shift"], Pd["pw_w"], Pd["pw_b"], K=c.K,
+                                       stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
+                                       with_mask=c.modulated)
+    torch.cuda.synchronize()
+    ro, rm = oracle_mod.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
+                                      P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated,
+                                      stride=c.stride, pad=c.pad, dil=c.dil)
+    assert normwise(off.cpu().numpy(), ro) < 1e-5
+    if c.modulated:
+        assert np.max(np.abs(msk.cpu().numpy() - rm)) < 1e-5
+    # the generated branch yields offsets of the intended scale (std ~ 1.5 px)
+    assert 0.5 < float(np.std(ro)) < 4.0
+
+
+def test_layer_chain_and_host_entry(oracle_mod, d, dev):
+    """Whole hot path (step 1 -> step 2) on C3 shapes (N reduced), device and host entry."""
+    c = configs.C3.replace(N=2)
+    x = inputs.gen_x(c)
+    w, b = inputs.gen_weight(c)
+    P, Pd = gen_branch_dev(c, dev)
+    xd, wd, bd = to_dev(x, torch.bfloat16, dev), to_dev(w, torch.bfloat16, dev), to_dev(b, torch.float32, dev)
+    off, msk = d.defcon_offset_dw_conv(xd, Pd["dw_w"], Pd["dw_scale"], Pd["dw_shift"], Pd["pw_w"],
+                                       Pd["pw_b"])
+    y = d.defcon_dcn_forward(xd, off, msk, wd, bd)
+    ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout), dtype=torch.uint8,
+                     device=dev)
+    xh = torch.from_numpy(x).to(torch.bfloat16).pin_memory()
+    yh = torch.empty(tuple(y.shape), dtype=torch.bfloat16).pin_memory()
+    d.defcon_layer_forward_host(xh, Pd, wd, bd, yh, ws)
+    torch.cuda.synchronize()
+    assert torch.equal(yh, y.cpu())
+    ro, rm = oracle_mod.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"], P["pw_b"])
+    r = np.random.default_rng(3)
+    idx = np.unique(np.concatenate([np.arange(200), r.integers(0, c.M, 300)]))
+    ref = oracle_mod.dcn_pixels(x, ro, w, idx, b, mask=rm)
+    assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
