@@ -135,6 +135,10 @@ class Layer:
         self.branch = branch_dev
         self.weight = weight
         self.bias = bias
+        import paper_conf_ipps_jayaweeralwrk24_b200 as d
+        nws = d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K, c.stride, c.pad,
+                                          c.dil, c.G, dt)
+        self.ws = torch.empty(max(nws, 16), dtype=torch.uint8, device=dev)
 
     def nbytes(self):
         return sum(t.numel() * t.element_size() for t in (self.x, self.off, self.msk, self.y,
@@ -150,7 +154,7 @@ def step1(d, c, L):
 
 def step2(d, c, L):
     d.defcon_dcn_forward(L.x, L.off, L.msk, L.weight, L.bias, stride=c.stride, pad=c.pad,
-                         dil=c.dil, offset_groups=c.G, y=L.y)
+                         dil=c.dil, offset_groups=c.G, y=L.y, workspace=L.ws)
 
 
 def capture(fn, stream):

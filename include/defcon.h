@@ -95,8 +95,9 @@ typedef struct defcon_tex_plan_s* defcon_tex_plan_t;
  *            DCN's Ho x Wo, R10) and G = cv.offset_groups
  *   offset   [N][Ho][Wo][G][K*K][2] fp32 (written)
  *   mask     [N][Ho][Wo][G][K*K] fp32 (written) or NULL (DCNv1: no mask rows)
- * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G <= 0; LIMIT if
- *   OC > 1024 or C > 4096; MISALIGNED for unaligned pointers.
+ * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G <= 0; UNSUPPORTED if
+ *   C % 8 != 0 (16-byte channel vectors); LIMIT if OC > 256 or a tensor needs >= 2^31
+ *   elements; MISALIGNED for unaligned pointers.
  */
 int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype,
                           const float* dw_w, const float* dw_scale, const float* dw_shift,
@@ -123,7 +124,9 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
  *   fp32_mode  used only when dtype == DEFCON_F32
  *   y        [N][Ho][Wo][Cout], dtype `dtype` (written)
  *   workspace / workspace_bytes: device scratch of at least defcon_dcn_workspace_size()
- *            bytes (may be NULL when that size is 0)
+ *            bytes (may be NULL when that size is 0).  The tensor-core path uses it for
+ *            stream-K tile counters (reset by the call itself, on `stream`) and fp32
+ *            partial tiles; calls that may run concurrently need distinct workspaces.
  * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G not dividing Cin, bad enums,
  *   NULL required pointers; UNSUPPORTED for (Cin/G) % 8 != 0 (bf16) or % 4 != 0 (fp32),
  *   or a Cout not multiple of 16 on the tensor-core paths; LIMIT when N*H*W*Cin >= 2^31

@@ -198,6 +198,11 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
     if y is None:
         y = torch.empty((N, Ho, Wo, Cout), device=x.device, dtype=x.dtype)
     _dev_tensor(y, "y", x.dtype, (N, Ho, Wo, Cout))
+    if workspace is None:
+        need = defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw, stride, pad, dil,
+                                         offset_groups, x.dtype, sampler, fp32_mode)
+        if need:
+            workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
     ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
     plan = None if tex_plan is None else tex_plan.handle
     rc = lib.defcon_dcn_forward(_ptr(x), N, H, W, Cin, _ptr(offset), _ptr(mask), _ptr(weight),

@@ -107,6 +107,10 @@ static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, 
     return DEFCON_OK;
 }
 
+static size_t path_workspace(const DcnGeom& g, Path path) {
+    return path == Path::TC_BF16 ? dcn_tc_bf16_workspace(g) : 0;
+}
+
 }  // namespace defcon
 
 using namespace defcon;
@@ -149,15 +153,15 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
     if (Ho <= 0 || Wo <= 0) return fail(DEFCON_ERR_INVALID_ARG, "output grid is empty");
     const int G = cv.offset_groups;
     const int OC = G * K * K * (mask ? 3 : 2);
-    if (OC > 512) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 512", OC);
+    if (OC > 256) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 256", OC);
+    if (C % 8 != 0) return fail(DEFCON_ERR_UNSUPPORTED, "offset branch needs C %% 8 == 0 (C = %d)", C);
     if ((long)N * H * W * C >= (1L << 31) || (long)N * Ho * Wo * OC >= (1L << 31))
         return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
     cudaError_t e = launch_offset_branch(x, x_dtype == DEFCON_BF16, N, H, W, C, dw_w, dw_scale,
                                          dw_shift, pw_w, pw_b, K, G, mask != nullptr, cv.stride_h,
                                          cv.stride_w, cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, Ho, Wo,
                                          offset, mask, static_cast<cudaStream_t>(stream));
-    if (e == cudaErrorInvalidValue)
-        return fail(DEFCON_ERR_LIMIT, "offset branch: C = %d needs more shared memory than available", C);
+    if (e == cudaErrorInvalidValue) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d unsupported", OC);
     if (e != cudaSuccess) return cuda_fail(e, "offset_branch launch");
     return DEFCON_OK;
 }
@@ -173,7 +177,7 @@ int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, in
     Path path;
     rc = select_path(g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
-    *bytes = 0;
+    *bytes = path_workspace(g, path);
     return DEFCON_OK;
 }
 
@@ -194,13 +198,15 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     rc = select_path(g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
     (void)tex_plan;
-    (void)workspace_bytes;
+    const size_t need = path_workspace(g, path);
+    if (need > 0 && (workspace == nullptr || workspace_bytes < need))
+        return fail(DEFCON_ERR_LIMIT, "workspace of %zu bytes < required %zu", workspace_bytes, need);
     DcnPtrs p{x, offset, mask, weight, bias, y};
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     const char* detail = "dcn launch";
     switch (path) {
-        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, st, &detail); break;
+        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, workspace, workspace_bytes, st, &detail); break;
         case Path::SIMT_BF16: e = launch_dcn_simt(g, p, true, st); break;
         default: e = launch_dcn_simt(g, p, false, st); break;
     }
@@ -228,7 +234,7 @@ static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
     c->off = align_up((size_t)g->M * g->G * g->KK * 2 * sizeof(float));
     c->msk = modulated ? align_up((size_t)g->M * g->G * g->KK * sizeof(float)) : 0;
     c->y = align_up((size_t)g->M * Cout * es);
-    c->ws = 0;
+    c->ws = align_up(path_workspace(*g, path));
     c->total = c->x + c->off + c->msk + c->y + c->ws;
     return DEFCON_OK;
 }

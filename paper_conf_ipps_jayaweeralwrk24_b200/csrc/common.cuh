@@ -197,6 +197,49 @@ DEFCON_DEVICE void st_shared_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t 
                  : "memory");
 }
 
+DEFCON_DEVICE uint4 ld_shared_v4(uint32_t addr) {
+    uint4 r;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "r"(addr));
+    return r;
+}
+
+// 64-bit address = base + 32-bit unsigned byte offset (one IMAD.WIDE.U32).
+DEFCON_DEVICE const void* add_u32(const void* base, uint32_t off) {
+    uint64_t p;
+    asm("mad.wide.u32 %0, %1, 1, %2;" : "=l"(p) : "r"(off), "l"(reinterpret_cast<uint64_t>(base)));
+    return reinterpret_cast<const void*>(p);
+}
+
+// ------------------------------------------------------------------ packed fp32 (FFMA2)
+// sm_100 executes two fp32 FMAs per instruction on a 64-bit register pair.
+DEFCON_DEVICE uint64_t f32x2_pack(float lo, float hi) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+    return r;
+}
+DEFCON_DEVICE uint64_t f32x2_fma(uint64_t a, uint64_t b, uint64_t c) {
+    uint64_t d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+    return d;
+}
+DEFCON_DEVICE uint64_t f32x2_mul(uint64_t a, uint64_t b) {
+    uint64_t d;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
+// bf16x2 word -> (lo, hi) fp32 pair (exact widening).
+DEFCON_DEVICE uint64_t bf16x2_to_f32x2(uint32_t w) {
+    return f32x2_pack(__uint_as_float(w << 16), __uint_as_float(w & 0xFFFF0000u));
+}
+// (lo, hi) fp32 pair -> bf16x2 word, round-to-nearest-even.
+DEFCON_DEVICE uint32_t f32x2_to_bf16x2(uint64_t v) {
+    uint32_t r;
+    asm("{.reg .f32 a, b;\n\tmov.b64 {a, b}, %1;\n\tcvt.rn.bf16x2.f32 %0, b, a;}" : "=r"(r) : "l"(v));
+    return r;
+}
+
 DEFCON_DEVICE uint4 ldg_nc_v4(const void* p) {
     uint4 r;
     asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"

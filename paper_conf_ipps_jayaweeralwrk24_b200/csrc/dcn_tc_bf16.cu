@@ -5,19 +5,26 @@
 //     Y[m, co] = bias[co] + sum_kd A[m, kd] * Wt[co, kd],   kd = tap * Cin + ci
 // where A[m, kd] = m_k * X(p_o + p_k + dp_k) is produced on the fly (never in HBM).
 //
-// Per CTA: one 128-row (output pixel) x BLOCK_N (output channel) tile.
-//   warps 0..NPW-1  A producers: bilinear gathers from NHWC bf16 x (16-byte vectors,
-//                   fp32 weights and lerp, RNE to bf16) written into the canonical
-//                   SWIZZLE_128B K-major smem layout; afterwards they run the epilogue
-//                   (tcgen05.ld -> + bias -> bf16 -> NHWC store).
-//   warp NPW        TMA producer for the weight tile (B, K-major, SWIZZLE_128B).
-//   warp NPW+1      TMEM allocator and single-thread tcgen05.mma issuer (M=128, N<=256
-//                   per instruction, K=16), fp32 accumulators in TMEM.
-// K loop: 64-channel chunks (outer) x taps (inner) so the taps of one chunk revisit
-// the same input neighbourhood while it is hot in L1.  Per-(row, tap) sampling
-// metadata (4 corner offsets, 4 mask-scaled weights) is computed once per offset group
-// into shared memory and reused by every chunk of that group.
-#include <cstdio>
+// Persistent, stream-K scheduled: the (tile, k-iteration) space -- tiles of 128 output
+// pixels x BLOCK_N output channels, k-iterations of 64 input channels x 1 tap -- is cut
+// into one contiguous, equal range per CTA (grid = #SMs), so there is no wave tail.
+// A tile split between CTAs is finished by whichever contributor arrives last on the
+// tile's counter, summing the fp32 partials in fixed segment order (deterministic).
+//
+// Warp roles (14 warps):
+//   0..7    A producers: bilinear gathers from NHWC bf16 x (16-byte vectors, fp32 weights
+//           and lerp, RNE to bf16) into the canonical SWIZZLE_128B K-major smem layout.
+//   8..11   epilogue: tcgen05.ld accumulators (TMEM lane = output row), + bias, bf16 NHWC
+//           store, or fp32 partial + stream-K fixup.
+//   12      TMA producer for the weight tile (B, K-major, SWIZZLE_128B).
+//   13      TMEM allocator and single-thread tcgen05.mma issuer (M=128, N<=256, K=16),
+//           fp32 accumulators double-buffered in TMEM when BLOCK_N <= 256.
+// K order inside a tile: 64-channel chunks (outer) x taps (inner), so the taps of one
+// chunk revisit the same input neighbourhood while it is hot in L1.  Per-(row, tap)
+// sampling metadata (4 corner offsets, 4 mask-scaled weights) is built once per
+// (tile, offset group) into shared memory and reused by every chunk of that group.
+#include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -29,6 +36,13 @@ constexpr int BM = 128;          // rows per tile (UMMA M)
 constexpr int BK = 64;           // bf16 elements per K chunk (= one 128-byte swizzle row)
 constexpr int A_STAGE_BYTES = BM * BK * 2;
 constexpr int META_ENTRY = 32;   // int4 corner offsets + float4 weights
+constexpr int NPW = 8;           // producer warps
+constexpr int EPI_WARP0 = 8;     // 4 epilogue warps: TMEM lane quarters 0..3
+constexpr int TMA_WARP = 12;
+constexpr int MMA_WARP = 13;
+constexpr int NUM_THREADS = 14 * 32;
+constexpr int NPT = NPW * 32;
+constexpr int ROWS = BM * 8 / NPT;   // A rows per producer thread (8 threads per 128-B row)
 
 struct TcArgs {
     const __nv_bfloat16* x;
@@ -36,11 +50,14 @@ struct TcArgs {
     const float* mask;
     const float* bias;
     __nv_bfloat16* y;
+    float* partials;       // [2 * gridDim.x][BLOCK_N / 4][BM][4] fp32
+    int* counters;         // [num_tiles], zeroed before launch
     int H, W, Cin, Cout, Kw, Ho, Wo;
     int sh, sw, ph, pw, dh, dw;
     int G, Cg, M, KK;
-    int num_chunks;   // Cin / BK
-    int num_iters;    // num_chunks * KK
+    int ipt;               // k-iterations per tile = (Cin / BK) * KK
+    int n_tiles_n;         // tiles along Cout
+    long long total_iters; // num_tiles * ipt
 };
 
 template <int BLOCK_N>
@@ -49,16 +66,34 @@ struct TcCfg {
     static constexpr int N_MMA = BLOCK_N / UMMA_N;
     static constexpr int B_STAGE_BYTES = BLOCK_N * BK * 2;
     static constexpr int STAGE_BYTES = A_STAGE_BYTES + B_STAGE_BYTES;
-    static constexpr int TMEM_COLS = BLOCK_N < 32 ? 32 : BLOCK_N;
+    static constexpr int NBUF = BLOCK_N <= 256 ? 2 : 1;      // TMEM accumulator buffers
+    static constexpr int TMEM_COLS = (BLOCK_N * NBUF) < 32 ? 32 : BLOCK_N * NBUF;
     static constexpr int TMA_BOX_N = BLOCK_N > 256 ? 256 : BLOCK_N;
 };
 
-// Sampling metadata for (row, tap) of offset group g: the element index of channel 0 of
-// each of the 4 bilinear corners and the 4 corner weights with the mask folded in.
-// Corners outside the image get weight 0 and a harmless in-bounds index 0 (R8).
+// Static stream-K partition: CTA b owns global iterations [it0(b), it0(b+1)).
+__device__ __forceinline__ long long range_begin(long long T, int G, int b) {
+    return (T * b) / G;
+}
+// The CTA whose range contains global iteration `it`.
+__device__ __forceinline__ int cta_of(long long T, int G, long long it) {
+    return (int)(((it + 1) * G - 1) / T);
+}
+
+// One segment = the part of one tile inside this CTA's range.
+struct Segment {
+    int tile;
+    int kb, ke;          // k-iteration range within the tile
+};
+
+
+// Sampling metadata for (row, tap) of offset group g: the byte offset (into x) of
+// channel 0 of each of the 4 bilinear corners and the 4 corner weights with the mask
+// folded in.  Corners outside the image get weight 0 and the harmless in-bounds
+// offset 0 (R8).
 __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int row, int tap, int g,
                                                  uint8_t* meta) {
-    int4 off = make_int4(0, 0, 0, 0);
+    uint4 off = make_uint4(0u, 0u, 0u, 0u);
     float4 wt = make_float4(0.f, 0.f, 0.f, 0.f);
     const int m = m0 + row;
     if (m < a.M) {
@@ -70,8 +105,8 @@ __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int ro
         const int i = tap / a.Kw;
         const int j = tap - i * a.Kw;
         const long pix = (long)m * a.G + g;
-        const float2 d = *reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tap) * 2);
-        const float mk = a.mask ? a.mask[pix * a.KK + tap] : 1.0f;
+        const float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tap) * 2));
+        const float mk = a.mask ? __ldg(a.mask + pix * a.KK + tap) : 1.0f;
         float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
         float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
         // Anything beyond one pixel outside samples only zeros; clamping keeps the
@@ -84,39 +119,187 @@ __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int ro
             const int y0 = (int)fy, x0 = (int)fx;
             const bool vy0 = (y0 >= 0) && (y0 < a.H), vy1 = (y0 + 1 >= 0) && (y0 + 1 < a.H);
             const bool vx0 = (x0 >= 0) && (x0 < a.W), vx1 = (x0 + 1 >= 0) && (x0 + 1 < a.W);
-            const int base = n * a.H;
-            if (vy0 && vx0) { off.x = ((base + y0) * a.W + x0) * a.Cin;         wt.x = (1.f - ly) * (1.f - lx) * mk; }
-            if (vy0 && vx1) { off.y = ((base + y0) * a.W + x0 + 1) * a.Cin;     wt.y = (1.f - ly) * lx * mk; }
-            if (vy1 && vx0) { off.z = ((base + y0 + 1) * a.W + x0) * a.Cin;     wt.z = ly * (1.f - lx) * mk; }
-            if (vy1 && vx1) { off.w = ((base + y0 + 1) * a.W + x0 + 1) * a.Cin; wt.w = ly * lx * mk; }
+            const uint32_t base = (uint32_t)(n * a.H);
+            const uint32_t rowb = (uint32_t)a.Cin * 2u;   // bytes per pixel
+            if (vy0 && vx0) { off.x = ((base + y0) * a.W + x0) * rowb;         wt.x = (1.f - ly) * (1.f - lx) * mk; }
+            if (vy0 && vx1) { off.y = ((base + y0) * a.W + x0 + 1) * rowb;     wt.y = (1.f - ly) * lx * mk; }
+            if (vy1 && vx0) { off.z = ((base + y0 + 1) * a.W + x0) * rowb;     wt.z = ly * (1.f - lx) * mk; }
+            if (vy1 && vx1) { off.w = ((base + y0 + 1) * a.W + x0 + 1) * rowb; wt.w = ly * lx * mk; }
         }
     }
     uint8_t* e = meta + (row * a.KK + tap) * META_ENTRY;
-    *reinterpret_cast<int4*>(e) = off;
+    *reinterpret_cast<uint4*>(e) = off;
     *reinterpret_cast<float4*>(e + 16) = wt;
 }
 
-__device__ __forceinline__ void lerp_accumulate(float (&acc)[8], const uint4& v, float w) {
-    acc[0] = fmaf(w, bf16lo_to_f32(v.x), acc[0]);
-    acc[1] = fmaf(w, bf16hi_to_f32(v.x), acc[1]);
-    acc[2] = fmaf(w, bf16lo_to_f32(v.y), acc[2]);
-    acc[3] = fmaf(w, bf16hi_to_f32(v.y), acc[3]);
-    acc[4] = fmaf(w, bf16lo_to_f32(v.z), acc[4]);
-    acc[5] = fmaf(w, bf16hi_to_f32(v.z), acc[5]);
-    acc[6] = fmaf(w, bf16lo_to_f32(v.w), acc[6]);
-    acc[7] = fmaf(w, bf16hi_to_f32(v.w), acc[7]);
+// The 4 corner vectors (8 channels each) of one A row and their weights.
+struct RowLoad {
+    uint4 v[4];
+    float4 w;
+};
+
+__device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr) {
+    const uint4 o = ld_shared_v4(meta_addr);
+    const uint4 wb = ld_shared_v4(meta_addr + 16);
+    L.w = make_float4(__uint_as_float(wb.x), __uint_as_float(wb.y), __uint_as_float(wb.z),
+                      __uint_as_float(wb.w));
+    L.v[0] = ldg_nc_v4(add_u32(xbase, o.x));
+    L.v[1] = ldg_nc_v4(add_u32(xbase, o.y));
+    L.v[2] = ldg_nc_v4(add_u32(xbase, o.z));
+    L.v[3] = ldg_nc_v4(add_u32(xbase, o.w));
 }
 
-template <int BLOCK_N, int STAGES, int NPW>
-__global__ void __launch_bounds__((NPW + 2) * 32, 1)
+// Eq.3 for 8 channels: sum_q w_q * corner_q, fp32 (packed FFMA2), RNE to bf16, into smem.
+__device__ __forceinline__ void lerp_store_row(const RowLoad& L, uint32_t dst) {
+    uint64_t acc[4];
+    const float wq[4] = {L.w.x, L.w.y, L.w.z, L.w.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const uint64_t w2 = f32x2_pack(wq[q], wq[q]);
+        const uint32_t u[4] = {L.v[q].x, L.v[q].y, L.v[q].z, L.v[q].w};
+#pragma unroll
+        for (int h = 0; h < 4; ++h) {
+            const uint64_t c = bf16x2_to_f32x2(u[h]);
+            acc[h] = q == 0 ? f32x2_mul(c, w2) : f32x2_fma(c, w2, acc[h]);
+        }
+    }
+    st_shared_v4(dst, f32x2_to_bf16x2(acc[0]), f32x2_to_bf16x2(acc[1]), f32x2_to_bf16x2(acc[2]),
+                 f32x2_to_bf16x2(acc[3]));
+}
+
+// CTA range -> segments helper (every role walks the same sequence).
+__device__ __forceinline__ int count_segments(const TcArgs& a, long long it_begin, long long it_end) {
+    if (it_end <= it_begin) return 0;
+    return (int)((it_end - 1) / a.ipt - it_begin / a.ipt) + 1;
+}
+
+__device__ __forceinline__ Segment segment_j(const TcArgs& a, long long it_begin, long long it_end, int j) {
+    Segment sg;
+    sg.tile = (int)(it_begin / a.ipt) + j;
+    const long long t0 = (long long)sg.tile * a.ipt;
+    sg.kb = (int)(max(it_begin, t0) - t0);
+    sg.ke = (int)(min(it_end, t0 + a.ipt) - t0);
+    return sg;
+}
+
+// Epilogue of one segment for NCOLS columns [col0, col0 + NCOLS) of row r (= TMEM lane).
+// whole tile: + bias -> bf16 -> y.  Partial: fp32 partial to `slot`; the last of the
+// tile's contributors to arrive sums every partial in segment order (deterministic).
+template <int BLOCK_N, int NCOLS>
+__device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment& sg, bool whole,
+                                                 int slot, uint32_t tacc, int r, int col0,
+                                                 int bar_id, int nthr, bool leader, int* fix_flag,
+                                                 long long T, int nct) {
+    constexpr int CH = NCOLS >= 32 ? 32 : 16;
+    const int m0 = (sg.tile / a.n_tiles_n) * BM;
+    const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
+    const int row = m0 + r;
+    const bool row_ok = row < a.M;
+    float* slotp = a.partials + (size_t)slot * BLOCK_N * BM;
+#pragma unroll 1
+    for (int c = col0; c < col0 + NCOLS; c += CH) {
+        uint32_t v[CH];
+        tmem_ld_32x32b_x16(tacc + c, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
+        if constexpr (CH == 32) tmem_ld_32x32b_x16(tacc + c + 16, *reinterpret_cast<uint32_t(*)[16]>(&v[16]));
+        tmem_ld_wait();
+        if (whole) {
+            if (row_ok) {
+#pragma unroll
+                for (int h = 0; h < CH; h += 16) {
+                    if (n0 + c + h < a.Cout) {
+                        uint32_t pk[8];
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) {
+                            const int co = n0 + c + h + 2 * u;
+                            const float b0 = a.bias ? __ldg(a.bias + co) : 0.f;
+                            const float b1 = a.bias ? __ldg(a.bias + co + 1) : 0.f;
+                            pk[u] = pack_bf16x2(__uint_as_float(v[h + 2 * u]) + b0,
+                                                __uint_as_float(v[h + 2 * u + 1]) + b1);
+                        }
+                        uint4* dst = reinterpret_cast<uint4*>(a.y + (size_t)row * a.Cout + n0 + c + h);
+                        dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                        dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+                    }
+                }
+            }
+        } else {
+            // fp32 partial, layout [col/4][row][4] (coalesced across lanes)
+#pragma unroll
+            for (int u = 0; u < CH / 4; ++u) {
+                const float4 f = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                                             __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
+                __stcg(reinterpret_cast<float4*>(slotp) + (size_t)((c >> 2) + u) * BM + r, f);
+            }
+        }
+    }
+    if (whole) return;
+
+    __threadfence();
+    named_bar_sync(bar_id, nthr);
+    const long long t0 = (long long)sg.tile * a.ipt;
+    const int b_lo = cta_of(T, nct, t0);
+    const int b_hi = cta_of(T, nct, t0 + a.ipt - 1);
+    if (leader) {
+        const int old = atomicAdd(a.counters + sg.tile, 1);
+        *fix_flag = (old == b_hi - b_lo) ? 1 : 0;
+    }
+    named_bar_sync(bar_id, nthr);
+    const bool finisher = *fix_flag != 0;
+    named_bar_sync(bar_id, nthr);   // fix_flag may be reused by the next segment
+    if (!finisher) return;
+    __threadfence();
+    if (!row_ok) return;
+#pragma unroll 1
+    for (int c = col0; c < col0 + NCOLS; c += 16) {
+        if (n0 + c >= a.Cout) break;
+        float acc[16];
+#pragma unroll
+        for (int u = 0; u < 16; ++u) acc[u] = 0.f;
+#pragma unroll 1
+        for (int b = b_lo; b <= b_hi; b += 2) {
+            float4 f[2][4];
+#pragma unroll
+            for (int s = 0; s < 2; ++s) {
+                if (b + s <= b_hi) {
+                    // slot 2b if this tile is b's first segment, else 2b+1
+                    const int bb = b + s;
+                    const int sidx = 2 * bb + ((range_begin(T, nct, bb) / a.ipt) == sg.tile ? 0 : 1);
+                    const float4* src = reinterpret_cast<const float4*>(a.partials + (size_t)sidx * BLOCK_N * BM);
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) f[s][u] = __ldcg(src + (size_t)((c >> 2) + u) * BM + r);
+                }
+            }
+#pragma unroll
+            for (int s = 0; s < 2; ++s) {
+                if (b + s <= b_hi) {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        acc[4 * u] += f[s][u].x; acc[4 * u + 1] += f[s][u].y;
+                        acc[4 * u + 2] += f[s][u].z; acc[4 * u + 3] += f[s][u].w;
+                    }
+                }
+            }
+        }
+        uint32_t pk[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const int co = n0 + c + 2 * u;
+            const float b0 = a.bias ? __ldg(a.bias + co) : 0.f;
+            const float b1 = a.bias ? __ldg(a.bias + co + 1) : 0.f;
+            pk[u] = pack_bf16x2(acc[2 * u] + b0, acc[2 * u + 1] + b1);
+        }
+        uint4* dst = reinterpret_cast<uint4*>(a.y + (size_t)row * a.Cout + n0 + c);
+        dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+    }
+}
+
+template <int BLOCK_N, int STAGES>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
     dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const TcArgs a) {
     using Cfg = TcCfg<BLOCK_N>;
-    constexpr int NPT = NPW * 32;                 // producer threads
-    constexpr int ROWS_PER_PASS = NPT / 8;        // 8 threads (16 B each) per 128-B row
-    constexpr int PASSES = BM / ROWS_PER_PASS;    // rows per producer thread
 
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    // 1024-byte alignment for the SWIZZLE_128B atoms.
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                ~uintptr_t(1023));
     uint8_t* sA = smem;
@@ -126,25 +309,33 @@ __global__ void __launch_bounds__((NPW + 2) * 32, 1)
     uint64_t* full_a = bars;
     uint64_t* full_b = bars + STAGES;
     uint64_t* empty = bars + 2 * STAGES;
-    uint64_t* accum_full = bars + 3 * STAGES;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * STAGES + 1);
+    uint64_t* tmem_full = bars + 3 * STAGES;
+    uint64_t* tmem_empty = tmem_full + Cfg::NBUF;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty + Cfg::NBUF);
+    int* fix_flag = reinterpret_cast<int*>(tmem_slot + 1);     // [0] epilogue, [1] producers
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
-    const int m0 = blockIdx.x * BM;
-    const int n0 = blockIdx.y * BLOCK_N;
+    const long long T = a.total_iters;
+    const int nct = gridDim.x;
+    const long long it_begin = range_begin(T, nct, blockIdx.x);
+    const long long it_end = range_begin(T, nct, blockIdx.x + 1);
+    const int nseg = count_segments(a, it_begin, it_end);
 
-    if (warp == NPW && lane == 0) {
+    if (warp == TMA_WARP && lane == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&full_a[s], NPW);
             mbar_init(&full_b[s], 1);
             mbar_init(&empty[s], 1);
         }
-        mbar_init(accum_full, 1);
+        for (int b = 0; b < Cfg::NBUF; ++b) {
+            mbar_init(&tmem_full[b], 1);
+            mbar_init(&tmem_empty[b], 4);
+        }
         fence_barrier_init();
         tma_prefetch_desc(&wmap);
     }
-    if (warp == NPW + 1) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    if (warp == MMA_WARP) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
@@ -153,145 +344,226 @@ __global__ void __launch_bounds__((NPW + 2) * 32, 1)
     if (warp < NPW) {
         // ===================== A producers =====================
         const int t = threadIdx.x;
-        const int cvec = t & 7;            // 16-byte vector within the 128-byte row
-        const int rsub = t >> 3;
-        int cur_group = -1;
-        for (int it = 0; it < a.num_iters; ++it) {
-            const int chunk = it / a.KK;
-            const int tap = it - chunk * a.KK;
-            const int g = (chunk * BK) / a.Cg;
-            if (g != cur_group) {
-                if (cur_group >= 0) named_bar_sync(1, NPT);   // old table no longer read
-                for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry(a, m0, e / a.KK, e % a.KK, g, meta);
-                named_bar_sync(1, NPT);
-                cur_group = g;
-            }
-            const int s = it % STAGES;
-            const uint32_t ph = (uint32_t)(it / STAGES) & 1u;
-            mbar_wait(&empty[s], ph ^ 1u);
-
-            const int ch = chunk * BK + cvec * 8;
-            const __nv_bfloat16* xc = a.x + ch;
-            uint4 v[PASSES][4];
-            float4 w[PASSES];
+        const int cvec = t & 7;              // 16-byte vector within the 128-byte row
+        const uint32_t meta_s = smem_u32(meta);
+        const uint32_t a_s = smem_u32(sA);
+        uint32_t dst[ROWS], mrow[ROWS];
 #pragma unroll
-            for (int p = 0; p < PASSES; ++p) {
-                const int row = rsub + p * ROWS_PER_PASS;
-                const uint8_t* e = meta + (row * a.KK + tap) * META_ENTRY;
-                const int4 o = *reinterpret_cast<const int4*>(e);
-                w[p] = *reinterpret_cast<const float4*>(e + 16);
-                v[p][0] = ldg_nc_v4(xc + o.x);
-                v[p][1] = ldg_nc_v4(xc + o.y);
-                v[p][2] = ldg_nc_v4(xc + o.z);
-                v[p][3] = ldg_nc_v4(xc + o.w);
-            }
-            const uint32_t a_stage = smem_u32(sA + s * A_STAGE_BYTES);
-#pragma unroll
-            for (int p = 0; p < PASSES; ++p) {
-                const int row = rsub + p * ROWS_PER_PASS;
-                float acc[8];
-#pragma unroll
-                for (int c = 0; c < 8; ++c) acc[c] = 0.f;
-                lerp_accumulate(acc, v[p][0], w[p].x);
-                lerp_accumulate(acc, v[p][1], w[p].y);
-                lerp_accumulate(acc, v[p][2], w[p].z);
-                lerp_accumulate(acc, v[p][3], w[p].w);
-                const uint32_t dst = a_stage + row * 128 + ((cvec ^ (row & 7)) << 4);
-                st_shared_v4(dst, pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]),
-                             pack_bf16x2(acc[4], acc[5]), pack_bf16x2(acc[6], acc[7]));
-            }
-            fence_proxy_async_smem();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&full_a[s]);
+        for (int p = 0; p < ROWS; ++p) {
+            const int row = (t >> 3) + p * (NPT / 8);
+            dst[p] = row * 128 + ((cvec ^ (row & 7)) << 4);
+            mrow[p] = meta_s + row * a.KK * META_ENTRY;
         }
-
-        // ===================== epilogue =====================
-        mbar_wait(accum_full, 0);
-        tc_fence_after();
-        const int q = warp & 3;                    // TMEM lane quarter of this warp
-        constexpr int SLICES = NPW / 4;
-        constexpr int COLS = BLOCK_N / SLICES;
-        const int col0 = (warp >> 2) * COLS;
-        const int row = m0 + q * 32 + lane;
-        __nv_bfloat16* yrow = a.y + (size_t)row * a.Cout + n0;
-#pragma unroll 1
-        for (int c = col0; c < col0 + COLS; c += 16) {
-            uint32_t r[16];
-            tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)c, r);
-            tmem_ld_wait();
-            if (row < a.M && n0 + c < a.Cout) {
-                uint32_t pk[8];
+        int q = 0;                           // running k-iteration (stage) counter
+        for (int j = 0; j < nseg; ++j) {
+            const Segment sg = segment_j(a, it_begin, it_end, j);
+            const int m0 = (sg.tile / a.n_tiles_n) * BM;
+            int chunk = sg.kb / a.KK;
+            int tap = sg.kb - chunk * a.KK;
+            int g = (chunk * BK) / a.Cg;
+            named_bar_sync(1, NPT);          // previous table no longer read
+            for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry(a, m0, e / a.KK, e % a.KK, g, meta);
+            named_bar_sync(1, NPT);
+            const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + cvec * 8) * 2;
+            RowLoad L[ROWS];
 #pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                    float b0 = a.bias ? __ldg(a.bias + n0 + c + 2 * j) : 0.f;
-                    float b1 = a.bias ? __ldg(a.bias + n0 + c + 2 * j + 1) : 0.f;
-                    pk[j] = pack_bf16x2(__uint_as_float(r[2 * j]) + b0,
-                                        __uint_as_float(r[2 * j + 1]) + b1);
+            for (int p = 0; p < ROWS; ++p) issue_row(L[p], xb, mrow[p] + tap * META_ENTRY);
+            for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
+                int ntap = tap + 1, nchunk = chunk;
+                if (ntap == a.KK) { ntap = 0; ++nchunk; }
+                const bool has_next = kt + 1 < sg.ke;
+                int ng = g;
+                if (has_next && nchunk != chunk) ng = (nchunk * BK) / a.Cg;
+                const bool prefetch = has_next && ng == g;
+                const uint8_t* nxb = nchunk != chunk ? xb + BK * 2 : xb;
+
+                const int s = q % STAGES;
+                mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
+                const uint32_t stage = a_s + s * A_STAGE_BYTES;
+#pragma unroll
+                for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
+                    lerp_store_row(L[p], stage + dst[p]);
+                    if (prefetch) issue_row(L[p], nxb, mrow[p] + ntap * META_ENTRY);
                 }
-                uint4* dst = reinterpret_cast<uint4*>(yrow + c);
-                dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-                dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+                fence_proxy_async_smem();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&full_a[s]);
+
+                if (has_next && !prefetch) {          // offset group changes: new table
+                    named_bar_sync(1, NPT);
+                    for (int e = t; e < BM * a.KK; e += NPT)
+                        build_meta_entry(a, m0, e / a.KK, e % a.KK, ng, meta);
+                    named_bar_sync(1, NPT);
+                    g = ng;
+#pragma unroll
+                    for (int p = 0; p < ROWS; ++p) issue_row(L[p], nxb, mrow[p] + ntap * META_ENTRY);
+                }
+                tap = ntap;
+                chunk = nchunk;
+                xb = nxb;
             }
         }
-    } else if (warp == NPW) {
+        // The producers (4 lane quarters x NPW/4 column slices) run the last segment's
+        // epilogue, which would otherwise be exposed at the end of the CTA's range.
+        if (nseg > 0) {
+            const int j = nseg - 1;
+            const Segment sg = segment_j(a, it_begin, it_end, j);
+            const int buf = j % Cfg::NBUF;
+            mbar_wait(&tmem_full[buf], (uint32_t)(j / Cfg::NBUF) & 1u);
+            tc_fence_after();
+            const int qd = warp & 3;
+            const int r = qd * 32 + lane;
+            const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
+            const bool whole = sg.kb == 0 && sg.ke == a.ipt;
+            const int slot = 2 * blockIdx.x + (j == 0 ? 0 : 1);
+            constexpr int SLICE = BLOCK_N / (NPW / 4);
+            epilogue_segment<BLOCK_N, SLICE>(a, sg, whole, slot, tacc, r, (warp >> 2) * SLICE,
+                                             1, NPT, t == 0, fix_flag + 1, T, nct);
+        }
+    } else if (warp < EPI_WARP0 + 4) {
+        // ===================== epilogue (all segments but the last) =====================
+        const int qd = warp & 3;                    // TMEM lane quarter of this warp
+        const int r = qd * 32 + lane;               // row within the tile (= TMEM lane)
+        for (int j = 0; j + 1 < nseg; ++j) {
+            const Segment sg = segment_j(a, it_begin, it_end, j);
+            const int buf = j % Cfg::NBUF;
+            mbar_wait(&tmem_full[buf], (uint32_t)(j / Cfg::NBUF) & 1u);
+            tc_fence_after();
+            const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
+            const bool whole = sg.kb == 0 && sg.ke == a.ipt;
+            const int slot = 2 * blockIdx.x + (j == 0 ? 0 : 1);
+            // Release the accumulator as soon as it is in registers / written out.
+            epilogue_segment<BLOCK_N, BLOCK_N>(a, sg, whole, slot, tacc, r, 0, 2, 128,
+                                               threadIdx.x == EPI_WARP0 * 32, fix_flag, T, nct);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&tmem_empty[buf]);
+        }
+    } else if (warp == TMA_WARP) {
         // ===================== TMA producer (weights) =====================
         if (lane == 0) {
-            for (int it = 0; it < a.num_iters; ++it) {
-                const int chunk = it / a.KK;
-                const int tap = it - chunk * a.KK;
-                const int s = it % STAGES;
-                const uint32_t ph = (uint32_t)(it / STAGES) & 1u;
-                mbar_wait(&empty[s], ph ^ 1u);
-                mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
-                const int kd = tap * a.Cin + chunk * BK;
+            int q = 0;
+            for (int j = 0; j < nseg; ++j) {
+                const Segment sg = segment_j(a, it_begin, it_end, j);
+                const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
+                int chunk = sg.kb / a.KK;
+                int tap = sg.kb - chunk * a.KK;
+                for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
+                    const int s = q % STAGES;
+                    mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
+                    mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
+                    const int kd = tap * a.Cin + chunk * BK;
 #pragma unroll
-                for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h)
-                    tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + h * Cfg::TMA_BOX_N * 128, &wmap,
-                                &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+                    for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h)
+                        tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + h * Cfg::TMA_BOX_N * 128, &wmap,
+                                    &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+                    if (++tap == a.KK) { tap = 0; ++chunk; }
+                }
             }
         }
     } else {
         // ===================== MMA issuer =====================
         if (lane == 0) {
             constexpr uint32_t idesc = make_idesc(1u /*BF16*/, BM, Cfg::UMMA_N);
-            for (int it = 0; it < a.num_iters; ++it) {
-                const int s = it % STAGES;
-                const uint32_t ph = (uint32_t)(it / STAGES) & 1u;
-                mbar_wait(&full_a[s], ph);
-                mbar_wait(&full_b[s], ph);
+            int q = 0;
+            for (int j = 0; j < nseg; ++j) {
+                const Segment sg = segment_j(a, it_begin, it_end, j);
+                const int buf = j % Cfg::NBUF;
+                mbar_wait(&tmem_empty[buf], ((uint32_t)(j / Cfg::NBUF) & 1u) ^ 1u);
                 tc_fence_after();
-                const uint32_t a_addr = smem_u32(sA + s * A_STAGE_BYTES);
-                const uint32_t b_addr = smem_u32(sB + s * Cfg::B_STAGE_BYTES);
+                const uint32_t d_base = tmem_base + (uint32_t)(buf * BLOCK_N);
+                for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
+                    const int s = q % STAGES;
+                    const uint32_t ph = (uint32_t)(q / STAGES) & 1u;
+                    mbar_wait(&full_a[s], ph);
+                    mbar_wait(&full_b[s], ph);
+                    tc_fence_after();
+                    const uint32_t a_addr = smem_u32(sA + s * A_STAGE_BYTES);
+                    const uint32_t b_addr = smem_u32(sB + s * Cfg::B_STAGE_BYTES);
 #pragma unroll
-                for (int kk = 0; kk < BK / 16; ++kk) {
-                    const uint64_t adesc = make_sw128_desc(a_addr + kk * 32);
+                    for (int kk = 0; kk < BK / 16; ++kk) {
+                        const uint64_t adesc = make_sw128_desc(a_addr + kk * 32);
 #pragma unroll
-                    for (int h = 0; h < Cfg::N_MMA; ++h) {
-                        const uint64_t bdesc =
-                            make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
-                        mma_bf16_ss(tmem_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
-                                    (it | kk) != 0 ? 1u : 0u);
+                        for (int h = 0; h < Cfg::N_MMA; ++h) {
+                            const uint64_t bdesc =
+                                make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
+                            mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
+                                        (kt != sg.kb || kk != 0) ? 1u : 0u);
+                        }
                     }
+                    mma_commit(&empty[s]);
                 }
-                mma_commit(&empty[s]);
+                mma_commit(&tmem_full[buf]);
             }
-            mma_commit(accum_full);
         }
     }
 
     __syncwarp();
     tc_fence_before();
     __syncthreads();
-    if (warp == NPW + 1) {
+    if (warp == MMA_WARP) {
         tc_fence_after();
         tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
     }
 }
 
-template <int BLOCK_N, int STAGES, int NPW>
-cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, cudaStream_t stream,
-                        const char** detail) {
+int num_sms() {
+    static int n = 0;
+    if (n == 0) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+template <int BLOCK_N>
+struct Plan {
+    int grid;
+    int n_tiles;
+    int n_tiles_n;
+    int ipt;
+    long long total;
+    size_t counters_bytes;
+    size_t partial_bytes;
+};
+
+template <int BLOCK_N>
+Plan<BLOCK_N> make_plan(const DcnGeom& g) {
+    Plan<BLOCK_N> p;
+    p.n_tiles_n = (g.Cout + BLOCK_N - 1) / BLOCK_N;
+    p.n_tiles = ((g.M + BM - 1) / BM) * p.n_tiles_n;
+    p.ipt = (g.Cin / BK) * g.KK;
+    p.total = (long long)p.n_tiles * p.ipt;
+    // At least 4 k-iterations per CTA; DEFCON_MAX_CTAS caps the grid (tests use it to
+    // force long persistent ranges and many whole tiles per CTA).
+    long long grid = std::min<long long>(num_sms(), (p.total + 3) / 4);
+    if (const char* env = getenv("DEFCON_MAX_CTAS")) {
+        const long long cap = atoll(env);
+        if (cap > 0) grid = std::min(grid, cap);
+    }
+    p.grid = (int)std::max<long long>(grid, 1);
+    p.counters_bytes = ((size_t)p.n_tiles * sizeof(int) + 255) & ~size_t(255);
+    p.partial_bytes = (size_t)2 * p.grid * BLOCK_N * BM * sizeof(float);
+    return p;
+}
+
+template <int BLOCK_N>
+size_t workspace_impl(const DcnGeom& g) {
+    auto p = make_plan<BLOCK_N>(g);
+    return p.counters_bytes + p.partial_bytes;
+}
+
+template <int BLOCK_N, int STAGES>
+cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
+                        cudaStream_t stream, const char** detail) {
     using Cfg = TcCfg<BLOCK_N>;
+    auto plan = make_plan<BLOCK_N>(g);
+    if (ws_bytes < plan.counters_bytes + plan.partial_bytes || ws == nullptr) {
+        *detail = "workspace too small for the stream-K partials";
+        return cudaErrorInvalidValue;
+    }
     PFN_encodeTiled encode = get_encode_tiled();
     if (!encode) {
         *detail = "cuTensorMapEncodeTiled entry point unavailable";
@@ -317,22 +589,29 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, cudaStream_t stream,
     a.mask = p.mask;
     a.bias = p.bias;
     a.y = static_cast<__nv_bfloat16*>(p.y);
+    a.counters = static_cast<int*>(ws);
+    a.partials = reinterpret_cast<float*>(static_cast<uint8_t*>(ws) + plan.counters_bytes);
     a.H = g.H; a.W = g.W; a.Cin = g.Cin; a.Cout = g.Cout; a.Kw = g.Kw; a.Ho = g.Ho; a.Wo = g.Wo;
     a.sh = g.sh; a.sw = g.sw; a.ph = g.ph; a.pw = g.pw; a.dh = g.dh; a.dw = g.dw;
     a.G = g.G; a.Cg = g.Cg; a.M = g.M; a.KK = g.KK;
-    a.num_chunks = g.Cin / BK;
-    a.num_iters = a.num_chunks * g.KK;
+    a.ipt = plan.ipt;
+    a.n_tiles_n = plan.n_tiles_n;
+    a.total_iters = plan.total;
 
+    cudaError_t e = cudaMemsetAsync(a.counters, 0, plan.counters_bytes, stream);
+    if (e != cudaSuccess) {
+        *detail = "cudaMemsetAsync of the stream-K tile counters failed";
+        return e;
+    }
     const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + (size_t)BM * g.KK * META_ENTRY +
-                        (3 * STAGES + 1) * 8 + 16;
-    auto kern = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                        (3 * STAGES + 2 * Cfg::NBUF) * 8 + 32;
+    auto kern = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES>;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) {
         *detail = "cudaFuncSetAttribute(MaxDynamicSharedMemorySize) failed";
         return e;
     }
-    dim3 grid((g.M + BM - 1) / BM, (g.Cout + BLOCK_N - 1) / BLOCK_N);
-    kern<<<grid, (NPW + 2) * 32, smem, stream>>>(wmap, a);
+    kern<<<plan.grid, NUM_THREADS, smem, stream>>>(wmap, a);
     e = cudaGetLastError();
     if (e != cudaSuccess) *detail = "dcn_fwd_bf16_tc_kernel launch failed";
     return e;
@@ -340,7 +619,7 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, cudaStream_t stream,
 
 }  // namespace
 
-// Shared-memory budget: stages + metadata for up to 5x5 taps must fit in 227 KB.
+// Shared-memory budget: stages + metadata for up to 12 taps must fit in 227 KB.
 bool dcn_tc_bf16_supported(const DcnGeom& g) {
     if (g.Cin % BK != 0 || g.Cg % BK != 0) return false;
     if (g.Cout % 16 != 0) return false;
@@ -348,12 +627,19 @@ bool dcn_tc_bf16_supported(const DcnGeom& g) {
     return true;
 }
 
-cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, cudaStream_t stream,
-                               const char** detail) {
-    if (g.Cout <= 64) return launch_impl<64, 6, 8>(g, p, stream, detail);
-    if (g.Cout <= 128) return launch_impl<128, 4, 8>(g, p, stream, detail);
-    if (g.Cout <= 256) return launch_impl<256, 3, 8>(g, p, stream, detail);
-    return launch_impl<512, 2, 8>(g, p, stream, detail);
+size_t dcn_tc_bf16_workspace(const DcnGeom& g) {
+    if (g.Cout <= 64) return workspace_impl<64>(g);
+    if (g.Cout <= 128) return workspace_impl<128>(g);
+    if (g.Cout <= 256) return workspace_impl<256>(g);
+    return workspace_impl<512>(g);
+}
+
+cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
+                               cudaStream_t stream, const char** detail) {
+    if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, stream, detail);
+    if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, stream, detail);
+    if (g.Cout <= 256) return launch_impl<256, 3>(g, p, ws, ws_bytes, stream, detail);
+    return launch_impl<512, 2>(g, p, ws, ws_bytes, stream, detail);
 }
 
 }  // namespace defcon

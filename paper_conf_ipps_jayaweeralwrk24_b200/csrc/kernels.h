@@ -39,8 +39,9 @@ cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaS
 
 // ---- step 2, fused gather + tcgen05 implicit GEMM, bf16 (dcn_tc_bf16.cu)
 bool dcn_tc_bf16_supported(const DcnGeom& g);
-cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, cudaStream_t stream,
-                               const char** detail);
+size_t dcn_tc_bf16_workspace(const DcnGeom& g);   // stream-K counters + fp32 partials
+cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
+                               cudaStream_t stream, const char** detail);
 
 // ---- driver entry point for cuTensorMapEncodeTiled (api.cu)
 typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,

@@ -99,7 +99,11 @@ def test_offset_branch_validation(lib):
 
 def test_workspace_size_and_layer_size(lib):
     out = ctypes.c_size_t(99)
+    # bf16 tensor-core path: stream-K counters + fp32 partial tiles
     assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(), 1, 0, 1, ctypes.byref(out)) == 0
+    assert out.value > 0
+    # fp32 CUDA-core path needs none
+    assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(), 0, 0, 1, ctypes.byref(out)) == 0
     assert out.value == 0
     assert lib.defcon_layer_workspace_size(2, 8, 8, 64, 1, 64, 3, _conv(), 1, 0, 1, ctypes.byref(out)) == 0
     # x (2*8*8*64*2) + offsets + mask + y, each 256-aligned

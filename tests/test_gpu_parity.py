@@ -104,6 +104,21 @@ def test_dcn_special_offsets(oracle_mod, d, dev, dist, dtype):
         assert normwise(y, ref) < TOL[dtype] / (2 if dtype == "bf16" else 1)
 
 
+@pytest.mark.parametrize("ctas", ["1", "3", "37"])
+def test_dcn_stream_k_partitions(oracle_mod, d, dev, monkeypatch, ctas):
+    """Same result for any persistent grid: 1 CTA (every tile whole, TMEM double buffer
+    cycles many times), 3 and 37 CTAs (tiles split across CTAs, stream-K fixup)."""
+    c = small("streamk", Cout=256, Cin=64)
+    L = inputs.gen_layer(c)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
+    monkeypatch.setenv("DEFCON_MAX_CTAS", ctas)
+    y = run_dcn(d, dev, c, L)
+    assert normwise(y, ref) < TOL["bf16"]
+    monkeypatch.delenv("DEFCON_MAX_CTAS")
+    y_default = run_dcn(d, dev, c, L)
+    assert np.max(np.abs(y - y_default)) <= 2e-2 * np.max(np.abs(ref))
+
+
 def test_dcn_deterministic(d, dev):
     c = small("det")
     L = inputs.gen_layer(c)
