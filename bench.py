@@ -139,6 +139,9 @@ class Layer:
         nws = d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K, c.stride, c.pad,
                                           c.dil, c.G, dt)
         self.ws = torch.empty(max(nws, 16), dtype=torch.uint8, device=dev)
+        self.tws = torch.empty(d.defcon_offset_workspace_size(c.N, c.H, c.W, c.Cin, c.K, c.stride,
+                                                              c.pad, c.dil, c.G),
+                               dtype=torch.uint8, device=dev)
 
     def nbytes(self):
         return sum(t.numel() * t.element_size() for t in (self.x, self.off, self.msk, self.y,
@@ -149,7 +152,7 @@ def step1(d, c, L):
     B = L.branch
     d.defcon_offset_dw_conv(L.x, B["dw_w"], B["dw_scale"], B["dw_shift"], B["pw_w"], B["pw_b"],
                             K=c.K, stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
-                            with_mask=c.modulated, offset=L.off, mask=L.msk)
+                            with_mask=c.modulated, offset=L.off, mask=L.msk, workspace=L.tws)
 
 
 def step2(d, c, L):

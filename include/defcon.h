@@ -95,14 +95,21 @@ typedef struct defcon_tex_plan_s* defcon_tex_plan_t;
  *            DCN's Ho x Wo, R10) and G = cv.offset_groups
  *   offset   [N][Ho][Wo][G][K*K][2] fp32 (written)
  *   mask     [N][Ho][Wo][G][K*K] fp32 (written) or NULL (DCNv1: no mask rows)
+ *   workspace  device scratch of defcon_offset_workspace_size() bytes (the fp32 t between the
+ *            depthwise and the 1x1 launches; distinct per concurrently running call)
  * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G <= 0; UNSUPPORTED if
- *   C % 8 != 0 (16-byte channel vectors); LIMIT if OC > 256 or a tensor needs >= 2^31
- *   elements; MISALIGNED for unaligned pointers.
+ *   C % 8 != 0 (16-byte channel vectors); LIMIT if OC > 256, a tensor needs >= 2^31
+ *   elements or the workspace is too small; MISALIGNED for unaligned pointers.
  */
 int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype,
                           const float* dw_w, const float* dw_scale, const float* dw_shift,
                           const float* pw_w, const float* pw_b, int K, defcon_conv_t cv,
-                          float* offset, float* mask, void* stream);
+                          float* offset, float* mask, void* workspace, size_t workspace_bytes,
+                          void* stream);
+
+/* Device workspace defcon_offset_dw_conv needs: the fp32 intermediate t, N*Ho*Wo*C*4 bytes. */
+int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_t cv,
+                                 size_t* bytes);
 
 /*
  * Step 2 -- deformable convolution forward, Eq.2 + Eq.3:

@@ -23,7 +23,8 @@ DEFCON_FP32_3XTF32, DEFCON_FP32_SIMT = 0, 1
 
 # Every symbol include/defcon.h declares (checked by tests/test_abi.py).
 EXPORTED = (
-    "defcon_offset_dw_conv", "defcon_dcn_forward", "defcon_dcn_workspace_size",
+    "defcon_offset_dw_conv", "defcon_offset_workspace_size", "defcon_dcn_forward",
+    "defcon_dcn_workspace_size",
     "defcon_layer_forward_host", "defcon_layer_workspace_size", "defcon_tex_plan_create",
     "defcon_tex_plan_destroy", "defcon_tex_filter_probe", "defcon_status_string",
     "defcon_last_error_detail", "defcon_abi_version",
@@ -61,7 +62,9 @@ def load_library(path: str = LIB_PATH):
     lib = ctypes.CDLL(path)
     vp, fp, i, sz = ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_size_t
     conv = defcon_conv_t
-    lib.defcon_offset_dw_conv.argtypes = [vp, i, i, i, i, i, fp, fp, fp, fp, fp, i, conv, fp, fp, vp]
+    lib.defcon_offset_dw_conv.argtypes = [vp, i, i, i, i, i, fp, fp, fp, fp, fp, i, conv, fp, fp, vp,
+                                          sz, vp]
+    lib.defcon_offset_workspace_size.argtypes = [i, i, i, i, i, conv, ctypes.POINTER(sz)]
     lib.defcon_dcn_forward.argtypes = [vp, i, i, i, i, fp, fp, vp, fp, i, i, i, conv, i, i, i, vp, vp,
                                        sz, vp, vp]
     lib.defcon_dcn_workspace_size.argtypes = [i, i, i, i, i, i, i, conv, i, i, i,
@@ -131,9 +134,18 @@ def _stream_handle(stream):
     return ctypes.c_void_p(s.cuda_stream)
 
 
+def defcon_offset_workspace_size(N, H, W, C, K=3, stride=1, pad=1, dil=1, offset_groups=1) -> int:
+    lib = load_library()
+    out = ctypes.c_size_t(0)
+    rc = lib.defcon_offset_workspace_size(N, H, W, C, K, _conv(stride, pad, dil, offset_groups),
+                                          ctypes.byref(out))
+    _check(rc, "defcon_offset_workspace_size")
+    return int(out.value)
+
+
 def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, stride=1, pad=1,
                           dil=1, offset_groups=1, with_mask=True, offset=None, mask=None,
-                          stream=None):
+                          workspace=None, stream=None):
     """Step 1: lightweight offset branch.  Returns (offset, mask|None)."""
     lib = load_library()
     _dev_tensor(x, "x")
@@ -158,9 +170,15 @@ def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, str
         _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, KK))
     else:
         mask = None
+    if workspace is None:
+        workspace = torch.empty(defcon_offset_workspace_size(N, H, W, C, K, stride, pad, dil,
+                                                             offset_groups),
+                                dtype=torch.uint8, device=x.device)
     rc = lib.defcon_offset_dw_conv(_ptr(x), N, H, W, C, _DTYPES[x.dtype], _ptr(dw_w), _ptr(dw_scale),
                                    _ptr(dw_shift), _ptr(pw_w), _ptr(pw_b), K, cv, _ptr(offset),
-                                   _ptr(mask), _stream_handle(stream))
+                                   _ptr(mask), _ptr(workspace),
+                                   workspace.numel() * workspace.element_size(),
+                                   _stream_handle(stream))
     _check(rc, "defcon_offset_dw_conv")
     return offset, mask
 

@@ -133,34 +133,58 @@ const char* defcon_last_error_detail(void) { return g_detail; }
 
 int defcon_abi_version(void) { return DEFCON_ABI_VERSION; }
 
-int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype,
-                          const float* dw_w, const float* dw_scale, const float* dw_shift,
-                          const float* pw_w, const float* pw_b, int K, defcon_conv_t cv,
-                          float* offset, float* mask, void* stream) {
-    g_detail[0] = 0;
+static int branch_geom(int N, int H, int W, int C, int K, const defcon_conv_t& cv, int* Ho, int* Wo) {
     if (N <= 0 || H <= 0 || W <= 0 || C <= 0 || K <= 0)
         return fail(DEFCON_ERR_INVALID_ARG, "sizes must be positive");
     int rc = check_conv(cv);
     if (rc) return rc;
+    *Ho = out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h);
+    *Wo = out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w);
+    if (*Ho <= 0 || *Wo <= 0) return fail(DEFCON_ERR_INVALID_ARG, "output grid is empty");
+    if (C % 8 != 0) return fail(DEFCON_ERR_UNSUPPORTED, "offset branch needs C %% 8 == 0 (C = %d)", C);
+    if ((long)N * H * W * C >= (1L << 31) || (long)N * *Ho * *Wo * C >= (1L << 31))
+        return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
+    return DEFCON_OK;
+}
+
+int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_t cv, size_t* bytes) {
+    g_detail[0] = 0;
+    if (!bytes) return fail(DEFCON_ERR_INVALID_ARG, "bytes is NULL");
+    int Ho, Wo;
+    int rc = branch_geom(N, H, W, C, K, cv, &Ho, &Wo);
+    if (rc) return rc;
+    *bytes = offset_branch_workspace(N * Ho * Wo, C);
+    return DEFCON_OK;
+}
+
+int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype,
+                          const float* dw_w, const float* dw_scale, const float* dw_shift,
+                          const float* pw_w, const float* pw_b, int K, defcon_conv_t cv,
+                          float* offset, float* mask, void* workspace, size_t workspace_bytes,
+                          void* stream) {
+    g_detail[0] = 0;
+    int Ho, Wo;
+    int rc = branch_geom(N, H, W, C, K, cv, &Ho, &Wo);
+    if (rc) return rc;
     if (x_dtype != DEFCON_F32 && x_dtype != DEFCON_BF16) return fail(DEFCON_ERR_INVALID_ARG, "bad dtype");
     if (!x || !dw_w || !dw_scale || !dw_shift || !pw_w || !offset)
         return fail(DEFCON_ERR_INVALID_ARG, "NULL tensor pointer");
-    const void* ptrs[] = {x, dw_w, dw_scale, dw_shift, pw_w, pw_b, offset, mask};
+    const void* ptrs[] = {x, dw_w, dw_scale, dw_shift, pw_w, pw_b, offset, mask, workspace};
     for (const void* p : ptrs)
         if (p && !aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "tensor pointer not 16-byte aligned");
-    const int Ho = out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h);
-    const int Wo = out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w);
-    if (Ho <= 0 || Wo <= 0) return fail(DEFCON_ERR_INVALID_ARG, "output grid is empty");
     const int G = cv.offset_groups;
     const int OC = G * K * K * (mask ? 3 : 2);
     if (OC > 256) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 256", OC);
-    if (C % 8 != 0) return fail(DEFCON_ERR_UNSUPPORTED, "offset branch needs C %% 8 == 0 (C = %d)", C);
-    if ((long)N * H * W * C >= (1L << 31) || (long)N * Ho * Wo * OC >= (1L << 31))
+    if ((long)N * Ho * Wo * OC >= (1L << 31))
         return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
+    const size_t need = offset_branch_workspace(N * Ho * Wo, C);
+    if (!workspace || workspace_bytes < need)
+        return fail(DEFCON_ERR_LIMIT, "workspace of %zu bytes < required %zu", workspace_bytes, need);
     cudaError_t e = launch_offset_branch(x, x_dtype == DEFCON_BF16, N, H, W, C, dw_w, dw_scale,
                                          dw_shift, pw_w, pw_b, K, G, mask != nullptr, cv.stride_h,
                                          cv.stride_w, cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, Ho, Wo,
-                                         offset, mask, static_cast<cudaStream_t>(stream));
+                                         offset, mask, static_cast<float*>(workspace),
+                                         static_cast<cudaStream_t>(stream));
     if (e == cudaErrorInvalidValue) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d unsupported", OC);
     if (e != cudaSuccess) return cuda_fail(e, "offset_branch launch");
     return DEFCON_OK;
@@ -218,7 +242,7 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
 static size_t align_up(size_t v) { return (v + 255) & ~size_t(255); }
 
 struct LayerCarve {
-    size_t x, off, msk, y, ws, total;
+    size_t x, off, msk, y, ws, tws, total;
 };
 
 static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
@@ -235,7 +259,8 @@ static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
     c->msk = modulated ? align_up((size_t)g->M * g->G * g->KK * sizeof(float)) : 0;
     c->y = align_up((size_t)g->M * Cout * es);
     c->ws = align_up(path_workspace(*g, path));
-    c->total = c->x + c->off + c->msk + c->y + c->ws;
+    c->tws = align_up(offset_branch_workspace(g->M, Cin));
+    c->total = c->x + c->off + c->msk + c->y + c->ws + c->tws;
     return DEFCON_OK;
 }
 
@@ -272,12 +297,13 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
     float* mskd = modulated ? reinterpret_cast<float*>(base + c.x + c.off) : nullptr;
     void* yd = base + c.x + c.off + c.msk;
     void* wsd = c.ws ? base + c.x + c.off + c.msk + c.y : nullptr;
+    void* twsd = base + c.x + c.off + c.msk + c.y + c.ws;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
     cudaError_t e = cudaMemcpyAsync(xd, x_host, (size_t)N * H * W * Cin * es, cudaMemcpyHostToDevice, st);
     if (e != cudaSuccess) return cuda_fail(e, "H2D copy of x");
     rc = defcon_offset_dw_conv(xd, N, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
-                               offd, mskd, stream);
+                               offd, mskd, twsd, c.tws, stream);
     if (rc) return rc;
     if (out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h) != g.Ho ||
         out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w) != g.Wo)

@@ -240,6 +240,19 @@ DEFCON_DEVICE uint32_t f32x2_to_bf16x2(uint64_t v) {
     return r;
 }
 
+// 256-bit read-only global load (sm_100: LDG.E.256), p must be 32-byte aligned.
+struct U8x32 {
+    uint32_t w[8];
+};
+DEFCON_DEVICE U8x32 ldg_nc_v8(const void* p) {
+    U8x32 r;
+    asm volatile("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.w[0]), "=r"(r.w[1]), "=r"(r.w[2]), "=r"(r.w[3]), "=r"(r.w[4]),
+                   "=r"(r.w[5]), "=r"(r.w[6]), "=r"(r.w[7])
+                 : "l"(p));
+    return r;
+}
+
 DEFCON_DEVICE uint4 ldg_nc_v4(const void* p) {
     uint4 r;
     asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"

@@ -58,6 +58,7 @@ struct TcArgs {
     int ipt;               // k-iterations per tile = (Cin / BK) * KK
     int n_tiles_n;         // tiles along Cout
     long long total_iters; // num_tiles * ipt
+    int probe;             // 0 in production; bit flags disable parts for bottleneck probes
 };
 
 template <int BLOCK_N>
@@ -138,11 +139,16 @@ struct RowLoad {
     float4 w;
 };
 
-__device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr) {
+__device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr,
+                                          int probe = 0) {
     const uint4 o = ld_shared_v4(meta_addr);
     const uint4 wb = ld_shared_v4(meta_addr + 16);
     L.w = make_float4(__uint_as_float(wb.x), __uint_as_float(wb.y), __uint_as_float(wb.z),
                       __uint_as_float(wb.w));
+    if (probe & 2) {   // probe: no gathers
+        L.v[0] = L.v[1] = L.v[2] = L.v[3] = o;
+        return;
+    }
     L.v[0] = ldg_nc_v4(add_u32(xbase, o.x));
     L.v[1] = ldg_nc_v4(add_u32(xbase, o.y));
     L.v[2] = ldg_nc_v4(add_u32(xbase, o.z));
@@ -191,6 +197,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
                                                  int bar_id, int nthr, bool leader, int* fix_flag,
                                                  long long T, int nct) {
     constexpr int CH = NCOLS >= 32 ? 32 : 16;
+    if (a.probe & 32) return;   // probe: no epilogue
     const int m0 = (sg.tile / a.n_tiles_n) * BM;
     const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
     const int row = m0 + r;
@@ -362,12 +369,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             int tap = sg.kb - chunk * a.KK;
             int g = (chunk * BK) / a.Cg;
             named_bar_sync(1, NPT);          // previous table no longer read
-            for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry(a, m0, e / a.KK, e % a.KK, g, meta);
+            if (!(a.probe & 16) || j == 0)
+                for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry(a, m0, e / a.KK, e % a.KK, g, meta);
             named_bar_sync(1, NPT);
             const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + cvec * 8) * 2;
             RowLoad L[ROWS];
 #pragma unroll
-            for (int p = 0; p < ROWS; ++p) issue_row(L[p], xb, mrow[p] + tap * META_ENTRY);
+            for (int p = 0; p < ROWS; ++p) issue_row(L[p], xb, mrow[p] + tap * META_ENTRY, a.probe);
             for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                 int ntap = tap + 1, nchunk = chunk;
                 if (ntap == a.KK) { ntap = 0; ++nchunk; }
@@ -382,8 +390,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 const uint32_t stage = a_s + s * A_STAGE_BYTES;
 #pragma unroll
                 for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
-                    lerp_store_row(L[p], stage + dst[p]);
-                    if (prefetch) issue_row(L[p], nxb, mrow[p] + ntap * META_ENTRY);
+                    if (a.probe & 4)   // probe: no lerp, store one corner
+                        st_shared_v4(stage + dst[p], L[p].v[0].x ^ L[p].v[1].x, L[p].v[2].y ^ L[p].v[3].y,
+                                     L[p].v[0].z, L[p].v[1].w);
+                    else
+                        lerp_store_row(L[p], stage + dst[p]);
+                    if (prefetch) issue_row(L[p], nxb, mrow[p] + ntap * META_ENTRY, a.probe);
                 }
                 fence_proxy_async_smem();
                 __syncwarp();
@@ -451,6 +463,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                     const int s = q % STAGES;
                     mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
+                    if (a.probe & 8) {    // probe: no weight TMA
+                        mbar_arrive(&full_b[s]);
+                        if (++tap == a.KK) { tap = 0; ++chunk; }
+                        continue;
+                    }
                     mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
                     const int kd = tap * a.Cin + chunk * BK;
 #pragma unroll
@@ -487,8 +504,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         for (int h = 0; h < Cfg::N_MMA; ++h) {
                             const uint64_t bdesc =
                                 make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
-                            mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
-                                        (kt != sg.kb || kk != 0) ? 1u : 0u);
+                            if (!(a.probe & 1))   // probe: no MMA
+                                mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
+                                            (kt != sg.kb || kk != 0) ? 1u : 0u);
                         }
                     }
                     mma_commit(&empty[s]);
@@ -597,6 +615,8 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.ipt = plan.ipt;
     a.n_tiles_n = plan.n_tiles_n;
     a.total_iters = plan.total;
+    a.probe = 0;
+    if (const char* env = getenv("DEFCON_PROBE")) a.probe = atoi(env);
 
     cudaError_t e = cudaMemsetAsync(a.counters, 0, plan.counters_bytes, stream);
     if (e != cudaSuccess) {

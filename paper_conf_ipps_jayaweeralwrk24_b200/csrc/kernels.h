@@ -32,7 +32,8 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                 float* offset, float* mask, cudaStream_t stream);
+                                 float* offset, float* mask, float* t_ws, cudaStream_t stream);
+size_t offset_branch_workspace(int M, int C);   // bytes of the fp32 t buffer
 
 // ---- step 2, CUDA-core anchor (dcn_simt.cu): fp32 math for fp32 or bf16 storage
 cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaStream_t stream);

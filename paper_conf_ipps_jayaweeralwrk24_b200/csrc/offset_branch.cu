@@ -1,23 +1,23 @@
-// offset_branch.cu -- the paper's lightweight offset branch,
-// fused into one NHWC pass:
+// offset_branch.cu -- the paper's lightweight offset branch:
 //   t[c] = ReLU(scale[c] * sum_{3x3} W1[c] * x + shift[c])    depthwise 3x3 + folded BN
 //   u[o] = b2[o] + sum_c W2[o][c] * t[c]                      1x1 to OC = G*K*K*(2|3)
 //   offset = u[0 : 2GK^2] ([G][K*K][2] = (dy, dx), R4),  mask = sigmoid(u[2GK^2 :]) (R6)
-// One block owns PIX = 64 consecutive output pixels and walks the channels in chunks
-// of 64: phase 1 computes the chunk of t (16-byte vector loads of x, 8 channels per
-// task) into shared memory, phase 2 accumulates the 1x1 projection for the chunk with
-// a 4-pixel x OCT-output register tile per thread.  t never leaves the SM; x is read
-// once from HBM (the 3x3 halo re-reads hit L1/L2).  fp32 arithmetic throughout.
+//
+// Two launches, both sized for latency hiding rather than fused into one block-local
+// pass (which left one 170-register block per SM and three serialized waves):
+//   dw_bn_relu_kernel  thread = (8 channels, 4 pixels), taps outer so each tap's weights
+//                      are read once from shared memory for 4 pixels; 16-byte loads of x
+//                      (lanes along channels, coalesced), fp32 FMA, BN + ReLU, t ->
+//                      workspace (fp32, [M][C], L2-resident between the two launches).
+//   pw_sigmoid_kernel  the 1x1 projection [M x C] x [C x OC] on the tensor cores
+//                      (mma.sync m16n8k8 TF32 with the 3xTF32 split for fp32-level
+//                      accuracy), then offsets and sigmoid(mask logits) written out.
+// bf16 x is widened exactly; all sums are fp32.
 #include "common.cuh"
 #include "kernels.h"
 
 namespace defcon {
 namespace {
-
-constexpr int THREADS = 256;
-constexpr int PIX = 64;        // output pixels per block
-constexpr int CCH = 64;        // channels per chunk
-constexpr int TS = PIX + 4;    // t_s row stride (floats), keeps float4 alignment
 
 struct BranchArgs {
     const void* x;
@@ -26,12 +26,23 @@ struct BranchArgs {
     const float* dw_shift;
     const float* pw_w;
     const float* pw_b;
+    float* t;          // workspace [M][C]
     float* offset;
     float* mask;
     int N, H, W, C, Ho, Wo, M;
     int sh, sw, ph, pw, dh, dw;
     int n_off, n_msk, OC;
 };
+
+// ------------------------------------------------------------------ depthwise 3x3
+// Thread = (8 channels, 4 pixels).  Taps are the outer loop: the 8 weights of a tap are
+// read once from shared memory (layout [tap][half][vector][4], conflict-free) and used
+// for all 4 pixels, so registers stay low and occupancy high.
+constexpr int DW_CH = 64;                  // channels per block (8 vectors of 8)
+constexpr int DW_LANES = 32;               // pixel lanes per block
+constexpr int DW_PPT = 4;                  // pixels per thread
+constexpr int DW_THREADS = DW_LANES * DW_CH / 8;
+constexpr int DW_PIX = DW_LANES * DW_PPT;  // pixels per block
 
 template <bool BF16>
 __device__ __forceinline__ void load8(const void* x, long idx, float (&v)[8]) {
@@ -49,173 +60,280 @@ __device__ __forceinline__ void load8(const void* x, long idx, float (&v)[8]) {
     }
 }
 
-// OCT = outputs per thread along OC; 16 threads span OCP = 16 * OCT >= OC outputs.
-template <bool BF16, int OCT>
-__global__ void __launch_bounds__(THREADS) offset_branch_kernel(const BranchArgs a) {
-    constexpr int OCP = 16 * OCT;
-    extern __shared__ __align__(16) float smem_f[];
-    float* t_s = smem_f;                                   // [CCH][TS]   t, pixel-minor
-    float* w_s = t_s + CCH * TS;                           // [CCH][OCP]  W2^T, zero padded
-    float* dw_s = w_s + CCH * OCP;                         // [9][CCH]
-    float* sc_s = dw_s + 9 * CCH;                          // [CCH]
-    float* sf_s = sc_s + CCH;                              // [CCH]
-    int4* pix_s = reinterpret_cast<int4*>(sf_s + CCH);     // [PIX] (n, ho, wo, valid)
+// 32 zero bytes: the load target of taps that fall into the zero padding, so the tap
+// loop needs no branches.
+__device__ __align__(32) const uint32_t g_zero32[8] = {0, 0, 0, 0, 0, 0, 0, 0};
 
+template <bool BF16>
+__global__ void __launch_bounds__(DW_THREADS) dw_bn_relu_kernel(const BranchArgs a) {
+    __shared__ __align__(16) float w_s[9 * DW_CH];     // [tap][half][vector][4]
+    __shared__ __align__(16) float sc_s[DW_CH], sf_s[DW_CH];
     const int tid = threadIdx.x;
-    const int m0 = blockIdx.x * PIX;
-    if (tid < PIX) {
-        const int m = m0 + tid;
-        int4 q = make_int4(0, 0, 0, 0);
+    const int c0 = blockIdx.y * DW_CH;
+    const int cn = min(DW_CH, a.C - c0);                // multiple of 8
+    for (int e = tid; e < cn * 9; e += DW_THREADS) {    // coalesced along dw_w ([C][9])
+        const int c = e / 9, k = e - c * 9;
+        const int vv = c >> 3, u = c & 7;
+        w_s[((k * 2 + (u >> 2)) * 8 + vv) * 4 + (u & 3)] = __ldg(a.dw_w + (long)c0 * 9 + e);
+    }
+    for (int e = tid; e < cn; e += DW_THREADS) {
+        sc_s[e] = __ldg(a.dw_scale + c0 + e);
+        sf_s[e] = __ldg(a.dw_shift + c0 + e);
+    }
+    __syncthreads();
+    const int v = tid & 7;                 // 8-channel vector within the 64-channel slice
+    const int lane_p = tid >> 3;           // pixel lane
+    if (v * 8 >= cn) return;
+    constexpr int ES = BF16 ? 2 : 4;       // bytes per element of x
+    const int hw = a.Ho * a.Wo;
+    const long pix_bytes = (long)a.C * ES;
+    // per pixel: byte pointer of tap (0,0) and a 9-bit mask of taps inside the image
+    const uint8_t* base[DW_PPT];
+    uint32_t valid[DW_PPT];
+#pragma unroll
+    for (int pp = 0; pp < DW_PPT; ++pp) {
+        const int m = blockIdx.x * DW_PIX + pp * DW_LANES + lane_p;
+        valid[pp] = 0u;
+        base[pp] = reinterpret_cast<const uint8_t*>(a.x);
         if (m < a.M) {
-            const int hw = a.Ho * a.Wo;
-            q.x = m / hw;
-            const int rem = m - q.x * hw;
-            q.y = rem / a.Wo;
-            q.z = rem - q.y * a.Wo;
-            q.w = 1;
+            const int n = m / hw;
+            const int rem = m - n * hw;
+            const int ho = rem / a.Wo;
+            const int y0 = ho * a.sh - a.ph, x0 = (rem - ho * a.Wo) * a.sw - a.pw;
+#pragma unroll
+            for (int k = 0; k < 9; ++k) {
+                const int yy = y0 + (k / 3) * a.dh, xx = x0 + (k % 3) * a.dw;
+                if (yy >= 0 && yy < a.H && xx >= 0 && xx < a.W) valid[pp] |= 1u << k;
+            }
+            // may point outside x for padded taps; only dereferenced for valid taps
+            base[pp] = reinterpret_cast<const uint8_t*>(a.x) +
+                       (((long)n * a.H + y0) * a.W + x0) * pix_bytes + (long)(c0 + v * 8) * ES;
         }
-        pix_s[tid] = q;
     }
-    const int tp = tid >> 4;     // pixel group: pixels 4tp .. 4tp+3
-    const int to = tid & 15;     // output group: outputs to*OCT .. to*OCT+OCT-1
-    float acc[4][OCT];
+    uint64_t s[DW_PPT][4];                 // 8 channels as fp32 pairs (FFMA2)
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
+    for (int pp = 0; pp < DW_PPT; ++pp)
 #pragma unroll
-        for (int j = 0; j < OCT; ++j) acc[i][j] = 0.f;
-
-    for (int c0 = 0; c0 < a.C; c0 += CCH) {
-        const int cn = min(CCH, a.C - c0);     // multiple of 8
-        __syncthreads();                        // previous chunk fully consumed
-        for (int e = tid; e < cn * 9; e += THREADS) {
-            const int c = e / 9, k = e - (e / 9) * 9;
-            dw_s[k * CCH + c] = __ldg(a.dw_w + (long)(c0 + c) * 9 + k);
-        }
-        for (int e = tid; e < cn; e += THREADS) {
-            sc_s[e] = __ldg(a.dw_scale + c0 + e);
-            sf_s[e] = __ldg(a.dw_shift + c0 + e);
-        }
-        for (int e = tid; e < CCH * OCP; e += THREADS) {
-            const int c = e / OCP, o = e - (e / OCP) * OCP;
-            w_s[e] = (c < cn && o < a.OC) ? __ldg(a.pw_w + (long)o * a.C + c0 + c) : 0.f;
-        }
-        __syncthreads();
-
-        // ---- phase 1: t[c][p] for this chunk, 8 channels per task
-        const int nvec = cn >> 3;
-        for (int task = tid; task < PIX * nvec; task += THREADS) {
-            const int p = task & (PIX - 1);
-            const int v = task >> 6;
-            const int4 q = pix_s[p];
-            float s[8];
+        for (int u = 0; u < 4; ++u) s[pp][u] = 0ull;
 #pragma unroll
-            for (int u = 0; u < 8; ++u) s[u] = 0.f;
-            if (q.w) {
+    for (int k = 0; k < 9; ++k) {
+        const long tap_off = ((long)(k / 3) * a.dh * a.W + (k % 3) * a.dw) * pix_bytes;
+        const float4 w0 = *reinterpret_cast<const float4*>(w_s + ((k * 2 + 0) * 8 + v) * 4);
+        const float4 w1 = *reinterpret_cast<const float4*>(w_s + ((k * 2 + 1) * 8 + v) * 4);
+        const uint64_t wp[4] = {f32x2_pack(w0.x, w0.y), f32x2_pack(w0.z, w0.w), f32x2_pack(w1.x, w1.y),
+                                f32x2_pack(w1.z, w1.w)};
 #pragma unroll
-                for (int i = 0; i < 3; ++i) {
-                    const int yy = q.y * a.sh - a.ph + i * a.dh;
-                    if (yy < 0 || yy >= a.H) continue;
-#pragma unroll
-                    for (int j = 0; j < 3; ++j) {
-                        const int xx = q.z * a.sw - a.pw + j * a.dw;
-                        if (xx < 0 || xx >= a.W) continue;
-                        float xv[8];
-                        load8<BF16>(a.x, ((long)(q.x * a.H + yy) * a.W + xx) * a.C + c0 + v * 8, xv);
-                        const float4 w0 = *reinterpret_cast<const float4*>(dw_s + (i * 3 + j) * CCH + v * 8);
-                        const float4 w1 = *reinterpret_cast<const float4*>(dw_s + (i * 3 + j) * CCH + v * 8 + 4);
-                        s[0] = fmaf(w0.x, xv[0], s[0]); s[1] = fmaf(w0.y, xv[1], s[1]);
-                        s[2] = fmaf(w0.z, xv[2], s[2]); s[3] = fmaf(w0.w, xv[3], s[3]);
-                        s[4] = fmaf(w1.x, xv[4], s[4]); s[5] = fmaf(w1.y, xv[5], s[5]);
-                        s[6] = fmaf(w1.z, xv[6], s[6]); s[7] = fmaf(w1.w, xv[7], s[7]);
-                    }
-                }
-            }
-#pragma unroll
-            for (int u = 0; u < 8; ++u) {
-                const int c = v * 8 + u;
-                t_s[c * TS + p] = q.w ? fmaxf(fmaf(sc_s[c], s[u], sf_s[c]), 0.f) : 0.f;
-            }
-        }
-        __syncthreads();
-
-        // ---- phase 2: acc[p][o] += sum_c t[c][p] * W2[o][c]
-#pragma unroll 4
-        for (int c = 0; c < cn; ++c) {
-            const float4 tv = *reinterpret_cast<const float4*>(t_s + c * TS + 4 * tp);
-            float wv[OCT];
-            if constexpr (OCT % 4 == 0) {
-#pragma unroll
-                for (int j = 0; j < OCT; j += 4) {
-                    const float4 w4 = *reinterpret_cast<const float4*>(w_s + c * OCP + to * OCT + j);
-                    wv[j] = w4.x; wv[j + 1] = w4.y; wv[j + 2] = w4.z; wv[j + 3] = w4.w;
-                }
+        for (int pp = 0; pp < DW_PPT; ++pp) {
+            const void* src = (valid[pp] >> k) & 1u ? static_cast<const void*>(base[pp] + tap_off)
+                                                   : static_cast<const void*>(g_zero32);
+            uint64_t xp[4];
+            if (BF16) {
+                const uint4 u4 = __ldg(static_cast<const uint4*>(src));
+                xp[0] = bf16x2_to_f32x2(u4.x); xp[1] = bf16x2_to_f32x2(u4.y);
+                xp[2] = bf16x2_to_f32x2(u4.z); xp[3] = bf16x2_to_f32x2(u4.w);
             } else {
-#pragma unroll
-                for (int j = 0; j < OCT; j += 2) {
-                    const float2 w2 = *reinterpret_cast<const float2*>(w_s + c * OCP + to * OCT + j);
-                    wv[j] = w2.x; wv[j + 1] = w2.y;
-                }
+                const float4 f0 = __ldg(static_cast<const float4*>(src));
+                const float4 f1 = __ldg(static_cast<const float4*>(src) + 1);
+                xp[0] = f32x2_pack(f0.x, f0.y); xp[1] = f32x2_pack(f0.z, f0.w);
+                xp[2] = f32x2_pack(f1.x, f1.y); xp[3] = f32x2_pack(f1.z, f1.w);
             }
 #pragma unroll
-            for (int j = 0; j < OCT; ++j) {
-                acc[0][j] = fmaf(tv.x, wv[j], acc[0][j]);
-                acc[1][j] = fmaf(tv.y, wv[j], acc[1][j]);
-                acc[2][j] = fmaf(tv.z, wv[j], acc[2][j]);
-                acc[3][j] = fmaf(tv.w, wv[j], acc[3][j]);
-            }
+            for (int u = 0; u < 4; ++u) s[pp][u] = f32x2_fma(wp[u], xp[u], s[pp][u]);
         }
     }
-
-    // ---- outputs
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-        const int m = m0 + 4 * tp + i;
+    for (int pp = 0; pp < DW_PPT; ++pp) {
+        const int m = blockIdx.x * DW_PIX + pp * DW_LANES + lane_p;
         if (m >= a.M) continue;
+        float r[8];
 #pragma unroll
-        for (int j = 0; j < OCT; ++j) {
-            const int o = to * OCT + j;
-            if (o >= a.OC) continue;
-            const float u = acc[i][j] + (a.pw_b ? __ldg(a.pw_b + o) : 0.f);
-            if (o < a.n_off)
-                a.offset[(long)m * a.n_off + o] = u;
-            else
-                a.mask[(long)m * a.n_msk + (o - a.n_off)] = 1.f / (1.f + __expf(-u));
+        for (int u = 0; u < 4; ++u) {
+            r[2 * u] = __uint_as_float((uint32_t)(s[pp][u] & 0xFFFFFFFFull));
+            r[2 * u + 1] = __uint_as_float((uint32_t)(s[pp][u] >> 32));
         }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) r[u] = fmaxf(fmaf(sc_s[v * 8 + u], r[u], sf_s[v * 8 + u]), 0.f);
+        float4* dst = reinterpret_cast<float4*>(a.t + (long)m * a.C + c0 + v * 8);
+        dst[0] = make_float4(r[0], r[1], r[2], r[3]);
+        dst[1] = make_float4(r[4], r[5], r[6], r[7]);
     }
 }
 
-template <int OCT>
-cudaError_t launch_oct(const BranchArgs& a, bool bf16, cudaStream_t stream) {
-    const int blocks = (a.M + PIX - 1) / PIX;
-    const size_t smem = sizeof(float) * ((size_t)CCH * TS + (size_t)CCH * 16 * OCT + 11 * CCH) +
-                        sizeof(int4) * PIX;
-    auto kern = bf16 ? offset_branch_kernel<true, OCT> : offset_branch_kernel<false, OCT>;
+// ------------------------------------------------------------------ 1x1 + sigmoid
+// [M x C] x [C x OC] on the tensor cores with mma.sync m16n8k8 TF32 and the 3xTF32 split
+// (a = a_hi + a_lo, hi = a truncated to tf32; a*b ~ a_hi*b_hi + a_hi*b_lo + a_lo*b_hi),
+// i.e. fp32-level accuracy.  Block = 8 warps over a 64-pixel tile: warp w owns m-tile
+// (w % 4) and every other 8-channel k-step of each chunk (w / 4); the two K halves are
+// added in shared memory at the end.  64-channel chunks of t and W2 are staged with
+// cp.async, double-buffered.
+constexpr int PW_WARPS = 8;
+constexpr int PW_PIX = 64;                 // pixels per block
+constexpr int PW_KC = 64;                  // channels per K chunk
+constexpr int PW_S = PW_KC + 4;            // smem row stride (floats): conflict-free fragments
+
+__device__ __forceinline__ void mma_tf32(float (&d)[4], const uint32_t (&a)[4], const uint32_t (&b)[2]) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b[0]), "r"(b[1]));
+}
+
+__device__ __forceinline__ void split_tf32(float f, uint32_t& hi, uint32_t& lo) {
+    hi = __float_as_uint(f) & 0xFFFFE000u;
+    lo = __float_as_uint(f - __uint_as_float(hi)) & 0xFFFFE000u;
+}
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool valid) {
+    const uint32_t s = smem_u32(smem);
+    const int n = valid ? 16 : 0;   // zero-fill when invalid
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
+}
+
+template <int NT>
+__global__ void __launch_bounds__(PW_WARPS * 32) pw_sigmoid_kernel(const BranchArgs a) {
+    constexpr int OCP = 8 * NT;
+    constexpr int STAGE = (PW_PIX + OCP) * PW_S;           // floats per stage
+    extern __shared__ __align__(16) float sm[];
+    const int tid = threadIdx.x;
+    const int warp = tid >> 5, lane = tid & 31;
+    const int g = lane >> 2, tq = lane & 3;
+    const int mt = warp & 3, kh = warp >> 2;
+    const int m0 = blockIdx.x * PW_PIX;
+    const int nchunks = (a.C + PW_KC - 1) / PW_KC;
+
+    auto stage_chunk = [&](int ch, int buf) {
+        float* ts = sm + buf * STAGE;
+        float* ws = ts + PW_PIX * PW_S;
+        const int c0 = ch * PW_KC;
+        for (int e = tid; e < (PW_PIX + OCP) * (PW_KC / 4); e += PW_WARPS * 32) {
+            const int r = e / (PW_KC / 4), q = e - r * (PW_KC / 4);
+            const int c = c0 + q * 4;
+            if (r < PW_PIX) {
+                const int m = m0 + r;
+                const bool ok = m < a.M && c < a.C;
+                cp_async16(ts + r * PW_S + q * 4, ok ? a.t + (long)m * a.C + c : a.t, ok);
+            } else {
+                const int o = r - PW_PIX;
+                const bool ok = o < a.OC && c < a.C;
+                cp_async16(ws + o * PW_S + q * 4, ok ? a.pw_w + (long)o * a.C + c : a.pw_w, ok);
+            }
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+
+    float acc[NT][4];
+#pragma unroll
+    for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc[nt][u] = 0.f;
+
+    stage_chunk(0, 0);
+    for (int ch = 0; ch < nchunks; ++ch) {
+        if (ch + 1 < nchunks) {
+            stage_chunk(ch + 1, (ch + 1) & 1);
+            asm volatile("cp.async.wait_group 1;" ::: "memory");
+        } else {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
+        __syncthreads();
+        const float* ts = sm + (ch & 1) * STAGE + (mt * 16) * PW_S;
+        const float* ws = sm + (ch & 1) * STAGE + PW_PIX * PW_S;
+#pragma unroll
+        for (int k0 = kh * 8; k0 < PW_KC; k0 += 16) {
+            uint32_t ahi[4], alo[4];
+            split_tf32(ts[g * PW_S + k0 + tq], ahi[0], alo[0]);
+            split_tf32(ts[(g + 8) * PW_S + k0 + tq], ahi[1], alo[1]);
+            split_tf32(ts[g * PW_S + k0 + tq + 4], ahi[2], alo[2]);
+            split_tf32(ts[(g + 8) * PW_S + k0 + tq + 4], ahi[3], alo[3]);
+#pragma unroll
+            for (int nt = 0; nt < NT; ++nt) {
+                uint32_t bhi[2], blo[2];
+                split_tf32(ws[(nt * 8 + g) * PW_S + k0 + tq], bhi[0], blo[0]);
+                split_tf32(ws[(nt * 8 + g) * PW_S + k0 + tq + 4], bhi[1], blo[1]);
+                mma_tf32(acc[nt], alo, bhi);
+                mma_tf32(acc[nt], ahi, blo);
+                mma_tf32(acc[nt], ahi, bhi);
+            }
+        }
+        __syncthreads();   // buffer (ch & 1) is refilled two iterations later
+    }
+    // reduce the two K halves: warps 4..7 hand their accumulators to warps 0..3
+    float* red = sm;   // reuse stage memory: [4 warps][NT][4][32]
+    if (kh == 1) {
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int u = 0; u < 4; ++u) red[((mt * NT + nt) * 4 + u) * 32 + lane] = acc[nt][u];
+    }
+    __syncthreads();
+    if (kh == 1) return;
+#pragma unroll
+    for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc[nt][u] += red[((mt * NT + nt) * 4 + u) * 32 + lane];
+    // D fragment: rows g and g+8, columns 2tq and 2tq+1 of each n-tile
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        const int m = m0 + mt * 16 + g + h * 8;
+        if (m >= a.M) continue;
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+                const int o = nt * 8 + 2 * tq + u;
+                if (o >= a.OC) continue;
+                const float val = acc[nt][h * 2 + u] + (a.pw_b ? __ldg(a.pw_b + o) : 0.f);
+                if (o < a.n_off)
+                    a.offset[(long)m * a.n_off + o] = val;
+                else
+                    a.mask[(long)m * a.n_msk + (o - a.n_off)] = 1.f / (1.f + __expf(-val));
+            }
+    }
+}
+
+template <int NT>
+cudaError_t launch_pw(const BranchArgs& a, cudaStream_t stream) {
+    constexpr int OCP = 8 * NT;
+    size_t smem = sizeof(float) * 2 * (PW_PIX + OCP) * PW_S;
+    const size_t red = sizeof(float) * 4 * NT * 4 * 32;
+    if (red > smem) smem = red;
+    auto kern = pw_sigmoid_kernel<NT>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    kern<<<blocks, THREADS, smem, stream>>>(a);
+    kern<<<(a.M + PW_PIX - 1) / PW_PIX, PW_WARPS * 32, smem, stream>>>(a);
     return cudaGetLastError();
 }
 
 }  // namespace
 
+size_t offset_branch_workspace(int M, int C) { return (size_t)M * C * sizeof(float); }
+
 cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W, int C,
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                 float* offset, float* mask, cudaStream_t stream) {
+                                 float* offset, float* mask, float* t_ws, cudaStream_t stream) {
     BranchArgs a;
     a.x = x; a.dw_w = dw_w; a.dw_scale = dw_scale; a.dw_shift = dw_shift;
-    a.pw_w = pw_w; a.pw_b = pw_b; a.offset = offset; a.mask = mask;
+    a.pw_w = pw_w; a.pw_b = pw_b; a.t = t_ws; a.offset = offset; a.mask = mask;
     a.N = N; a.H = H; a.W = W; a.C = C; a.Ho = Ho; a.Wo = Wo; a.M = N * Ho * Wo;
     a.sh = s_h; a.sw = s_w; a.ph = p_h; a.pw = p_w; a.dh = d_h; a.dw = d_w;
     a.n_off = 2 * G * K * K;
     a.n_msk = with_mask ? G * K * K : 0;
     a.OC = a.n_off + a.n_msk;
-    if (a.OC <= 32) return launch_oct<2>(a, x_bf16, stream);
-    if (a.OC <= 64) return launch_oct<4>(a, x_bf16, stream);
-    if (a.OC <= 128) return launch_oct<8>(a, x_bf16, stream);
-    if (a.OC <= 256) return launch_oct<16>(a, x_bf16, stream);
-    return cudaErrorInvalidValue;   // api.cu maps this to DEFCON_ERR_LIMIT
+    if (a.OC > 256) return cudaErrorInvalidValue;   // api.cu maps this to DEFCON_ERR_LIMIT
+    dim3 g1((a.M + DW_PIX - 1) / DW_PIX, (C + DW_CH - 1) / DW_CH);
+    if (x_bf16)
+        dw_bn_relu_kernel<true><<<g1, DW_THREADS, 0, stream>>>(a);
+    else
+        dw_bn_relu_kernel<false><<<g1, DW_THREADS, 0, stream>>>(a);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    if (a.OC <= 32) return launch_pw<4>(a, stream);
+    if (a.OC <= 64) return launch_pw<8>(a, stream);
+    if (a.OC <= 128) return launch_pw<16>(a, stream);
+    return launch_pw<32>(a, stream);
 }
 
 }  // namespace defcon

@@ -89,12 +89,18 @@ def test_dcn_forward_limit(lib):
 def test_offset_branch_validation(lib):
     V = ctypes.c_void_p
     args = [V(FAKE), 1, 8, 8, 16, 1, V(FAKE), V(FAKE), V(FAKE), V(FAKE), V(FAKE), 3]
-    assert lib.defcon_offset_dw_conv(*args, _conv(), V(0), V(FAKE), None) == 1      # offset NULL
-    assert lib.defcon_offset_dw_conv(*args, _conv(), V(FAKE + 4), V(FAKE), None) == 3
-    assert lib.defcon_offset_dw_conv(*args, _conv(offset_groups=64), V(FAKE), V(FAKE), None) == 5
+    big = 1 << 30
+    assert lib.defcon_offset_dw_conv(*args, _conv(), V(0), V(FAKE), V(FAKE), big, None) == 1  # offset NULL
+    assert lib.defcon_offset_dw_conv(*args, _conv(), V(FAKE + 4), V(FAKE), V(FAKE), big, None) == 3
+    assert lib.defcon_offset_dw_conv(*args, _conv(offset_groups=64), V(FAKE), V(FAKE), V(FAKE), big,
+                                     None) == 5
+    assert lib.defcon_offset_dw_conv(*args, _conv(), V(FAKE), V(FAKE), V(FAKE), 16, None) == 5  # ws
     bad = list(args)
     bad[1] = 0
-    assert lib.defcon_offset_dw_conv(*bad, _conv(), V(FAKE), V(FAKE), None) == 1
+    assert lib.defcon_offset_dw_conv(*bad, _conv(), V(FAKE), V(FAKE), V(FAKE), big, None) == 1
+    out = ctypes.c_size_t(0)
+    assert lib.defcon_offset_workspace_size(1, 8, 8, 16, 3, _conv(), ctypes.byref(out)) == 0
+    assert out.value == 8 * 8 * 16 * 4
 
 
 def test_workspace_size_and_layer_size(lib):

@@ -1,0 +1,64 @@
+"""Time the fused DCN kernel alone on a BASELINE config under DEFCON_PROBE settings.
+
+Used to locate the bottleneck: probe bit 1 drops the
+MMAs, bit 2 the gathers, bit 4 the lerp.  Prints one line per (config, probe).
+"""
+import json
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from defcon_workloads import configs, inputs  # noqa: E402
+import paper_conf_ipps_jayaweeralwrk24_b200 as d  # noqa: E402
+
+
+def time_cfg(c, probe, reps=200):
+    os.environ["DEFCON_PROBE"] = str(probe)
+    dev = torch.device("cuda")
+    L = inputs.gen_layer(c)
+    dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
+    x = torch.from_numpy(L["x"]).to(dev, dt)
+    off = torch.from_numpy(L["offset"]).to(dev)
+    msk = torch.from_numpy(L["mask"]).to(dev)
+    w = torch.from_numpy(L["weight"]).to(dev, dt)
+    b = torch.from_numpy(L["bias"]).to(dev)
+    y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
+    ws = torch.empty(max(16, d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K,
+                                                         c.stride, c.pad, c.dil, c.G, dt)),
+                     dtype=torch.uint8, device=dev)
+    fn = lambda: d.defcon_dcn_forward(x, off, msk, w, b, stride=c.stride, pad=c.pad, dil=c.dil,
+                                      offset_groups=c.G, y=y, workspace=ws)
+    for _ in range(5):
+        fn()
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(10):
+            fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps // 10):
+        g.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    us = e0.elapsed_time(e1) * 1e3 / reps
+    return us, configs.contraction_flops(c) / (us * 1e-6) / 1e12
+
+
+if __name__ == "__main__":
+    names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["yolact_r101_c4_v2"]
+    probes = [int(p) for p in sys.argv[2].split(",")] if len(sys.argv) > 2 else [0, 1, 2, 4, 6, 7]
+    d.load_library()
+    for n in names:
+        if ":" in n:          # name:N override, e.g. yolact_r101_c4_v2:8
+            base, nn = n.split(":")
+            c = configs.SINGLE_LAYER[base].replace(N=int(nn))
+        else:
+            c = configs.SINGLE_LAYER[n]
+        for p in probes:
+            us, tf = time_cfg(c, p)
+            print(json.dumps({"config": n, "probe": p, "us": round(us, 2), "tflops": round(tf, 1)}))
