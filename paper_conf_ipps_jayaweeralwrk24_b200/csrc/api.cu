@@ -95,8 +95,13 @@ static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, 
         return fail(DEFCON_ERR_INVALID_ARG, "bad sampler");
     if (fp32_mode != DEFCON_FP32_3XTF32 && fp32_mode != DEFCON_FP32_SIMT)
         return fail(DEFCON_ERR_INVALID_ARG, "bad fp32_mode");
-    if (sampler == DEFCON_SAMPLER_TEX)
-        return fail(DEFCON_ERR_UNSUPPORTED, "texture sampler not built in this version");
+    if (sampler == DEFCON_SAMPLER_TEX) {
+        if (dtype != DEFCON_BF16 || !dcn_tc_bf16_supported(g))
+            return fail(DEFCON_ERR_UNSUPPORTED,
+                        "texture sampler is built for the bf16 tensor-core path (Cin/G %% 64 == 0)");
+        *path = Path::TC_BF16;
+        return DEFCON_OK;
+    }
     if (dtype == DEFCON_BF16) {
         *path = dcn_tc_bf16_supported(g) ? Path::TC_BF16 : Path::SIMT_BF16;
     } else {
@@ -221,7 +226,12 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     Path path;
     rc = select_path(g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
-    (void)tex_plan;
+    TexPlan* tp = nullptr;
+    if (sampler == DEFCON_SAMPLER_TEX) {
+        tp = reinterpret_cast<TexPlan*>(tex_plan);
+        if (!tex_plan_matches(tp, N, H, W, Cin, dtype == DEFCON_BF16))
+            return fail(DEFCON_ERR_INVALID_ARG, "tex_plan missing or made for another shape/dtype");
+    }
     const size_t need = path_workspace(g, path);
     if (need > 0 && (workspace == nullptr || workspace_bytes < need))
         return fail(DEFCON_ERR_LIMIT, "workspace of %zu bytes < required %zu", workspace_bytes, need);
@@ -229,8 +239,12 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     const char* detail = "dcn launch";
+    if (tp) {
+        e = tex_plan_stage(tp, x, st);
+        if (e != cudaSuccess) return cuda_fail(e, "texture staging launch");
+    }
     switch (path) {
-        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, workspace, workspace_bytes, st, &detail); break;
+        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, workspace, workspace_bytes, tp, st, &detail); break;
         case Path::SIMT_BF16: e = launch_dcn_simt(g, p, true, st); break;
         default: e = launch_dcn_simt(g, p, false, st); break;
     }
@@ -320,19 +334,37 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
 
 int defcon_tex_plan_create(int N, int H, int W, int Cin, int dtype, defcon_tex_plan_t* plan) {
     g_detail[0] = 0;
-    (void)N; (void)H; (void)W; (void)Cin; (void)dtype;
-    if (plan) *plan = nullptr;
-    return fail(DEFCON_ERR_UNSUPPORTED, "texture sampler not built in this version");
+    if (!plan) return fail(DEFCON_ERR_INVALID_ARG, "plan is NULL");
+    *plan = nullptr;
+    if (N <= 0 || H <= 0 || W <= 0 || Cin <= 0) return fail(DEFCON_ERR_INVALID_ARG, "sizes must be positive");
+    if (dtype != DEFCON_F32 && dtype != DEFCON_BF16) return fail(DEFCON_ERR_INVALID_ARG, "bad dtype");
+    if (Cin % 4 != 0) return fail(DEFCON_ERR_UNSUPPORTED, "texture plan needs Cin %% 4 == 0");
+    int dev = 0, max_layers = 2048, max_w = 32768, max_h = 32768;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&max_layers, cudaDevAttrMaxTexture2DLayeredLayers, dev);
+    cudaDeviceGetAttribute(&max_w, cudaDevAttrMaxTexture2DLayeredWidth, dev);
+    cudaDeviceGetAttribute(&max_h, cudaDevAttrMaxTexture2DLayeredHeight, dev);
+    if (Cin / 4 > max_layers || W > max_w || (long)N * (H + 1) > max_h)
+        return fail(DEFCON_ERR_LIMIT, "layered texture limits exceeded (layers %d / %d, %d x %ld texels)",
+                    Cin / 4, max_layers, W, (long)N * (H + 1));
+    TexPlan* p = nullptr;
+    cudaError_t e = tex_plan_create(N, H, W, Cin, dtype == DEFCON_BF16, &p);
+    if (e != cudaSuccess) return cuda_fail(e, "texture plan allocation");
+    *plan = reinterpret_cast<defcon_tex_plan_t>(p);
+    return DEFCON_OK;
 }
 
 int defcon_tex_plan_destroy(defcon_tex_plan_t plan) {
-    (void)plan;
+    tex_plan_destroy(reinterpret_cast<TexPlan*>(plan));
     return DEFCON_OK;
 }
 
 int defcon_tex_filter_probe(const float* px, const float* py, float* out, int n, void* stream) {
-    (void)px; (void)py; (void)out; (void)n; (void)stream;
-    return fail(DEFCON_ERR_UNSUPPORTED, "texture sampler not built in this version");
+    g_detail[0] = 0;
+    if (!px || !py || !out || n <= 0) return fail(DEFCON_ERR_INVALID_ARG, "bad probe arguments");
+    cudaError_t e = tex_filter_probe(px, py, out, n, static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "texture filter probe");
+    return DEFCON_OK;
 }
 
 }  // extern "C"

@@ -58,7 +58,7 @@ struct TcArgs {
     int ipt;               // k-iterations per tile = (Cin / BK) * KK
     int n_tiles_n;         // tiles along Cout
     long long total_iters; // num_tiles * ipt
-    int probe;             // 0 in production; bit flags disable parts for bottleneck probes
+    unsigned long long tex;          // DEFCON_SAMPLER_TEX: stacked-image texture object, else 0
 };
 
 template <int BLOCK_N>
@@ -92,8 +92,38 @@ struct Segment {
 // channel 0 of each of the 4 bilinear corners and the 4 corner weights with the mask
 // folded in.  Corners outside the image get weight 0 and the harmless in-bounds
 // offset 0 (R8).
+template <bool TEX>
 __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int row, int tap, int g,
                                                  uint8_t* meta) {
+    if constexpr (TEX) {
+        // texture sampler: unnormalised texel coordinates (texel centres at +0.5, R7) in the
+        // stacked-image texture (image n occupies rows n*(H+1) .. n*(H+1)+H-1, row
+        // n*(H+1)+H is zero) and the mask.  Clamping to [-1, H] x [-1, W] keeps samples
+        // beyond the image on zero texels.
+        float4 c = make_float4(-4.f, -4.f, 0.f, 0.f);
+        const int m = m0 + row;
+        if (m < a.M) {
+            const int hw = a.Ho * a.Wo;
+            const int n = m / hw;
+            const int rem = m - n * hw;
+            const int ho = rem / a.Wo;
+            const int wo = rem - ho * a.Wo;
+            const int i = tap / a.Kw;
+            const int j = tap - i * a.Kw;
+            const long pix = (long)m * a.G + g;
+            const float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tap) * 2));
+            const float mk = a.mask ? __ldg(a.mask + pix * a.KK + tap) : 1.0f;
+            const float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
+            const float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
+            if (px == px && py == py) {
+                c.x = fminf(fmaxf(px, -1.0f), (float)a.W) + 0.5f;
+                c.y = (float)(n * (a.H + 1)) + fminf(fmaxf(py, -1.0f), (float)a.H) + 0.5f;
+                c.z = mk;
+            }
+        }
+        *reinterpret_cast<float4*>(meta + (row * a.KK + tap) * META_ENTRY) = c;
+        return;
+    }
     uint4 off = make_uint4(0u, 0u, 0u, 0u);
     float4 wt = make_float4(0.f, 0.f, 0.f, 0.f);
     const int m = m0 + row;
@@ -139,16 +169,11 @@ struct RowLoad {
     float4 w;
 };
 
-__device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr,
-                                          int probe = 0) {
+__device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr) {
     const uint4 o = ld_shared_v4(meta_addr);
     const uint4 wb = ld_shared_v4(meta_addr + 16);
     L.w = make_float4(__uint_as_float(wb.x), __uint_as_float(wb.y), __uint_as_float(wb.z),
                       __uint_as_float(wb.w));
-    if (probe & 2) {   // probe: no gathers
-        L.v[0] = L.v[1] = L.v[2] = L.v[3] = o;
-        return;
-    }
     L.v[0] = ldg_nc_v4(add_u32(xbase, o.x));
     L.v[1] = ldg_nc_v4(add_u32(xbase, o.y));
     L.v[2] = ldg_nc_v4(add_u32(xbase, o.z));
@@ -172,6 +197,49 @@ __device__ __forceinline__ void lerp_store_row(const RowLoad& L, uint32_t dst) {
     st_shared_v4(dst, f32x2_to_bf16x2(acc[0]), f32x2_to_bf16x2(acc[1]), f32x2_to_bf16x2(acc[2]),
                  f32x2_to_bf16x2(acc[3]));
 }
+
+// Texture-sampler counterpart of RowLoad: 8 channels = 2 texels of 4 channels, already
+// bilinearly filtered by the texture unit, and the mask.
+struct TexLoad {
+    float4 t0, t1;
+    float m;
+};
+
+__device__ __forceinline__ void issue_row_tex(TexLoad& L, cudaTextureObject_t tex, int layer,
+                                              uint32_t meta_addr) {
+    const uint4 c = ld_shared_v4(meta_addr);
+    const float fx = __uint_as_float(c.x), fy = __uint_as_float(c.y);
+    L.m = __uint_as_float(c.z);
+    L.t0 = tex2DLayered<float4>(tex, fx, fy, layer);
+    L.t1 = tex2DLayered<float4>(tex, fx, fy, layer + 1);
+}
+
+__device__ __forceinline__ void tex_store_row(const TexLoad& L, uint32_t dst) {
+    st_shared_v4(dst, pack_bf16x2(L.t0.x * L.m, L.t0.y * L.m), pack_bf16x2(L.t0.z * L.m, L.t0.w * L.m),
+                 pack_bf16x2(L.t1.x * L.m, L.t1.y * L.m), pack_bf16x2(L.t1.z * L.m, L.t1.w * L.m));
+}
+
+// Sampler policy: LDG gathers + software lerp, or texture fetches with hardware filtering.
+template <bool TEX>
+struct Sampler;
+template <>
+struct Sampler<false> {
+    using Load = RowLoad;
+    static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
+                                                 uint32_t meta) {
+        issue_row(L, xb, meta);
+    }
+    static __device__ __forceinline__ void store(const Load& L, uint32_t dst) { lerp_store_row(L, dst); }
+};
+template <>
+struct Sampler<true> {
+    using Load = TexLoad;
+    static __device__ __forceinline__ void issue(Load& L, const uint8_t*, unsigned long long tex, int layer,
+                                                 uint32_t meta) {
+        issue_row_tex(L, (cudaTextureObject_t)tex, layer, meta);
+    }
+    static __device__ __forceinline__ void store(const Load& L, uint32_t dst) { tex_store_row(L, dst); }
+};
 
 // CTA range -> segments helper (every role walks the same sequence).
 __device__ __forceinline__ int count_segments(const TcArgs& a, long long it_begin, long long it_end) {
@@ -197,7 +265,6 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
                                                  int bar_id, int nthr, bool leader, int* fix_flag,
                                                  long long T, int nct) {
     constexpr int CH = NCOLS >= 32 ? 32 : 16;
-    if (a.probe & 32) return;   // probe: no epilogue
     const int m0 = (sg.tile / a.n_tiles_n) * BM;
     const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
     const int row = m0 + r;
@@ -301,7 +368,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
     }
 }
 
-template <int BLOCK_N, int STAGES>
+template <int BLOCK_N, int STAGES, bool TEX>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const TcArgs a) {
     using Cfg = TcCfg<BLOCK_N>;
@@ -361,6 +428,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             dst[p] = row * 128 + ((cvec ^ (row & 7)) << 4);
             mrow[p] = meta_s + row * a.KK * META_ENTRY;
         }
+        using Smp = Sampler<TEX>;
         int q = 0;                           // running k-iteration (stage) counter
         for (int j = 0; j < nseg; ++j) {
             const Segment sg = segment_j(a, it_begin, it_end, j);
@@ -369,13 +437,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             int tap = sg.kb - chunk * a.KK;
             int g = (chunk * BK) / a.Cg;
             named_bar_sync(1, NPT);          // previous table no longer read
-            if (!(a.probe & 16) || j == 0)
-                for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry(a, m0, e / a.KK, e % a.KK, g, meta);
+            for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry<TEX>(a, m0, e / a.KK, e % a.KK, g, meta);
             named_bar_sync(1, NPT);
+            // position of this thread's 8 channels: byte pointer (LDG) / texture layer (TEX)
             const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + cvec * 8) * 2;
-            RowLoad L[ROWS];
+            int layer = chunk * (BK / 4) + cvec * 2;
+            typename Smp::Load L[ROWS];
 #pragma unroll
-            for (int p = 0; p < ROWS; ++p) issue_row(L[p], xb, mrow[p] + tap * META_ENTRY, a.probe);
+            for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], xb, a.tex, layer, mrow[p] + tap * META_ENTRY);
             for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                 int ntap = tap + 1, nchunk = chunk;
                 if (ntap == a.KK) { ntap = 0; ++nchunk; }
@@ -384,18 +453,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 if (has_next && nchunk != chunk) ng = (nchunk * BK) / a.Cg;
                 const bool prefetch = has_next && ng == g;
                 const uint8_t* nxb = nchunk != chunk ? xb + BK * 2 : xb;
+                const int nlayer = nchunk != chunk ? layer + BK / 4 : layer;
 
                 const int s = q % STAGES;
                 mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
                 const uint32_t stage = a_s + s * A_STAGE_BYTES;
 #pragma unroll
                 for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
-                    if (a.probe & 4)   // probe: no lerp, store one corner
-                        st_shared_v4(stage + dst[p], L[p].v[0].x ^ L[p].v[1].x, L[p].v[2].y ^ L[p].v[3].y,
-                                     L[p].v[0].z, L[p].v[1].w);
-                    else
-                        lerp_store_row(L[p], stage + dst[p]);
-                    if (prefetch) issue_row(L[p], nxb, mrow[p] + ntap * META_ENTRY, a.probe);
+                    Smp::store(L[p], stage + dst[p]);
+                    if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
                 }
                 fence_proxy_async_smem();
                 __syncwarp();
@@ -404,12 +470,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 if (has_next && !prefetch) {          // offset group changes: new table
                     named_bar_sync(1, NPT);
                     for (int e = t; e < BM * a.KK; e += NPT)
-                        build_meta_entry(a, m0, e / a.KK, e % a.KK, ng, meta);
+                        build_meta_entry<TEX>(a, m0, e / a.KK, e % a.KK, ng, meta);
                     named_bar_sync(1, NPT);
                     g = ng;
 #pragma unroll
-                    for (int p = 0; p < ROWS; ++p) issue_row(L[p], nxb, mrow[p] + ntap * META_ENTRY);
+                    for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
                 }
+                layer = nlayer;
                 tap = ntap;
                 chunk = nchunk;
                 xb = nxb;
@@ -463,11 +530,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                     const int s = q % STAGES;
                     mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
-                    if (a.probe & 8) {    // probe: no weight TMA
-                        mbar_arrive(&full_b[s]);
-                        if (++tap == a.KK) { tap = 0; ++chunk; }
-                        continue;
-                    }
                     mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
                     const int kd = tap * a.Cin + chunk * BK;
 #pragma unroll
@@ -504,9 +566,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         for (int h = 0; h < Cfg::N_MMA; ++h) {
                             const uint64_t bdesc =
                                 make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
-                            if (!(a.probe & 1))   // probe: no MMA
-                                mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
-                                            (kt != sg.kb || kk != 0) ? 1u : 0u);
+                            mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
+                                        (kt != sg.kb || kk != 0) ? 1u : 0u);
                         }
                     }
                     mma_commit(&empty[s]);
@@ -575,7 +636,7 @@ size_t workspace_impl(const DcnGeom& g) {
 
 template <int BLOCK_N, int STAGES>
 cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
-                        cudaStream_t stream, const char** detail) {
+                        const TexPlan* tex, cudaStream_t stream, const char** detail) {
     using Cfg = TcCfg<BLOCK_N>;
     auto plan = make_plan<BLOCK_N>(g);
     if (ws_bytes < plan.counters_bytes + plan.partial_bytes || ws == nullptr) {
@@ -615,8 +676,7 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.ipt = plan.ipt;
     a.n_tiles_n = plan.n_tiles_n;
     a.total_iters = plan.total;
-    a.probe = 0;
-    if (const char* env = getenv("DEFCON_PROBE")) a.probe = atoi(env);
+    a.tex = tex ? tex_plan_texture(tex) : 0ull;
 
     cudaError_t e = cudaMemsetAsync(a.counters, 0, plan.counters_bytes, stream);
     if (e != cudaSuccess) {
@@ -625,7 +685,8 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     }
     const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + (size_t)BM * g.KK * META_ENTRY +
                         (3 * STAGES + 2 * Cfg::NBUF) * 8 + 32;
-    auto kern = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES>;
+    auto kern = tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, true>
+                    : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, false>;
     e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) {
         *detail = "cudaFuncSetAttribute(MaxDynamicSharedMemorySize) failed";
@@ -655,11 +716,11 @@ size_t dcn_tc_bf16_workspace(const DcnGeom& g) {
 }
 
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
-                               cudaStream_t stream, const char** detail) {
-    if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, stream, detail);
-    if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, stream, detail);
-    if (g.Cout <= 256) return launch_impl<256, 3>(g, p, ws, ws_bytes, stream, detail);
-    return launch_impl<512, 2>(g, p, ws, ws_bytes, stream, detail);
+                               const TexPlan* tex, cudaStream_t stream, const char** detail) {
+    if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, stream, detail);
+    if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, stream, detail);
+    if (g.Cout <= 256) return launch_impl<256, 3>(g, p, ws, ws_bytes, tex, stream, detail);
+    return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, stream, detail);
 }
 
 }  // namespace defcon

@@ -41,8 +41,18 @@ cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaS
 // ---- step 2, fused gather + tcgen05 implicit GEMM, bf16 (dcn_tc_bf16.cu)
 bool dcn_tc_bf16_supported(const DcnGeom& g);
 size_t dcn_tc_bf16_workspace(const DcnGeom& g);   // stream-K counters + fp32 partials
+struct TexPlan;
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
-                               cudaStream_t stream, const char** detail);
+                               const TexPlan* tex, cudaStream_t stream, const char** detail);
+
+// ---- texture sampler resources (tex_plan.cu)
+struct TexPlan;
+cudaError_t tex_plan_create(int N, int H, int W, int C, bool half, TexPlan** out);
+void tex_plan_destroy(TexPlan* p);
+bool tex_plan_matches(const TexPlan* p, int N, int H, int W, int C, bool half);
+unsigned long long tex_plan_texture(const TexPlan* p);            // texture object handle
+cudaError_t tex_plan_stage(const TexPlan* p, const void* x, cudaStream_t stream);
+cudaError_t tex_filter_probe(const float* px, const float* py, float* out, int n, cudaStream_t stream);
 
 // ---- driver entry point for cuTensorMapEncodeTiled (api.cu)
 typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,

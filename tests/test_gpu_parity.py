@@ -43,12 +43,13 @@ def to_dev(a, dtype, dev):
     return None if a is None else torch.from_numpy(np.ascontiguousarray(a)).to(dev, dtype)
 
 
-def run_dcn(d, dev, c, L, sampler="ldg", fp32_mode="simt"):
+def run_dcn(d, dev, c, L, sampler="ldg", fp32_mode="simt", tex_plan=None):
     dt = TDT[c.dtype]
     y = d.defcon_dcn_forward(to_dev(L["x"], dt, dev), to_dev(L["offset"], torch.float32, dev),
                              to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], dt, dev),
                              to_dev(L["bias"], torch.float32, dev), stride=c.stride, pad=c.pad,
-                             dil=c.dil, offset_groups=c.G, sampler=sampler, fp32_mode=fp32_mode)
+                             dil=c.dil, offset_groups=c.G, sampler=sampler, fp32_mode=fp32_mode,
+                             tex_plan=tex_plan)
     torch.cuda.synchronize()
     return y.float().cpu().numpy()
 
@@ -194,3 +195,49 @@ def test_layer_chain_and_host_entry(oracle_mod, d, dev):
     idx = np.unique(np.concatenate([np.arange(200), r.integers(0, c.M, 300)]))
     ref = oracle_mod.dcn_pixels(x, ro, w, idx, b, mask=rm)
     assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
+
+
+# ---------------------------------------------------------------- texture sampler
+def tex_mode(d, dev):
+    """Measure the texture unit's bilinear fraction handling (reading R14): sample a 2x2
+    float texture [[0,0],[0,1]] at px = 0.5 + f, py = 1.5 so the result is alpha_q(f)."""
+    f = torch.arange(0, 4096, dtype=torch.float32, device=dev) / 4096.0
+    px = (0.5 + f).contiguous()
+    py = torch.full_like(px, 1.5)
+    out = d.defcon_tex_filter_probe(px, py).cpu().numpy().astype(np.float64)
+    f = f.cpu().numpy().astype(np.float64)
+    q = out * 256.0
+    assert np.max(np.abs(q - np.round(q))) < 1e-6, "fraction is not on a 1/256 grid"
+    if np.all(np.abs(out - np.floor(f * 256.0 + 0.5) / 256.0) < 1e-7):
+        return "round"
+    if np.all(np.abs(out - np.floor(f * 256.0) / 256.0) < 1e-7):
+        return "trunc"
+    raise AssertionError("texture fraction neither rounds nor truncates to 1/256")
+
+
+def test_tex_filter_fixed_point(d, dev):
+    mode = tex_mode(d, dev)
+    print("texture filter fraction mode:", mode)
+
+
+@pytest.mark.parametrize("c", [small("tex_c128", Cout=128), small("tex_v1", modulated=False),
+                               small("tex_g2", G=2), small("tex_g2_v1", G=2, modulated=False),
+                               configs.C5.replace(N=2), small("tex_s2", stride=2, H=23, W=21)],
+                         ids=lambda c: c.name)
+def test_tex_sampler_parity(oracle_mod, d, dev, c):
+    """TEX sampler: equals the texture-model oracle (fp16 texels, 1/256 fractions,
+    measured rounding) to bf16 precision, and the exact oracle within the 5e-3 gate."""
+    mode = tex_mode(d, dev)
+    L = inputs.gen_layer(c)
+    plan = d.TexPlan(c.N, c.H, c.W, c.Cin, torch.bfloat16)
+    y = run_dcn(d, dev, c, dict(L), sampler="tex", tex_plan=plan)
+    x16 = inputs.round_to(L["x"], "f16")
+    refq = oracle_mod.dcn_forward_texq(x16, L["offset"], L["weight"], L["bias"], mask=L["mask"],
+                                       stride=c.stride, pad=c.pad, dil=c.dil, G=c.G, quant=mode)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
+                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    e_q, e_x = normwise(y, refq), normwise(y, ref)
+    print(f"{c.name}: vs texture model {e_q:.2e}, vs exact oracle {e_x:.2e}")
+    assert e_q < 1e-2
+    assert e_x < 5e-3
+    plan.close()

@@ -1,13 +1,13 @@
-"""Time the fused DCN kernel alone on a BASELINE config under DEFCON_PROBE settings.
+"""Time the fused DCN kernel alone (graph-replayed launches) per config and sampler.
 
-Used to locate the bottleneck: probe bit 1 drops the
-MMAs, bit 2 the gathers, bit 4 the lerp.  Prints one line per (config, probe).
+  python tools/probe_dcn.py [config[:N],...] [ldg,tex]
+Prints one JSON line per (config, sampler): microseconds per launch (incl. the texture
+staging pass for the TEX sampler) and contraction TFLOP/s.
 """
 import json
 import os
 import sys
 
-import numpy as np
 import torch
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -15,8 +15,7 @@ from defcon_workloads import configs, inputs  # noqa: E402
 import paper_conf_ipps_jayaweeralwrk24_b200 as d  # noqa: E402
 
 
-def time_cfg(c, probe, reps=200):
-    os.environ["DEFCON_PROBE"] = str(probe)
+def time_cfg(c, sampler, reps=200):
     dev = torch.device("cuda")
     L = inputs.gen_layer(c)
     dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
@@ -27,10 +26,12 @@ def time_cfg(c, probe, reps=200):
     b = torch.from_numpy(L["bias"]).to(dev)
     y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
     ws = torch.empty(max(16, d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K,
-                                                         c.stride, c.pad, c.dil, c.G, dt)),
+                                                         c.stride, c.pad, c.dil, c.G, dt, sampler)),
                      dtype=torch.uint8, device=dev)
+    plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler == "tex" else None
     fn = lambda: d.defcon_dcn_forward(x, off, msk, w, b, stride=c.stride, pad=c.pad, dil=c.dil,
-                                      offset_groups=c.G, y=y, workspace=ws)
+                                      offset_groups=c.G, y=y, workspace=ws, sampler=sampler,
+                                      tex_plan=plan)
     for _ in range(5):
         fn()
     g = torch.cuda.CUDAGraph()
@@ -51,7 +52,7 @@ def time_cfg(c, probe, reps=200):
 
 if __name__ == "__main__":
     names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["yolact_r101_c4_v2"]
-    probes = [int(p) for p in sys.argv[2].split(",")] if len(sys.argv) > 2 else [0, 1, 2, 4, 6, 7]
+    samplers = sys.argv[2].split(",") if len(sys.argv) > 2 else ["ldg", "tex"]
     d.load_library()
     for n in names:
         if ":" in n:          # name:N override, e.g. yolact_r101_c4_v2:8
@@ -59,6 +60,6 @@ if __name__ == "__main__":
             c = configs.SINGLE_LAYER[base].replace(N=int(nn))
         else:
             c = configs.SINGLE_LAYER[n]
-        for p in probes:
-            us, tf = time_cfg(c, p)
-            print(json.dumps({"config": n, "probe": p, "us": round(us, 2), "tflops": round(tf, 1)}))
+        for smp in samplers:
+            us, tf = time_cfg(c, smp)
+            print(json.dumps({"config": n, "sampler": smp, "us": round(us, 2), "tflops": round(tf, 1)}))
