@@ -29,12 +29,12 @@ import torch
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-from defcon_workloads import configs, inputs  # noqa: E402
+from defcon_workloads import configs, inputs, sharding  # noqa: E402
 
 WORKLOAD = configs.C4
 L2_BYTES = 126 * 2**20
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
-NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary.json")
+NCU_SUMMARY_GLOB = os.path.join(ROOT, "profiles", "r*_ncu_summary.json")
 
 
 def metric_name():
@@ -175,7 +175,7 @@ def gpu_arm(args, rank, world, local_rank, dist):
     d.load_library()
     c = WORKLOAD
     # per-rank images: weak scaling, each rank regenerates exactly its own shard
-    images = list(range(rank * c.N, (rank + 1) * c.N))
+    images = sharding.shard_images(rank, world, c.N)
     P = inputs.gen_offset_branch(c)
     w, b = inputs.gen_weight(c)
     dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
@@ -283,10 +283,8 @@ def gpu_arm(args, rank, world, local_rank, dist):
     ms_e2e = a.elapsed_time(bq) / e2e_steps
 
     # ---------------- max over ranks
-    vals = torch.tensor([ms_total, ms_e2e, ms_dcn, ms_branch], dtype=torch.float64, device=dev)
-    if dist is not None:
-        dist.all_reduce(vals, op=dist.ReduceOp.MAX)
-    ms_total, ms_e2e, ms_dcn, ms_branch = [float(v) for v in vals.cpu()]
+    ms_total, ms_e2e, ms_dcn, ms_branch = sharding.max_over_ranks(
+        dist, [ms_total, ms_e2e, ms_dcn, ms_branch], dev)
 
     flops = configs.contraction_flops(c)
     ms_step = ms_total / args.steps
@@ -294,8 +292,10 @@ def gpu_arm(args, rank, world, local_rank, dist):
     peaks, peak_src = load_peaks()
     achieved = flops / (ms_dcn * 1e-3) / 1e12
     traffic = None
-    try:
-        with open(NCU_SUMMARY) as f:
+    try:   # dram read+write bytes per launch of the DCN kernel, latest committed ncu capture
+        import glob
+        latest = sorted(glob.glob(NCU_SUMMARY_GLOB))[-1]
+        with open(latest) as f:
             traffic = json.load(f).get("dcn_dram_bytes_per_launch")
     except Exception:
         pass
@@ -339,37 +339,41 @@ def gpu_arm(args, rank, world, local_rank, dist):
             "ms_per_step": round(ms_e2e, 4),
             "api": "defcon_layer_forward_host (C ABI, pinned host x -> y)",
         },
-        "gpu_launches": 2 * args.steps,
+        "gpu_launches": 3 * args.steps,   # dw_bn_relu + pw_sigmoid (step 1) + dcn_fwd (step 2)
     }
     return line
 
 
 # ------------------------------------------------------------------ oracle (CPU) legs
-def oracle_sample(c, target_s):
+def oracle_sample(c, target_s, images=4):
     """Time the oracle as it stands on a bounded sample of the workload: the offset branch
-    of image 0 plus the DCN at `n_pix` output pixels; returns (TFLOP/s, seconds, sample)."""
+    of `images` images plus the DCN at n_pix of their output pixels (calibrated so the sample
+    takes about target_s seconds); returns (TFLOP/s, seconds, description, n_pix)."""
     import oracle
     oracle.build()
-    x = inputs.gen_x(c, images=[0])
+    ci = c.replace(N=images)
+    x = inputs.gen_x(ci, images=list(range(images)))
     P = inputs.gen_offset_branch(c)
     w, b = inputs.gen_weight(c)
-    c1 = c.replace(N=1)
 
     def once(n_pix):
         t0 = time.perf_counter()
         off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
                                         P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated,
                                         stride=c.stride, pad=c.pad, dil=c.dil)
-        idx = np.arange(n_pix) % c1.M
+        idx = np.arange(n_pix) % ci.M
         oracle.dcn_pixels(x, off, w, idx, b, mask=msk, stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
         return time.perf_counter() - t0
 
-    t_cal = once(64)
-    n_pix = int(np.clip(64 * target_s / max(t_cal, 1e-3), 64, 4 * c1.M))
+    t_small = once(256)
+    t_big = once(2048)
+    per_pix = max((t_big - t_small) / (2048 - 256), 1e-7)
+    fixed = max(t_small - 256 * per_pix, 0.0)
+    n_pix = int(np.clip((target_s - fixed) / per_pix, 256, 50 * ci.M))
     dt = once(n_pix)
     flops = 2 * n_pix * c.Cout * c.K * c.K * c.Cin
-    sample = (f"{c.name}: offset branch of 1 image + DCN at {n_pix} output pixels "
-              f"({flops / 1e9:.2f} GFLOP contraction), fp64")
+    sample = (f"{c.name}: offset branch of {images} images + DCN at {n_pix} of their output "
+              f"pixels ({flops / 1e9:.1f} GFLOP contraction), fp64 C oracle, OpenMP")
     return flops / dt / 1e12, dt, sample, n_pix
 
 
@@ -381,19 +385,23 @@ def cpu_baseline(c):
 
 
 def reference_arm(args, world):
-    """--impl reference: the fp64 oracle, as it stands, on the host cores (rank 0 only)."""
+    """--impl reference: the fp64 oracle, as it stands, on the host cores (rank 0 only).
+    Each step is a bounded sample of the workload (see oracle_sample), sized so that the
+    whole --steps/--warmup run finishes within a few minutes."""
     import oracle
     c = WORKLOAD
-    per_step_s = 6.0
+    per_step_s = float(np.clip(150.0 / max(args.steps + args.warmup, 1), 1.0, 10.0))
     _, _, _, n_pix = oracle_sample(c, target_s=per_step_s)
-    x = inputs.gen_x(c, images=[0])
+    images = 4
+    ci = c.replace(N=images)
+    x = inputs.gen_x(ci, images=list(range(images)))
     P = inputs.gen_offset_branch(c)
     w, b = inputs.gen_weight(c)
 
     def step():
         off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
                                         P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated)
-        oracle.dcn_pixels(x, off, w, np.arange(n_pix) % c.replace(N=1).M, b, mask=msk, G=c.G)
+        oracle.dcn_pixels(x, off, w, np.arange(n_pix) % ci.M, b, mask=msk, G=c.G)
 
     for _ in range(args.warmup):
         step()
@@ -403,8 +411,8 @@ def reference_arm(args, world):
     dt = time.perf_counter() - t0
     flops = 2 * n_pix * c.Cout * c.K * c.K * c.Cin
     value = flops * args.steps / dt / 1e12
-    sample = (f"{c.name}: per step the offset branch of 1 image + DCN at {n_pix} output pixels, "
-              f"fp64 C oracle with OpenMP")
+    sample = (f"{c.name}: per step the offset branch of {images} images + DCN at {n_pix} of their "
+              f"output pixels, fp64 C oracle with OpenMP")
     return {
         "impl": "reference",
         "metric": metric_name(),
