@@ -256,115 +256,143 @@ __device__ __forceinline__ Segment segment_j(const TcArgs& a, long long it_begin
     return sg;
 }
 
+// Processing order of a CTA's segments: the last one (the head of a tile whose remaining
+// k-iterations belong to later CTAs) first, so its partial is published early; then the
+// rest in order.  The tail segment of a split tile -- its "owner", which holds the tile's
+// last k-iteration -- is then processed while the other contributors' partials are
+// already in L2.
+__device__ __forceinline__ int seg_order(int o, int nseg) {
+    if (nseg <= 1) return o;
+    return o == 0 ? nseg - 1 : o - 1;
+}
+
+__device__ __forceinline__ int ld_acquire_gpu(const int* p) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
 // Epilogue of one segment for NCOLS columns [col0, col0 + NCOLS) of row r (= TMEM lane).
-// whole tile: + bias -> bf16 -> y.  Partial: fp32 partial to `slot`; the last of the
-// tile's contributors to arrive sums every partial in segment order (deterministic).
+// Whole tile: + bias -> bf16 -> y.  Split tile (stream-K): non-owner contributors publish an
+// fp32 partial (slot = CTA index) and count themselves on the tile counter.  The owner, if
+// every other contributor has arrived (the normal case, see seg_order), adds the partials in
+// k order to its own TMEM accumulator and writes y; otherwise it publishes its accumulator too
+// (slot = grid + CTA) and whoever arrives last sums all partials.  Fixed summation order in
+// both cases: contributors by ascending k range, owner last -> deterministic.
 template <int BLOCK_N, int NCOLS>
-__device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment& sg, bool whole,
-                                                 int slot, uint32_t tacc, int r, int col0,
-                                                 int bar_id, int nthr, bool leader, int* fix_flag,
-                                                 long long T, int nct) {
-    constexpr int CH = NCOLS >= 32 ? 32 : 16;
+__device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment& sg, uint32_t tacc,
+                                                 int r, int col0, int bar_id, int nthr, bool leader,
+                                                 int* fix_flag, long long T, int nct) {
+    constexpr int CH = 16;
     const int m0 = (sg.tile / a.n_tiles_n) * BM;
     const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
     const int row = m0 + r;
     const bool row_ok = row < a.M;
-    float* slotp = a.partials + (size_t)slot * BLOCK_N * BM;
-#pragma unroll 1
-    for (int c = col0; c < col0 + NCOLS; c += CH) {
-        uint32_t v[CH];
-        tmem_ld_32x32b_x16(tacc + c, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
-        if constexpr (CH == 32) tmem_ld_32x32b_x16(tacc + c + 16, *reinterpret_cast<uint32_t(*)[16]>(&v[16]));
-        tmem_ld_wait();
-        if (whole) {
-            if (row_ok) {
-#pragma unroll
-                for (int h = 0; h < CH; h += 16) {
-                    if (n0 + c + h < a.Cout) {
-                        uint32_t pk[8];
-#pragma unroll
-                        for (int u = 0; u < 8; ++u) {
-                            const int co = n0 + c + h + 2 * u;
-                            const float b0 = a.bias ? __ldg(a.bias + co) : 0.f;
-                            const float b1 = a.bias ? __ldg(a.bias + co + 1) : 0.f;
-                            pk[u] = pack_bf16x2(__uint_as_float(v[h + 2 * u]) + b0,
-                                                __uint_as_float(v[h + 2 * u + 1]) + b1);
-                        }
-                        uint4* dst = reinterpret_cast<uint4*>(a.y + (size_t)row * a.Cout + n0 + c + h);
-                        dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-                        dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-                    }
-                }
-            }
-        } else {
-            // fp32 partial, layout [col/4][row][4] (coalesced across lanes)
-#pragma unroll
-            for (int u = 0; u < CH / 4; ++u) {
-                const float4 f = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
-                                             __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
-                __stcg(reinterpret_cast<float4*>(slotp) + (size_t)((c >> 2) + u) * BM + r, f);
-            }
-        }
-    }
-    if (whole) return;
-
-    __threadfence();
-    named_bar_sync(bar_id, nthr);
+    const bool owner = sg.ke == a.ipt;
     const long long t0 = (long long)sg.tile * a.ipt;
     const int b_lo = cta_of(T, nct, t0);
-    const int b_hi = cta_of(T, nct, t0 + a.ipt - 1);
-    if (leader) {
-        const int old = atomicAdd(a.counters + sg.tile, 1);
-        *fix_flag = (old == b_hi - b_lo) ? 1 : 0;
+    const int b_hi = cta_of(T, nct, t0 + a.ipt - 1);      // == owner CTA
+    const int ncontrib = b_hi - b_lo;                    // contributors other than the owner
+    const size_t slot_elems = (size_t)BLOCK_N * BM;
+    const float4* parts = reinterpret_cast<const float4*>(a.partials);
+
+    auto write_partial = [&](int slot) {
+        float4* dst = reinterpret_cast<float4*>(a.partials + (size_t)slot * slot_elems);
+#pragma unroll 1
+        for (int c = col0; c < col0 + NCOLS; c += CH) {
+            uint32_t v[CH];
+            tmem_ld_32x32b_x16(tacc + c, v);
+            tmem_ld_wait();
+#pragma unroll
+            for (int u = 0; u < CH / 4; ++u)
+                __stcg(dst + (size_t)((c >> 2) + u) * BM + r,
+                       make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                                   __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3])));
+        }
+        __threadfence();
+    };
+    // y = bias + sum(partials of contributors b_lo..b_hi-1) [+ own accumulator | owner slot]
+    auto finish = [&](bool own_from_tmem) {
+#pragma unroll 1
+        for (int c = col0; c < col0 + NCOLS; c += CH) {
+            uint32_t v[CH];
+            if (own_from_tmem) {
+                tmem_ld_32x32b_x16(tacc + c, v);
+                tmem_ld_wait();
+            }
+            if (!row_ok || n0 + c >= a.Cout) continue;
+            float acc[CH];
+#pragma unroll
+            for (int u = 0; u < CH; ++u) acc[u] = 0.f;
+#pragma unroll 1
+            for (int b = b_lo; b <= b_hi; ++b) {
+                float4 f[CH / 4];
+                if (b < b_hi || !own_from_tmem) {
+                    const int slot = b < b_hi ? b : nct + b;
+#pragma unroll
+                    for (int u = 0; u < CH / 4; ++u)
+                        f[u] = __ldcg(parts + (size_t)slot * (slot_elems / 4) + (size_t)((c >> 2) + u) * BM + r);
+                } else {
+#pragma unroll
+                    for (int u = 0; u < CH / 4; ++u)
+                        f[u] = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                                           __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
+                }
+#pragma unroll
+                for (int u = 0; u < CH / 4; ++u) {
+                    acc[4 * u] += f[u].x; acc[4 * u + 1] += f[u].y;
+                    acc[4 * u + 2] += f[u].z; acc[4 * u + 3] += f[u].w;
+                }
+            }
+            uint32_t pk[CH / 2];
+#pragma unroll
+            for (int u = 0; u < CH / 2; ++u) {
+                const int co = n0 + c + 2 * u;
+                const float b0 = a.bias ? __ldg(a.bias + co) : 0.f;
+                const float b1 = a.bias ? __ldg(a.bias + co + 1) : 0.f;
+                pk[u] = pack_bf16x2(acc[2 * u] + b0, acc[2 * u + 1] + b1);
+            }
+            uint4* dst = reinterpret_cast<uint4*>(a.y + (size_t)row * a.Cout + n0 + c);
+            dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+            dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+        }
+    };
+
+    if (owner && ncontrib == 0) {          // whole tile
+        finish(true);
+        return;
     }
+    if (!owner) {                          // non-owner contributor: publish, count
+        write_partial(blockIdx.x);
+        named_bar_sync(bar_id, nthr);
+        if (leader) *fix_flag = (atomicAdd(a.counters + sg.tile, 1) == ncontrib) ? 1 : 0;
+        named_bar_sync(bar_id, nthr);
+        const bool last = *fix_flag != 0;
+        named_bar_sync(bar_id, nthr);      // fix_flag reused by the next segment
+        if (last) {                        // owner took the slow path: finish from partials
+            __threadfence();
+            finish(false);
+        }
+        return;
+    }
+    // owner of a split tile
+    if (leader) *fix_flag = (ld_acquire_gpu(a.counters + sg.tile) == ncontrib) ? 1 : 0;
     named_bar_sync(bar_id, nthr);
-    const bool finisher = *fix_flag != 0;
-    named_bar_sync(bar_id, nthr);   // fix_flag may be reused by the next segment
-    if (!finisher) return;
-    __threadfence();
-    if (!row_ok) return;
-#pragma unroll 1
-    for (int c = col0; c < col0 + NCOLS; c += 16) {
-        if (n0 + c >= a.Cout) break;
-        float acc[16];
-#pragma unroll
-        for (int u = 0; u < 16; ++u) acc[u] = 0.f;
-#pragma unroll 1
-        for (int b = b_lo; b <= b_hi; b += 2) {
-            float4 f[2][4];
-#pragma unroll
-            for (int s = 0; s < 2; ++s) {
-                if (b + s <= b_hi) {
-                    // slot 2b if this tile is b's first segment, else 2b+1
-                    const int bb = b + s;
-                    const int sidx = 2 * bb + ((range_begin(T, nct, bb) / a.ipt) == sg.tile ? 0 : 1);
-                    const float4* src = reinterpret_cast<const float4*>(a.partials + (size_t)sidx * BLOCK_N * BM);
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) f[s][u] = __ldcg(src + (size_t)((c >> 2) + u) * BM + r);
-                }
-            }
-#pragma unroll
-            for (int s = 0; s < 2; ++s) {
-                if (b + s <= b_hi) {
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        acc[4 * u] += f[s][u].x; acc[4 * u + 1] += f[s][u].y;
-                        acc[4 * u + 2] += f[s][u].z; acc[4 * u + 3] += f[s][u].w;
-                    }
-                }
-            }
-        }
-        uint32_t pk[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-            const int co = n0 + c + 2 * u;
-            const float b0 = a.bias ? __ldg(a.bias + co) : 0.f;
-            const float b1 = a.bias ? __ldg(a.bias + co + 1) : 0.f;
-            pk[u] = pack_bf16x2(acc[2 * u] + b0, acc[2 * u + 1] + b1);
-        }
-        uint4* dst = reinterpret_cast<uint4*>(a.y + (size_t)row * a.Cout + n0 + c);
-        dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-        dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+    const bool all_in = *fix_flag != 0;
+    named_bar_sync(bar_id, nthr);
+    if (all_in) {                          // fast path: partials + own TMEM accumulator
+        finish(true);
+        return;
+    }
+    write_partial(nct + blockIdx.x);       // slow path: publish own accumulator as well
+    named_bar_sync(bar_id, nthr);
+    if (leader) *fix_flag = (atomicAdd(a.counters + sg.tile, 1) == ncontrib) ? 1 : 0;
+    named_bar_sync(bar_id, nthr);
+    const bool last = *fix_flag != 0;
+    named_bar_sync(bar_id, nthr);
+    if (last) {
+        __threadfence();
+        finish(false);
     }
 }
 
@@ -430,8 +458,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         using Smp = Sampler<TEX>;
         int q = 0;                           // running k-iteration (stage) counter
-        for (int j = 0; j < nseg; ++j) {
-            const Segment sg = segment_j(a, it_begin, it_end, j);
+        for (int o = 0; o < nseg; ++o) {
+            const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
             const int m0 = (sg.tile / a.n_tiles_n) * BM;
             int chunk = sg.kb / a.KK;
             int tap = sg.kb - chunk * a.KK;
@@ -482,38 +510,33 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 xb = nxb;
             }
         }
-        // The producers (4 lane quarters x NPW/4 column slices) run the last segment's
-        // epilogue, which would otherwise be exposed at the end of the CTA's range.
+        // The producers (4 lane quarters x NPW/4 column slices) run the last processed
+        // segment's epilogue, which would otherwise be exposed at the end of the CTA's range.
         if (nseg > 0) {
-            const int j = nseg - 1;
-            const Segment sg = segment_j(a, it_begin, it_end, j);
-            const int buf = j % Cfg::NBUF;
-            mbar_wait(&tmem_full[buf], (uint32_t)(j / Cfg::NBUF) & 1u);
+            const int o = nseg - 1;
+            const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
+            const int buf = o % Cfg::NBUF;
+            mbar_wait(&tmem_full[buf], (uint32_t)(o / Cfg::NBUF) & 1u);
             tc_fence_after();
             const int qd = warp & 3;
             const int r = qd * 32 + lane;
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
-            const bool whole = sg.kb == 0 && sg.ke == a.ipt;
-            const int slot = 2 * blockIdx.x + (j == 0 ? 0 : 1);
             constexpr int SLICE = BLOCK_N / (NPW / 4);
-            epilogue_segment<BLOCK_N, SLICE>(a, sg, whole, slot, tacc, r, (warp >> 2) * SLICE,
-                                             1, NPT, t == 0, fix_flag + 1, T, nct);
+            epilogue_segment<BLOCK_N, SLICE>(a, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT, t == 0,
+                                             fix_flag + 1, T, nct);
         }
     } else if (warp < EPI_WARP0 + 4) {
-        // ===================== epilogue (all segments but the last) =====================
+        // ===================== epilogue (all processed segments but the last) ============
         const int qd = warp & 3;                    // TMEM lane quarter of this warp
         const int r = qd * 32 + lane;               // row within the tile (= TMEM lane)
-        for (int j = 0; j + 1 < nseg; ++j) {
-            const Segment sg = segment_j(a, it_begin, it_end, j);
-            const int buf = j % Cfg::NBUF;
-            mbar_wait(&tmem_full[buf], (uint32_t)(j / Cfg::NBUF) & 1u);
+        for (int o = 0; o + 1 < nseg; ++o) {
+            const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
+            const int buf = o % Cfg::NBUF;
+            mbar_wait(&tmem_full[buf], (uint32_t)(o / Cfg::NBUF) & 1u);
             tc_fence_after();
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
-            const bool whole = sg.kb == 0 && sg.ke == a.ipt;
-            const int slot = 2 * blockIdx.x + (j == 0 ? 0 : 1);
-            // Release the accumulator as soon as it is in registers / written out.
-            epilogue_segment<BLOCK_N, BLOCK_N>(a, sg, whole, slot, tacc, r, 0, 2, 128,
-                                               threadIdx.x == EPI_WARP0 * 32, fix_flag, T, nct);
+            epilogue_segment<BLOCK_N, BLOCK_N>(a, sg, tacc, r, 0, 2, 128, threadIdx.x == EPI_WARP0 * 32,
+                                               fix_flag, T, nct);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&tmem_empty[buf]);
@@ -522,8 +545,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         // ===================== TMA producer (weights) =====================
         if (lane == 0) {
             int q = 0;
-            for (int j = 0; j < nseg; ++j) {
-                const Segment sg = segment_j(a, it_begin, it_end, j);
+            for (int o = 0; o < nseg; ++o) {
+                const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
                 const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
                 int chunk = sg.kb / a.KK;
                 int tap = sg.kb - chunk * a.KK;
@@ -545,10 +568,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (lane == 0) {
             constexpr uint32_t idesc = make_idesc(1u /*BF16*/, BM, Cfg::UMMA_N);
             int q = 0;
-            for (int j = 0; j < nseg; ++j) {
-                const Segment sg = segment_j(a, it_begin, it_end, j);
-                const int buf = j % Cfg::NBUF;
-                mbar_wait(&tmem_empty[buf], ((uint32_t)(j / Cfg::NBUF) & 1u) ^ 1u);
+            for (int o = 0; o < nseg; ++o) {
+                const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
+                const int buf = o % Cfg::NBUF;
+                mbar_wait(&tmem_empty[buf], ((uint32_t)(o / Cfg::NBUF) & 1u) ^ 1u);
                 tc_fence_after();
                 const uint32_t d_base = tmem_base + (uint32_t)(buf * BLOCK_N);
                 for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
