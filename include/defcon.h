@@ -57,8 +57,11 @@ typedef enum {
 
 typedef enum {
     DEFCON_SAMPLER_LDG = 0,  /* software bilinear: vectorised NHWC gathers, fp32 weights */
-    DEFCON_SAMPLER_TEX = 1   /* hardware bilinear: tex2DLayered, border (zero) addressing,
+    DEFCON_SAMPLER_TEX = 1,  /* hardware bilinear: tex2DLayered, border (zero) addressing,
                                 the paper's texel-based optimisation         */
+    DEFCON_SAMPLER_HYBRID = 2 /* half of the A-producer warps use TEX, half LDG, so the
+                                texture units and the FMA pipes work in parallel (SURVEY
+                                section 8(f) NEXT 1); needs a tex_plan like TEX         */
 } defcon_sampler_t;
 
 typedef enum {
@@ -125,9 +128,9 @@ int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_
  *   x        [N][H][W][Cin], dtype `dtype`
  *   offset   [N][Ho][Wo][G][Kh*Kw][2] fp32 (dy, dx);  mask [N][Ho][Wo][G][Kh*Kw] fp32 or NULL
  *   weight   [Cout][Kh][Kw][Cin], dtype `dtype`;  bias [Cout] fp32 or NULL (= 0)
- *   sampler  DEFCON_SAMPLER_LDG (any dtype) or DEFCON_SAMPLER_TEX (requires tex_plan made
- *            for the same N, H, W, Cin, dtype; the plan's array is (re)filled from x on
- *            `stream` by this call)
+ *   sampler  DEFCON_SAMPLER_LDG (any dtype), DEFCON_SAMPLER_TEX or DEFCON_SAMPLER_HYBRID
+ *            (bf16 tensor-core path; require tex_plan made for the same N, H, W, Cin, dtype;
+ *            the plan's array is (re)filled from x on `stream` by this call)
  *   fp32_mode  used only when dtype == DEFCON_F32
  *   y        [N][Ho][Wo][Cout], dtype `dtype` (written)
  *   workspace / workspace_bytes: device scratch of at least defcon_dcn_workspace_size()

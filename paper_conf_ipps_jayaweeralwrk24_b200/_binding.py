@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(HERE, "libdefcon.so")
 DEFCON_OK, DEFCON_ERR_INVALID_ARG, DEFCON_ERR_UNSUPPORTED, DEFCON_ERR_MISALIGNED, \
     DEFCON_ERR_CUDA, DEFCON_ERR_LIMIT = range(6)
 DEFCON_F32, DEFCON_BF16 = 0, 1
-DEFCON_SAMPLER_LDG, DEFCON_SAMPLER_TEX = 0, 1
+DEFCON_SAMPLER_LDG, DEFCON_SAMPLER_TEX, DEFCON_SAMPLER_HYBRID = 0, 1, 2
 DEFCON_FP32_3XTF32, DEFCON_FP32_SIMT = 0, 1
 
 # Every symbol include/defcon.h declares (checked by tests/test_abi.py).
@@ -31,7 +31,7 @@ EXPORTED = (
 )
 
 _DTYPES = {torch.float32: DEFCON_F32, torch.bfloat16: DEFCON_BF16}
-_SAMPLERS = {"ldg": DEFCON_SAMPLER_LDG, "tex": DEFCON_SAMPLER_TEX}
+_SAMPLERS = {"ldg": DEFCON_SAMPLER_LDG, "tex": DEFCON_SAMPLER_TEX, "hybrid": DEFCON_SAMPLER_HYBRID}
 _FP32_MODES = {"3xtf32": DEFCON_FP32_3XTF32, "simt": DEFCON_FP32_SIMT}
 
 

@@ -91,11 +91,11 @@ static int make_geom(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
 enum class Path { SIMT_F32, SIMT_BF16, TC_BF16 };
 
 static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, Path* path) {
-    if (sampler != DEFCON_SAMPLER_LDG && sampler != DEFCON_SAMPLER_TEX)
+    if (sampler != DEFCON_SAMPLER_LDG && sampler != DEFCON_SAMPLER_TEX && sampler != DEFCON_SAMPLER_HYBRID)
         return fail(DEFCON_ERR_INVALID_ARG, "bad sampler");
     if (fp32_mode != DEFCON_FP32_3XTF32 && fp32_mode != DEFCON_FP32_SIMT)
         return fail(DEFCON_ERR_INVALID_ARG, "bad fp32_mode");
-    if (sampler == DEFCON_SAMPLER_TEX) {
+    if (sampler == DEFCON_SAMPLER_TEX || sampler == DEFCON_SAMPLER_HYBRID) {
         if (dtype != DEFCON_BF16 || !dcn_tc_bf16_supported(g))
             return fail(DEFCON_ERR_UNSUPPORTED,
                         "texture sampler is built for the bf16 tensor-core path (Cin/G %% 64 == 0)");
@@ -227,7 +227,7 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     rc = select_path(g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
     TexPlan* tp = nullptr;
-    if (sampler == DEFCON_SAMPLER_TEX) {
+    if (sampler == DEFCON_SAMPLER_TEX || sampler == DEFCON_SAMPLER_HYBRID) {
         tp = reinterpret_cast<TexPlan*>(tex_plan);
         if (!tex_plan_matches(tp, N, H, W, Cin, dtype == DEFCON_BF16))
             return fail(DEFCON_ERR_INVALID_ARG, "tex_plan missing or made for another shape/dtype");
@@ -244,7 +244,8 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
         if (e != cudaSuccess) return cuda_fail(e, "texture staging launch");
     }
     switch (path) {
-        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, workspace, workspace_bytes, tp, st, &detail); break;
+        case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, workspace, workspace_bytes, tp,
+                                                   sampler == DEFCON_SAMPLER_HYBRID, st, &detail); break;
         case Path::SIMT_BF16: e = launch_dcn_simt(g, p, true, st); break;
         default: e = launch_dcn_simt(g, p, false, st); break;
     }

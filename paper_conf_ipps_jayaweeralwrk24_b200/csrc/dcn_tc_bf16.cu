@@ -92,10 +92,9 @@ struct Segment {
 // channel 0 of each of the 4 bilinear corners and the 4 corner weights with the mask
 // folded in.  Corners outside the image get weight 0 and the harmless in-bounds
 // offset 0 (R8).
-template <bool TEX>
 __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int row, int tap, int g,
-                                                 uint8_t* meta) {
-    if constexpr (TEX) {
+                                                 uint8_t* meta, bool tex_row) {
+    if (tex_row) {
         // texture sampler: unnormalised texel coordinates (texel centres at +0.5, R7) in the
         // stacked-image texture (image n occupies rows n*(H+1) .. n*(H+1)+H-1, row
         // n*(H+1)+H is zero) and the mask.  Clamping to [-1, H] x [-1, W] keeps samples
@@ -396,7 +395,74 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
     }
 }
 
-template <int BLOCK_N, int STAGES, bool TEX>
+// One producer warp's share of one segment: for every k-iteration, 4 A rows x 16 bytes per
+// thread, with the next k-iteration's gathers (or texture fetches) issued row by row as
+// soon as the row's registers are free (rolling prefetch).  Warps with TEXW use the texture
+// sampler, the others LDG gathers + software lerp; the metadata table holds each row in the
+// format its warp consumes (warp of row r = (r mod 32) / 4).
+template <bool TEXW, int STAGES, int NTEX>
+__device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
+                                                const uint32_t (&dst)[ROWS], const uint32_t (&mrow)[ROWS],
+                                                uint32_t a_s, uint64_t* empty, uint64_t* full_a, int t,
+                                                int cvec, int lane) {
+    using Smp = Sampler<TEXW>;
+    const int m0 = (sg.tile / a.n_tiles_n) * BM;
+    int chunk = sg.kb / a.KK;
+    int tap = sg.kb - chunk * a.KK;
+    int g = (chunk * BK) / a.Cg;
+    named_bar_sync(1, NPT);          // previous table no longer read
+    for (int e = t; e < BM * a.KK; e += NPT) {
+        const int row = e / a.KK;
+        build_meta_entry(a, m0, row, e - row * a.KK, g, meta, ((row & 31) >> 2) < NTEX);
+    }
+    named_bar_sync(1, NPT);
+    // position of this thread's 8 channels: byte pointer (LDG) / texture layer (TEX)
+    const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + cvec * 8) * 2;
+    int layer = chunk * (BK / 4) + cvec * 2;
+    typename Smp::Load L[ROWS];
+#pragma unroll
+    for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], xb, a.tex, layer, mrow[p] + tap * META_ENTRY);
+    for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
+        int ntap = tap + 1, nchunk = chunk;
+        if (ntap == a.KK) { ntap = 0; ++nchunk; }
+        const bool has_next = kt + 1 < sg.ke;
+        int ng = g;
+        if (has_next && nchunk != chunk) ng = (nchunk * BK) / a.Cg;
+        const bool prefetch = has_next && ng == g;
+        const uint8_t* nxb = nchunk != chunk ? xb + BK * 2 : xb;
+        const int nlayer = nchunk != chunk ? layer + BK / 4 : layer;
+
+        const int s = q % STAGES;
+        mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
+        const uint32_t stage = a_s + s * A_STAGE_BYTES;
+#pragma unroll
+        for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
+            Smp::store(L[p], stage + dst[p]);
+            if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&full_a[s]);
+
+        if (has_next && !prefetch) {          // offset group changes: new table
+            named_bar_sync(1, NPT);
+            for (int e = t; e < BM * a.KK; e += NPT) {
+                const int row = e / a.KK;
+                build_meta_entry(a, m0, row, e - row * a.KK, ng, meta, ((row & 31) >> 2) < NTEX);
+            }
+            named_bar_sync(1, NPT);
+            g = ng;
+#pragma unroll
+            for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
+        }
+        layer = nlayer;
+        tap = ntap;
+        chunk = nchunk;
+        xb = nxb;
+    }
+}
+
+template <int BLOCK_N, int STAGES, int NTEX>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const TcArgs a) {
     using Cfg = TcCfg<BLOCK_N>;
@@ -456,59 +522,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             dst[p] = row * 128 + ((cvec ^ (row & 7)) << 4);
             mrow[p] = meta_s + row * a.KK * META_ENTRY;
         }
-        using Smp = Sampler<TEX>;
         int q = 0;                           // running k-iteration (stage) counter
         for (int o = 0; o < nseg; ++o) {
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
-            const int m0 = (sg.tile / a.n_tiles_n) * BM;
-            int chunk = sg.kb / a.KK;
-            int tap = sg.kb - chunk * a.KK;
-            int g = (chunk * BK) / a.Cg;
-            named_bar_sync(1, NPT);          // previous table no longer read
-            for (int e = t; e < BM * a.KK; e += NPT) build_meta_entry<TEX>(a, m0, e / a.KK, e % a.KK, g, meta);
-            named_bar_sync(1, NPT);
-            // position of this thread's 8 channels: byte pointer (LDG) / texture layer (TEX)
-            const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + cvec * 8) * 2;
-            int layer = chunk * (BK / 4) + cvec * 2;
-            typename Smp::Load L[ROWS];
-#pragma unroll
-            for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], xb, a.tex, layer, mrow[p] + tap * META_ENTRY);
-            for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
-                int ntap = tap + 1, nchunk = chunk;
-                if (ntap == a.KK) { ntap = 0; ++nchunk; }
-                const bool has_next = kt + 1 < sg.ke;
-                int ng = g;
-                if (has_next && nchunk != chunk) ng = (nchunk * BK) / a.Cg;
-                const bool prefetch = has_next && ng == g;
-                const uint8_t* nxb = nchunk != chunk ? xb + BK * 2 : xb;
-                const int nlayer = nchunk != chunk ? layer + BK / 4 : layer;
-
-                const int s = q % STAGES;
-                mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
-                const uint32_t stage = a_s + s * A_STAGE_BYTES;
-#pragma unroll
-                for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
-                    Smp::store(L[p], stage + dst[p]);
-                    if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
-                }
-                fence_proxy_async_smem();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&full_a[s]);
-
-                if (has_next && !prefetch) {          // offset group changes: new table
-                    named_bar_sync(1, NPT);
-                    for (int e = t; e < BM * a.KK; e += NPT)
-                        build_meta_entry<TEX>(a, m0, e / a.KK, e % a.KK, ng, meta);
-                    named_bar_sync(1, NPT);
-                    g = ng;
-#pragma unroll
-                    for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
-                }
-                layer = nlayer;
-                tap = ntap;
-                chunk = nchunk;
-                xb = nxb;
-            }
+            if (warp < NTEX)
+                produce_segment<true, STAGES, NTEX>(a, sg, q, meta, dst, mrow, a_s, empty, full_a, t, cvec, lane);
+            else
+                produce_segment<false, STAGES, NTEX>(a, sg, q, meta, dst, mrow, a_s, empty, full_a, t, cvec, lane);
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
         // segment's epilogue, which would otherwise be exposed at the end of the CTA's range.
@@ -659,7 +679,7 @@ size_t workspace_impl(const DcnGeom& g) {
 
 template <int BLOCK_N, int STAGES>
 cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
-                        const TexPlan* tex, cudaStream_t stream, const char** detail) {
+                        const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
     using Cfg = TcCfg<BLOCK_N>;
     auto plan = make_plan<BLOCK_N>(g);
     if (ws_bytes < plan.counters_bytes + plan.partial_bytes || ws == nullptr) {
@@ -708,8 +728,9 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     }
     const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + (size_t)BM * g.KK * META_ENTRY +
                         (3 * STAGES + 2 * Cfg::NBUF) * 8 + 32;
-    auto kern = tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, true>
-                    : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, false>;
+    auto kern = !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0>
+                : hybrid ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW / 2>
+                         : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW>;
     e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) {
         *detail = "cudaFuncSetAttribute(MaxDynamicSharedMemorySize) failed";
@@ -739,11 +760,11 @@ size_t dcn_tc_bf16_workspace(const DcnGeom& g) {
 }
 
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
-                               const TexPlan* tex, cudaStream_t stream, const char** detail) {
-    if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, stream, detail);
-    if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, stream, detail);
-    if (g.Cout <= 256) return launch_impl<256, 3>(g, p, ws, ws_bytes, tex, stream, detail);
-    return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, stream, detail);
+                               const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
+    if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+    if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+    if (g.Cout <= 256) return launch_impl<256, 3>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+    return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 }
 
 }  // namespace defcon

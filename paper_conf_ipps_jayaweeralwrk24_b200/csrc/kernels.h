@@ -43,7 +43,7 @@ bool dcn_tc_bf16_supported(const DcnGeom& g);
 size_t dcn_tc_bf16_workspace(const DcnGeom& g);   // stream-K counters + fp32 partials
 struct TexPlan;
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
-                               const TexPlan* tex, cudaStream_t stream, const char** detail);
+                               const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail);
 
 // ---- texture sampler resources (tex_plan.cu)
 struct TexPlan;

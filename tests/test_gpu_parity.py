@@ -224,20 +224,21 @@ def test_tex_filter_fixed_point(d, dev):
                                small("tex_g2", G=2), small("tex_g2_v1", G=2, modulated=False),
                                configs.C5.replace(N=2), small("tex_s2", stride=2, H=23, W=21)],
                          ids=lambda c: c.name)
-def test_tex_sampler_parity(oracle_mod, d, dev, c):
+@pytest.mark.parametrize("sampler", ["tex", "hybrid"])
+def test_tex_sampler_parity(oracle_mod, d, dev, c, sampler):
     """TEX sampler: equals the texture-model oracle (fp16 texels, 1/256 fractions,
     measured rounding) to bf16 precision, and the exact oracle within the 5e-3 gate."""
     mode = tex_mode(d, dev)
     L = inputs.gen_layer(c)
     plan = d.TexPlan(c.N, c.H, c.W, c.Cin, torch.bfloat16)
-    y = run_dcn(d, dev, c, dict(L), sampler="tex", tex_plan=plan)
+    y = run_dcn(d, dev, c, dict(L), sampler=sampler, tex_plan=plan)
     x16 = inputs.round_to(L["x"], "f16")
     refq = oracle_mod.dcn_forward_texq(x16, L["offset"], L["weight"], L["bias"], mask=L["mask"],
                                        stride=c.stride, pad=c.pad, dil=c.dil, G=c.G, quant=mode)
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
                                  stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
     e_q, e_x = normwise(y, refq), normwise(y, ref)
-    print(f"{c.name}: vs texture model {e_q:.2e}, vs exact oracle {e_x:.2e}")
+    print(f"{c.name} {sampler}: vs texture model {e_q:.2e}, vs exact oracle {e_x:.2e}")
     assert e_q < 1e-2
     assert e_x < 5e-3
     plan.close()

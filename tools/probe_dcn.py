@@ -28,7 +28,7 @@ def time_cfg(c, sampler, reps=200):
     ws = torch.empty(max(16, d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K,
                                                          c.stride, c.pad, c.dil, c.G, dt, sampler)),
                      dtype=torch.uint8, device=dev)
-    plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler == "tex" else None
+    plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler in ("tex", "hybrid") else None
     fn = lambda: d.defcon_dcn_forward(x, off, msk, w, b, stride=c.stride, pad=c.pad, dil=c.dil,
                                       offset_groups=c.G, y=y, workspace=ws, sampler=sampler,
                                       tex_plan=plan)
@@ -52,7 +52,7 @@ def time_cfg(c, sampler, reps=200):
 
 if __name__ == "__main__":
     names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["yolact_r101_c4_v2"]
-    samplers = sys.argv[2].split(",") if len(sys.argv) > 2 else ["ldg", "tex"]
+    samplers = sys.argv[2].split(",") if len(sys.argv) > 2 else ["ldg", "tex", "hybrid"]
     d.load_library()
     for n in names:
         if ":" in n:          # name:N override, e.g. yolact_r101_c4_v2:8
