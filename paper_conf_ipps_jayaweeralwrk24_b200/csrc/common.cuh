@@ -198,6 +198,12 @@ DEFCON_DEVICE void st_shared_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t 
                  : "memory");
 }
 
+DEFCON_DEVICE uint32_t ld_shared_u32(uint32_t addr) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+}
+
 DEFCON_DEVICE uint4 ld_shared_v4(uint32_t addr) {
     uint4 r;
     asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"

@@ -42,7 +42,9 @@ constexpr int TMA_WARP = 12;
 constexpr int MMA_WARP = 13;
 constexpr int NUM_THREADS = 14 * 32;
 constexpr int NPT = NPW * 32;
-constexpr int ROWS = BM * 8 / NPT;   // A rows per producer thread (8 threads per 128-B row)
+constexpr int TPR = 4;               // producer threads per 128-byte A row (32 bytes each)
+constexpr int ROWS = BM * TPR / NPT; // A rows per producer thread
+constexpr int RPW = 32 / TPR;        // rows per warp per pass
 
 struct TcArgs {
     const __nv_bfloat16* x;
@@ -164,7 +166,7 @@ __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int ro
 
 // The 4 corner vectors (8 channels each) of one A row and their weights.
 struct RowLoad {
-    uint4 v[4];
+    U8x32 v[4];
     float4 w;
 };
 
@@ -173,34 +175,36 @@ __device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_
     const uint4 wb = ld_shared_v4(meta_addr + 16);
     L.w = make_float4(__uint_as_float(wb.x), __uint_as_float(wb.y), __uint_as_float(wb.z),
                       __uint_as_float(wb.w));
-    L.v[0] = ldg_nc_v4(add_u32(xbase, o.x));
-    L.v[1] = ldg_nc_v4(add_u32(xbase, o.y));
-    L.v[2] = ldg_nc_v4(add_u32(xbase, o.z));
-    L.v[3] = ldg_nc_v4(add_u32(xbase, o.w));
+    L.v[0] = ldg_nc_v8(add_u32(xbase, o.x));
+    L.v[1] = ldg_nc_v8(add_u32(xbase, o.y));
+    L.v[2] = ldg_nc_v8(add_u32(xbase, o.z));
+    L.v[3] = ldg_nc_v8(add_u32(xbase, o.w));
 }
 
-// Eq.3 for 8 channels: sum_q w_q * corner_q, fp32 (packed FFMA2), RNE to bf16, into smem.
-__device__ __forceinline__ void lerp_store_row(const RowLoad& L, uint32_t dst) {
-    uint64_t acc[4];
+// Eq.3 for 16 channels: sum_q w_q * corner_q, fp32 (packed FFMA2), RNE to bf16, into the
+// two 16-byte swizzled slots of this thread's part of the A row.
+__device__ __forceinline__ void lerp_store_row(const RowLoad& L, uint32_t dst_lo, uint32_t dst_hi) {
+    uint64_t acc[8];
     const float wq[4] = {L.w.x, L.w.y, L.w.z, L.w.w};
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
         const uint64_t w2 = f32x2_pack(wq[q], wq[q]);
-        const uint32_t u[4] = {L.v[q].x, L.v[q].y, L.v[q].z, L.v[q].w};
 #pragma unroll
-        for (int h = 0; h < 4; ++h) {
-            const uint64_t c = bf16x2_to_f32x2(u[h]);
+        for (int h = 0; h < 8; ++h) {
+            const uint64_t c = bf16x2_to_f32x2(L.v[q].w[h]);
             acc[h] = q == 0 ? f32x2_mul(c, w2) : f32x2_fma(c, w2, acc[h]);
         }
     }
-    st_shared_v4(dst, f32x2_to_bf16x2(acc[0]), f32x2_to_bf16x2(acc[1]), f32x2_to_bf16x2(acc[2]),
+    st_shared_v4(dst_lo, f32x2_to_bf16x2(acc[0]), f32x2_to_bf16x2(acc[1]), f32x2_to_bf16x2(acc[2]),
                  f32x2_to_bf16x2(acc[3]));
+    st_shared_v4(dst_hi, f32x2_to_bf16x2(acc[4]), f32x2_to_bf16x2(acc[5]), f32x2_to_bf16x2(acc[6]),
+                 f32x2_to_bf16x2(acc[7]));
 }
 
-// Texture-sampler counterpart of RowLoad: 8 channels = 2 texels of 4 channels, already
+// Texture-sampler counterpart of RowLoad: 16 channels = 4 texels of 4 channels, already
 // bilinearly filtered by the texture unit, and the mask.
 struct TexLoad {
-    float4 t0, t1;
+    float4 t[4];
     float m;
 };
 
@@ -209,13 +213,16 @@ __device__ __forceinline__ void issue_row_tex(TexLoad& L, cudaTextureObject_t te
     const uint4 c = ld_shared_v4(meta_addr);
     const float fx = __uint_as_float(c.x), fy = __uint_as_float(c.y);
     L.m = __uint_as_float(c.z);
-    L.t0 = tex2DLayered<float4>(tex, fx, fy, layer);
-    L.t1 = tex2DLayered<float4>(tex, fx, fy, layer + 1);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) L.t[i] = tex2DLayered<float4>(tex, fx, fy, layer + i);
 }
 
-__device__ __forceinline__ void tex_store_row(const TexLoad& L, uint32_t dst) {
-    st_shared_v4(dst, pack_bf16x2(L.t0.x * L.m, L.t0.y * L.m), pack_bf16x2(L.t0.z * L.m, L.t0.w * L.m),
-                 pack_bf16x2(L.t1.x * L.m, L.t1.y * L.m), pack_bf16x2(L.t1.z * L.m, L.t1.w * L.m));
+__device__ __forceinline__ void tex_store_row(const TexLoad& L, uint32_t dst_lo, uint32_t dst_hi) {
+    const float m = L.m;
+    st_shared_v4(dst_lo, pack_bf16x2(L.t[0].x * m, L.t[0].y * m), pack_bf16x2(L.t[0].z * m, L.t[0].w * m),
+                 pack_bf16x2(L.t[1].x * m, L.t[1].y * m), pack_bf16x2(L.t[1].z * m, L.t[1].w * m));
+    st_shared_v4(dst_hi, pack_bf16x2(L.t[2].x * m, L.t[2].y * m), pack_bf16x2(L.t[2].z * m, L.t[2].w * m),
+                 pack_bf16x2(L.t[3].x * m, L.t[3].y * m), pack_bf16x2(L.t[3].z * m, L.t[3].w * m));
 }
 
 // Sampler policy: LDG gathers + software lerp, or texture fetches with hardware filtering.
@@ -228,7 +235,9 @@ struct Sampler<false> {
                                                  uint32_t meta) {
         issue_row(L, xb, meta);
     }
-    static __device__ __forceinline__ void store(const Load& L, uint32_t dst) { lerp_store_row(L, dst); }
+    static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
+        lerp_store_row(L, lo, hi);
+    }
 };
 template <>
 struct Sampler<true> {
@@ -237,7 +246,9 @@ struct Sampler<true> {
                                                  uint32_t meta) {
         issue_row_tex(L, (cudaTextureObject_t)tex, layer, meta);
     }
-    static __device__ __forceinline__ void store(const Load& L, uint32_t dst) { tex_store_row(L, dst); }
+    static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
+        tex_store_row(L, lo, hi);
+    }
 };
 
 // CTA range -> segments helper (every role walks the same sequence).
@@ -395,16 +406,16 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
     }
 }
 
-// One producer warp's share of one segment: for every k-iteration, 4 A rows x 16 bytes per
-// thread, with the next k-iteration's gathers (or texture fetches) issued row by row as
+// One producer warp's share of one segment: for every k-iteration, 2 A rows x 32 bytes per
+// thread (one 256-bit gather per corner), with the next k-iteration's gathers (or texture fetches) issued row by row as
 // soon as the row's registers are free (rolling prefetch).  Warps with TEXW use the texture
 // sampler, the others LDG gathers + software lerp; the metadata table holds each row in the
-// format its warp consumes (warp of row r = (r mod 32) / 4).
+// format its warp consumes (warp of row r = (r mod 64) / 8).
 template <bool TEXW, int STAGES, int NTEX>
 __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
-                                                const uint32_t (&dst)[ROWS], const uint32_t (&mrow)[ROWS],
-                                                uint32_t a_s, uint64_t* empty, uint64_t* full_a, int t,
-                                                int cvec, int lane) {
+                                                const uint32_t (&dst_lo)[ROWS], const uint32_t (&dst_hi)[ROWS],
+                                                const uint32_t (&mrow)[ROWS], uint32_t a_s, uint64_t* empty,
+                                                uint64_t* full_a, int t, int sub, int lane) {
     using Smp = Sampler<TEXW>;
     const int m0 = (sg.tile / a.n_tiles_n) * BM;
     int chunk = sg.kb / a.KK;
@@ -413,12 +424,12 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     named_bar_sync(1, NPT);          // previous table no longer read
     for (int e = t; e < BM * a.KK; e += NPT) {
         const int row = e / a.KK;
-        build_meta_entry(a, m0, row, e - row * a.KK, g, meta, ((row & 31) >> 2) < NTEX);
+        build_meta_entry(a, m0, row, e - row * a.KK, g, meta, ((row % (NPW * RPW)) / RPW) < NTEX);
     }
     named_bar_sync(1, NPT);
-    // position of this thread's 8 channels: byte pointer (LDG) / texture layer (TEX)
-    const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + cvec * 8) * 2;
-    int layer = chunk * (BK / 4) + cvec * 2;
+    // position of this thread's 16 channels: byte pointer (LDG) / texture layer (TEX)
+    const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + sub * 16) * 2;
+    int layer = chunk * (BK / 4) + sub * 4;
     typename Smp::Load L[ROWS];
 #pragma unroll
     for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], xb, a.tex, layer, mrow[p] + tap * META_ENTRY);
@@ -437,7 +448,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         const uint32_t stage = a_s + s * A_STAGE_BYTES;
 #pragma unroll
         for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
-            Smp::store(L[p], stage + dst[p]);
+            Smp::store(L[p], stage + dst_lo[p], stage + dst_hi[p]);
             if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
         }
         fence_proxy_async_smem();
@@ -448,7 +459,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
             named_bar_sync(1, NPT);
             for (int e = t; e < BM * a.KK; e += NPT) {
                 const int row = e / a.KK;
-                build_meta_entry(a, m0, row, e - row * a.KK, ng, meta, ((row & 31) >> 2) < NTEX);
+                build_meta_entry(a, m0, row, e - row * a.KK, ng, meta, ((row % (NPW * RPW)) / RPW) < NTEX);
             }
             named_bar_sync(1, NPT);
             g = ng;
@@ -512,23 +523,26 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     if (warp < NPW) {
         // ===================== A producers =====================
         const int t = threadIdx.x;
-        const int cvec = t & 7;              // 16-byte vector within the 128-byte row
+        const int sub = t & (TPR - 1);       // 32-byte quarter of the 128-byte row
         const uint32_t meta_s = smem_u32(meta);
         const uint32_t a_s = smem_u32(sA);
-        uint32_t dst[ROWS], mrow[ROWS];
+        uint32_t dst_lo[ROWS], dst_hi[ROWS], mrow[ROWS];
 #pragma unroll
         for (int p = 0; p < ROWS; ++p) {
-            const int row = (t >> 3) + p * (NPT / 8);
-            dst[p] = row * 128 + ((cvec ^ (row & 7)) << 4);
+            const int row = (t / TPR) + p * (NPT / TPR);
+            dst_lo[p] = row * 128 + (((2 * sub) ^ (row & 7)) << 4);
+            dst_hi[p] = row * 128 + (((2 * sub + 1) ^ (row & 7)) << 4);
             mrow[p] = meta_s + row * a.KK * META_ENTRY;
         }
         int q = 0;                           // running k-iteration (stage) counter
         for (int o = 0; o < nseg; ++o) {
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
             if (warp < NTEX)
-                produce_segment<true, STAGES, NTEX>(a, sg, q, meta, dst, mrow, a_s, empty, full_a, t, cvec, lane);
+                produce_segment<true, STAGES, NTEX>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
+                                                    t, sub, lane);
             else
-                produce_segment<false, STAGES, NTEX>(a, sg, q, meta, dst, mrow, a_s, empty, full_a, t, cvec, lane);
+                produce_segment<false, STAGES, NTEX>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
+                                                     t, sub, lane);
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
         // segment's epilogue, which would otherwise be exposed at the end of the CTA's range.
