@@ -138,7 +138,7 @@ class Layer:
         import paper_conf_ipps_jayaweeralwrk24_b200 as d
         nws = d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K, c.stride, c.pad,
                                           c.dil, c.G, dt)
-        self.ws = torch.empty(max(nws, 16), dtype=torch.uint8, device=dev)
+        self.ws = torch.zeros(max(nws, 16), dtype=torch.uint8, device=dev)   # zero before first use
         self.tws = torch.empty(d.defcon_offset_workspace_size(c.N, c.H, c.W, c.Cin, c.K, c.stride,
                                                               c.pad, c.dil, c.G),
                                dtype=torch.uint8, device=dev)

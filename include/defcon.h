@@ -135,8 +135,12 @@ int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_
  *   y        [N][Ho][Wo][Cout], dtype `dtype` (written)
  *   workspace / workspace_bytes: device scratch of at least defcon_dcn_workspace_size()
  *            bytes (may be NULL when that size is 0).  The tensor-core path uses it for
- *            stream-K tile counters (reset by the call itself, on `stream`) and fp32
- *            partial tiles; calls that may run concurrently need distinct workspaces.
+ *            stream-K tile counters and fp32 partial tiles.  The workspace must be
+ *            ZERO-FILLED before its first use (e.g. one cudaMemset after allocation); every
+ *            completed call leaves it zero-filled again, so no per-call reset is launched
+ *            (graph-capture friendly).  Calls that may run concurrently need distinct
+ *            workspaces.  The kernels are launched with programmatic dependent launch: their
+ *            prologue may overlap the previous kernel on `stream`, never its data.
  * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G not dividing Cin, bad enums,
  *   NULL required pointers; UNSUPPORTED for (Cin/G) % 8 != 0 (bf16) or % 4 != 0 (fp32),
  *   or a Cout not multiple of 16 on the tensor-core paths; LIMIT when N*H*W*Cin >= 2^31

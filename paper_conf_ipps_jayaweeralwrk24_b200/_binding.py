@@ -51,11 +51,12 @@ class defcon_conv_t(ctypes.Structure):
 _lib = None
 
 
-def load_library(path: str = LIB_PATH):
+def load_library(path: str = None):
     """Load libdefcon.so; raises if it has not been built (no fallback)."""
     global _lib
     if _lib is not None:
         return _lib
+    path = path or os.environ.get("DEFCON_LIB") or LIB_PATH   # DEFCON_LIB: dev-probe builds
     if not os.path.exists(path):
         raise RuntimeError(f"{path} not built: run `python -m paper_conf_ipps_jayaweeralwrk24_b200.build`"
                            " (or __graft_entry__.build())")
@@ -220,7 +221,7 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
         need = defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw, stride, pad, dil,
                                          offset_groups, x.dtype, sampler, fp32_mode)
         if need:
-            workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
+            workspace = torch.zeros(need, dtype=torch.uint8, device=x.device)   # zero before first use
     ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
     plan = None if tex_plan is None else tex_plan.handle
     rc = lib.defcon_dcn_forward(_ptr(x), N, H, W, Cin, _ptr(offset), _ptr(mask), _ptr(weight),

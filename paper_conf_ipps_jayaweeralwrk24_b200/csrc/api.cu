@@ -323,6 +323,10 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
     if (out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h) != g.Ho ||
         out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w) != g.Wo)
         return fail(DEFCON_ERR_INVALID_ARG, "offset-branch grid differs from the DCN grid");
+    if (wsd) {   // the caller's dev_workspace carries no zero-fill guarantee: clear step 2's scratch
+        e = cudaMemsetAsync(wsd, 0, c.ws, st);
+        if (e != cudaSuccess) return cuda_fail(e, "workspace clear");
+    }
     rc = defcon_dcn_forward(xd, N, H, W, Cin, offd, mskd, weight, bias, Cout, K, K, cv, dtype,
                             sampler, fp32_mode, yd, wsd, c.ws, nullptr, stream);
     if (rc) return rc;

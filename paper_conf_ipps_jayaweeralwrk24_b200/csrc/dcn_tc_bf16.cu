@@ -46,6 +46,18 @@ constexpr int TPR = 4;               // producer threads per 128-byte A row (32 
 constexpr int ROWS = BM * TPR / NPT; // A rows per producer thread
 constexpr int RPW = 32 / TPR;        // rows per warp per pass
 
+#ifdef DEFCON_PROBE_TIMELINE   // dev probe: per-CTA phase timestamps (globaltimer, ns)
+__device__ unsigned long long g_tl[256][16];
+__device__ __forceinline__ void tl_stamp(int i) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_tl[blockIdx.x][i] = t;
+}
+#define TL(i) tl_stamp(i)
+#else
+#define TL(i) ((void)0)
+#endif
+
 struct TcArgs {
     const __nv_bfloat16* x;
     const float* offset;
@@ -61,7 +73,15 @@ struct TcArgs {
     int n_tiles_n;         // tiles along Cout
     long long total_iters; // num_tiles * ipt
     unsigned long long tex;          // DEFCON_SAMPLER_TEX: stacked-image texture object, else 0
+    int bias_in_smem;      // Cout <= BIAS_SMEM_MAX: bias (or zeros) staged in shared memory
 };
+
+constexpr int BIAS_SMEM_MAX = 1024;
+
+// Byte offset of the bias table behind the barriers / TMEM slot / fix flags (16-aligned).
+__host__ __device__ constexpr int bias_smem_offset(int stages, int nbuf) {
+    return (((3 * stages + 2 * nbuf) * 8 + 12) + 15) & ~15;
+}
 
 template <int BLOCK_N>
 struct TcCfg {
@@ -93,54 +113,62 @@ struct Segment {
 // Sampling metadata for (row, tap) of offset group g: the byte offset (into x) of
 // channel 0 of each of the 4 bilinear corners and the 4 corner weights with the mask
 // folded in.  Corners outside the image get weight 0 and the harmless in-bounds
-// offset 0 (R8).
-__device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int row, int tap, int g,
-                                                 uint8_t* meta, bool tex_row) {
+// offset 0 (R8).  Built in two passes over a thread's entries -- all offset/mask
+// loads first, then the arithmetic -- so a table costs one memory round trip, not one
+// per entry.
+struct MetaIn {
+    float2 d;     // (dy, dx) offset (R4)
+    float mk;     // mask (1 for DCNv1)
+};
+
+constexpr int META_MAX_PER_THREAD = 6;   // BM * KK / NPT for KK <= 12 (dcn_tc_bf16_supported)
+
+// Output pixel of tile row `row`: image n and the top-left tap position (R3).
+struct RowPos {
+    int n, yb, xb;
+    bool ok;
+};
+
+__device__ __forceinline__ RowPos row_pos(const TcArgs& a, int m) {
+    RowPos p;
+    p.ok = m < a.M;
+    const int mm = p.ok ? m : 0;
+    const int hw = a.Ho * a.Wo;
+    p.n = mm / hw;
+    const int rem = mm - p.n * hw;
+    const int ho = rem / a.Wo;
+    p.yb = ho * a.sh - a.ph;
+    p.xb = (rem - ho * a.Wo) * a.sw - a.pw;
+    return p;
+}
+
+__device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& rp, int i, int j, const MetaIn& in,
+                                                 uint8_t* e, bool tex_row) {
+    const float2 d = in.d;
+    const float mk = in.mk;
     if (tex_row) {
         // texture sampler: unnormalised texel coordinates (texel centres at +0.5, R7) in the
         // stacked-image texture (image n occupies rows n*(H+1) .. n*(H+1)+H-1, row
         // n*(H+1)+H is zero) and the mask.  Clamping to [-1, H] x [-1, W] keeps samples
         // beyond the image on zero texels.
         float4 c = make_float4(-4.f, -4.f, 0.f, 0.f);
-        const int m = m0 + row;
-        if (m < a.M) {
-            const int hw = a.Ho * a.Wo;
-            const int n = m / hw;
-            const int rem = m - n * hw;
-            const int ho = rem / a.Wo;
-            const int wo = rem - ho * a.Wo;
-            const int i = tap / a.Kw;
-            const int j = tap - i * a.Kw;
-            const long pix = (long)m * a.G + g;
-            const float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tap) * 2));
-            const float mk = a.mask ? __ldg(a.mask + pix * a.KK + tap) : 1.0f;
-            const float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
-            const float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
+        if (rp.ok) {
+            const float py = (float)(rp.yb + i * a.dh) + d.x;
+            const float px = (float)(rp.xb + j * a.dw) + d.y;
             if (px == px && py == py) {
                 c.x = fminf(fmaxf(px, -1.0f), (float)a.W) + 0.5f;
-                c.y = (float)(n * (a.H + 1)) + fminf(fmaxf(py, -1.0f), (float)a.H) + 0.5f;
+                c.y = (float)(rp.n * (a.H + 1)) + fminf(fmaxf(py, -1.0f), (float)a.H) + 0.5f;
                 c.z = mk;
             }
         }
-        *reinterpret_cast<float4*>(meta + (row * a.KK + tap) * META_ENTRY) = c;
+        *reinterpret_cast<float4*>(e) = c;
         return;
     }
     uint4 off = make_uint4(0u, 0u, 0u, 0u);
     float4 wt = make_float4(0.f, 0.f, 0.f, 0.f);
-    const int m = m0 + row;
-    if (m < a.M) {
-        const int hw = a.Ho * a.Wo;
-        const int n = m / hw;
-        const int rem = m - n * hw;
-        const int ho = rem / a.Wo;
-        const int wo = rem - ho * a.Wo;
-        const int i = tap / a.Kw;
-        const int j = tap - i * a.Kw;
-        const long pix = (long)m * a.G + g;
-        const float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tap) * 2));
-        const float mk = a.mask ? __ldg(a.mask + pix * a.KK + tap) : 1.0f;
-        float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
-        float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
+    if (rp.ok) {
+        float py = (float)(rp.yb + i * a.dh) + d.x;
+        float px = (float)(rp.xb + j * a.dw) + d.y;
         // Anything beyond one pixel outside samples only zeros; clamping keeps the
         // int conversion defined for huge / non-finite offsets.
         py = fminf(fmaxf(py, -2.0f), (float)a.H + 1.0f);
@@ -151,7 +179,7 @@ __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int ro
             const int y0 = (int)fy, x0 = (int)fx;
             const bool vy0 = (y0 >= 0) && (y0 < a.H), vy1 = (y0 + 1 >= 0) && (y0 + 1 < a.H);
             const bool vx0 = (x0 >= 0) && (x0 < a.W), vx1 = (x0 + 1 >= 0) && (x0 + 1 < a.W);
-            const uint32_t base = (uint32_t)(n * a.H);
+            const uint32_t base = (uint32_t)(rp.n * a.H);
             const uint32_t rowb = (uint32_t)a.Cin * 2u;   // bytes per pixel
             if (vy0 && vx0) { off.x = ((base + y0) * a.W + x0) * rowb;         wt.x = (1.f - ly) * (1.f - lx) * mk; }
             if (vy0 && vx1) { off.y = ((base + y0) * a.W + x0 + 1) * rowb;     wt.y = (1.f - ly) * lx * mk; }
@@ -159,9 +187,64 @@ __device__ __forceinline__ void build_meta_entry(const TcArgs& a, int m0, int ro
             if (vy1 && vx1) { off.w = ((base + y0 + 1) * a.W + x0 + 1) * rowb; wt.w = ly * lx * mk; }
         }
     }
-    uint8_t* e = meta + (row * a.KK + tap) * META_ENTRY;
     *reinterpret_cast<uint4*>(e) = off;
     *reinterpret_cast<float4*>(e + 16) = wt;
+}
+
+// The whole (tile, group) table, built by the NPT = 2*BM producer threads: thread t owns
+// row t/2 and taps (t&1), (t&1)+2, ...  The row's pixel decomposition is done once; the
+// offset/mask loads of a pass are all issued before any arithmetic (one round trip per
+// pass).  Rows of warp w use the format of that warp's sampler.
+static_assert(NPT == 2 * BM, "metadata build assumes two producer threads per tile row");
+template <int NTEX>
+__device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t) {
+    constexpr int PASS = 3;          // taps in flight per thread (register budget)
+    const int row = t >> 1;
+    const RowPos rp = row_pos(a, m0 + row);
+    const bool tex_row = ((row % (NPW * RPW)) / RPW) < NTEX;
+    const long pix = (long)(m0 + row) * a.G + g;
+    uint8_t* rmeta = meta + row * a.KK * META_ENTRY;
+    int tap = t & 1;
+    int i = tap / a.Kw, j = tap - (tap / a.Kw) * a.Kw;
+#pragma unroll 1
+    for (; tap < a.KK;) {
+        MetaIn in[PASS];
+#pragma unroll
+        for (int k = 0; k < PASS; ++k) {
+            const int tk = tap + 2 * k;
+            in[k].d = make_float2(0.f, 0.f);
+            in[k].mk = 0.f;
+            if (rp.ok && tk < a.KK) {
+                in[k].d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tk) * 2));
+                in[k].mk = a.mask ? __ldg(a.mask + pix * a.KK + tk) : 1.0f;
+            }
+        }
+#ifdef DEFCON_PROBE_TL_META
+        if (t == 0) TL(tap < 2 ? 6 : 7);
+#endif
+#pragma unroll
+        for (int k = 0; k < PASS; ++k) {
+            if (tap < a.KK) store_meta_entry(a, rp, i, j, in[k], rmeta + tap * META_ENTRY, tex_row);
+            tap += 2;
+            j += 2;
+            while (j >= a.Kw) { j -= a.Kw; ++i; }
+        }
+    }
+}
+
+// Pull the offsets/mask of the tile a CTA processes next into L2 while the current one runs.
+__device__ __forceinline__ void prefetch_meta_l2(const TcArgs& a, int m0, int t) {
+    if (m0 < 0) return;
+    const int rows = min(BM, a.M - m0);
+    const size_t per_pix = (size_t)a.G * a.KK;
+    const char* o0 = reinterpret_cast<const char*>(a.offset + (size_t)m0 * per_pix * 2);
+    const int o_lines = (int)((rows * per_pix * 8 + 127) / 128);
+    const char* k0 = a.mask ? reinterpret_cast<const char*>(a.mask + (size_t)m0 * per_pix) : nullptr;
+    const int k_lines = a.mask ? (int)((rows * per_pix * 4 + 127) / 128) : 0;
+    for (int l = t; l < o_lines + k_lines; l += NPT) {
+        const char* p = l < o_lines ? o0 + (size_t)l * 128 : k0 + (size_t)(l - o_lines) * 128;
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+    }
 }
 
 // The 4 corner vectors (8 channels each) of one A row and their weights.
@@ -175,15 +258,30 @@ __device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_
     const uint4 wb = ld_shared_v4(meta_addr + 16);
     L.w = make_float4(__uint_as_float(wb.x), __uint_as_float(wb.y), __uint_as_float(wb.z),
                       __uint_as_float(wb.w));
+#ifdef DEFCON_PROBE_SAME_ADDR   // dev probe: every gather hits the same line (L1-resident)
+    L.v[0] = ldg_nc_v8(add_u32(xbase, o.x & 0u));
+    L.v[1] = ldg_nc_v8(add_u32(xbase, o.y & 0u));
+    L.v[2] = ldg_nc_v8(add_u32(xbase, o.z & 0u));
+    L.v[3] = ldg_nc_v8(add_u32(xbase, o.w & 0u));
+#else
     L.v[0] = ldg_nc_v8(add_u32(xbase, o.x));
     L.v[1] = ldg_nc_v8(add_u32(xbase, o.y));
     L.v[2] = ldg_nc_v8(add_u32(xbase, o.z));
     L.v[3] = ldg_nc_v8(add_u32(xbase, o.w));
+#endif
 }
 
 // Eq.3 for 16 channels: sum_q w_q * corner_q, fp32 (packed FFMA2), RNE to bf16, into the
 // two 16-byte swizzled slots of this thread's part of the A row.
 __device__ __forceinline__ void lerp_store_row(const RowLoad& L, uint32_t dst_lo, uint32_t dst_hi) {
+#ifdef DEFCON_PROBE_NO_MATH   // dev probe: no lerp, the 4 corners xor-ed (keeps every load live)
+    uint32_t o[8];
+#pragma unroll
+    for (int h = 0; h < 8; ++h) o[h] = L.v[0].w[h] ^ L.v[1].w[h] ^ L.v[2].w[h] ^ L.v[3].w[h] ^ __float_as_uint(L.w.x);
+    st_shared_v4(dst_lo, o[0], o[1], o[2], o[3]);
+    st_shared_v4(dst_hi, o[4], o[5], o[6], o[7]);
+    return;
+#endif
     uint64_t acc[8];
     const float wq[4] = {L.w.x, L.w.y, L.w.z, L.w.w};
 #pragma unroll
@@ -289,14 +387,47 @@ __device__ __forceinline__ int ld_acquire_gpu(const int* p) {
 // k order to its own TMEM accumulator and writes y; otherwise it publishes its accumulator too
 // (slot = grid + CTA) and whoever arrives last sums all partials.  Fixed summation order in
 // both cases: contributors by ascending k range, owner last -> deterministic.
+// Output tile store: every warp owns 32 rows (its TMEM lane quarter); a group of CS = 32
+// columns is packed to bf16, written to a 2 KB warp-private shared buffer in the 64-byte
+// swizzled layout (conflict-free) and stored by one TMA bulk-tensor store (rows >= M and
+// columns >= Cout are clipped by the TMA unit).  Two buffers alternate per warp.
+constexpr int CS = 32;
+constexpr int EPI_SCRATCH_PER_WARP = 2 * 2048;
+
+__device__ __forceinline__ void store_group_tma(const CUtensorMap* ymap, uint8_t* scratch, int gi,
+                                                const uint32_t (&pk)[CS / 2], int col, int row0,
+                                                int lane) {
+    uint8_t* buf = scratch + (gi & 1) * 2048;
+    if (gi >= 2) {                         // the store that used this buffer has read it
+        if (lane == 0) bulk_wait_read<1>();
+        __syncwarp();
+    }
+    const uint32_t base = smem_u32(buf) + lane * 64;
+#pragma unroll
+    for (int cc = 0; cc < 4; ++cc)
+        st_shared_v4(base + ((cc ^ ((lane >> 1) & 3)) << 4), pk[4 * cc], pk[4 * cc + 1], pk[4 * cc + 2],
+                     pk[4 * cc + 3]);
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {
+        tma_store_2d(ymap, buf, col, row0);
+        bulk_commit();
+    }
+}
+
 template <int BLOCK_N, int NCOLS>
-__device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment& sg, uint32_t tacc,
-                                                 int r, int col0, int bar_id, int nthr, bool leader,
-                                                 int* fix_flag, long long T, int nct) {
-    constexpr int CH = 16;
+__device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensorMap* ymap, const Segment& sg,
+                                                 uint32_t tacc, int r, int col0, int bar_id, int nthr,
+                                                 bool leader, int* fix_flag, long long T, int nct,
+                                                 const float* bias_s, uint8_t* scratch,
+                                                 uint8_t* stage_smem = nullptr, size_t stage_bytes = 0,
+                                                 int sid = 0) {
+    constexpr int CH = 16;     // columns per partial write
+    const int lane = threadIdx.x & 31;
     const int m0 = (sg.tile / a.n_tiles_n) * BM;
     const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
     const int row = m0 + r;
+    const int row0 = m0 + (r & ~31);
     const bool row_ok = row < a.M;
     const bool owner = sg.ke == a.ipt;
     const long long t0 = (long long)sg.tile * a.ipt;
@@ -321,57 +452,102 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
         }
         __threadfence();
     };
-    // y = bias + sum(partials of contributors b_lo..b_hi-1) [+ own accumulator | owner slot]
-    auto finish = [&](bool own_from_tmem) {
+    // y = bias + sum(partials of contributors b_lo..b_hi-1) [+ own accumulator | owner slot],
+    // in this fixed order whichever path runs, CS columns at a time.  With `st` the partial
+    // float4s come from this thread's shared-memory staging slots (finish_staged: slot of
+    // slab j, float4 u at st + (j * spj + u) * st_stride), else from L2.
+    auto sum_group = [&](bool own_from_tmem, int c, int gi, const uint8_t* st, int st_stride, int spj,
+                         int cbase) {
+        uint32_t v[CS];
+        if (own_from_tmem) {
+            tmem_ld_32x32b_x32(tacc + c, v);
+            tmem_ld_wait();
+        }
+        if (n0 + c >= a.Cout) return;      // warp-uniform
+        const int nslab = (b_hi - b_lo) + (own_from_tmem ? 0 : 1);
+        float acc[CS];
+#pragma unroll
+        for (int u = 0; u < CS; ++u) acc[u] = 0.f;
+        if (row_ok) {
 #pragma unroll 1
-        for (int c = col0; c < col0 + NCOLS; c += CH) {
-            uint32_t v[CH];
-            if (own_from_tmem) {
-                tmem_ld_32x32b_x16(tacc + c, v);
-                tmem_ld_wait();
-            }
-            if (!row_ok || n0 + c >= a.Cout) continue;
-            float acc[CH];
+            for (int j = 0; j < nslab; ++j) {
+                const int slot = b_lo + j < b_hi ? b_lo + j : nct + b_hi;
+                float4 f[CS / 4];
 #pragma unroll
-            for (int u = 0; u < CH; ++u) acc[u] = 0.f;
-#pragma unroll 1
-            for (int b = b_lo; b <= b_hi; ++b) {
-                float4 f[CH / 4];
-                if (b < b_hi || !own_from_tmem) {
-                    const int slot = b < b_hi ? b : nct + b;
+                for (int u = 0; u < CS / 4; ++u)
+                    f[u] = st ? *reinterpret_cast<const float4*>(st + (size_t)(j * spj + ((c - cbase) >> 2) + u) * st_stride)
+                              : __ldcg(parts + (size_t)slot * (slot_elems / 4) + (size_t)((c >> 2) + u) * BM + r);
 #pragma unroll
-                    for (int u = 0; u < CH / 4; ++u)
-                        f[u] = __ldcg(parts + (size_t)slot * (slot_elems / 4) + (size_t)((c >> 2) + u) * BM + r);
-                } else {
-#pragma unroll
-                    for (int u = 0; u < CH / 4; ++u)
-                        f[u] = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
-                                           __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
-                }
-#pragma unroll
-                for (int u = 0; u < CH / 4; ++u) {
+                for (int u = 0; u < CS / 4; ++u) {
                     acc[4 * u] += f[u].x; acc[4 * u + 1] += f[u].y;
                     acc[4 * u + 2] += f[u].z; acc[4 * u + 3] += f[u].w;
                 }
             }
-            uint32_t pk[CH / 2];
-#pragma unroll
-            for (int u = 0; u < CH / 2; ++u) {
-                const int co = n0 + c + 2 * u;
-                const float b0 = a.bias ? __ldg(a.bias + co) : 0.f;
-                const float b1 = a.bias ? __ldg(a.bias + co + 1) : 0.f;
-                pk[u] = pack_bf16x2(acc[2 * u] + b0, acc[2 * u + 1] + b1);
-            }
-            uint4* dst = reinterpret_cast<uint4*>(a.y + (size_t)row * a.Cout + n0 + c);
-            dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-            dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
         }
+        if (own_from_tmem) {
+#pragma unroll
+            for (int u = 0; u < CS; ++u) acc[u] += __uint_as_float(v[u]);
+        }
+        uint32_t pk[CS / 2];
+#pragma unroll
+        for (int u = 0; u < CS / 4; ++u) {
+            const int co = n0 + c + 4 * u;
+            float4 bb = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (bias_s) bb = *reinterpret_cast<const float4*>(bias_s + co);     // broadcast
+            else if (a.bias && co < a.Cout) bb = __ldg(reinterpret_cast<const float4*>(a.bias + co));
+            pk[2 * u] = pack_bf16x2(acc[4 * u] + bb.x, acc[4 * u + 1] + bb.y);
+            pk[2 * u + 1] = pack_bf16x2(acc[4 * u + 2] + bb.z, acc[4 * u + 3] + bb.w);
+        }
+        store_group_tma(ymap, scratch, gi, pk, n0 + c, row0, lane);
     };
+    auto drain = [&]() {
+        if (lane == 0) bulk_wait_all();
+        __syncwarp();
+    };
+    auto finish = [&](bool own_from_tmem) {
+        int gi = 0;
+#pragma unroll 1
+        for (int c = col0; c < col0 + NCOLS; c += CS, ++gi) sum_group(own_from_tmem, c, gi, nullptr, 0, 0, 0);
+        drain();
+    };
+    // Staged variant (the producer-run last epilogue, when the pipeline's B stage buffers are
+    // idle): the partial float4s of a pass of `pwc` columns are copied to shared memory with
+    // cp.async first -- all in flight at once, no registers held -- so each pass costs about
+    // one L2 round trip.  Thread `sid` of `nthr` owns slot sid of each float4 row.
+    const int nslab_fast = b_hi - b_lo;
+    int pwc = NCOLS;
+    while (pwc > CS && (size_t)nslab_fast * (pwc / 4) * nthr * 16 > stage_bytes) pwc >>= 1;
+    auto finish_staged = [&](uint8_t* st) {
+        int gi = 0;
+#pragma unroll 1
+        for (int p0 = col0; p0 < col0 + NCOLS; p0 += pwc) {
+            if (row_ok) {
+                for (int j = 0; j < nslab_fast; ++j) {
+                    const float4* src = parts + (size_t)(b_lo + j) * (slot_elems / 4) + (size_t)(p0 >> 2) * BM + r;
+#pragma unroll 4
+                    for (int u = 0; u < pwc / 4; ++u)
+                        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(
+                                         st + (size_t)((j * (pwc / 4) + u) * nthr + sid) * 16)),
+                                     "l"(src + (size_t)u * BM)
+                                     : "memory");
+                }
+                asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+            }
+            if (sid == 0) TL(7);
+#pragma unroll 1
+            for (int c = p0; c < p0 + pwc; c += CS, ++gi)
+                sum_group(true, c, gi, st + (size_t)sid * 16, nthr * 16, pwc / 4, p0);
+        }
+        drain();
+    };
+    const bool staged = stage_smem != nullptr && (size_t)nslab_fast * (pwc / 4) * nthr * 16 <= stage_bytes;
 
     if (owner && ncontrib == 0) {          // whole tile
         finish(true);
         return;
     }
+    // The party that finishes a split tile resets its counter to 0, so the workspace is
+    // zero again after every launch (no per-call memset; see defcon_dcn_forward).
     if (!owner) {                          // non-owner contributor: publish, count
         write_partial(blockIdx.x);
         named_bar_sync(bar_id, nthr);
@@ -382,6 +558,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
         if (last) {                        // owner took the slow path: finish from partials
             __threadfence();
             finish(false);
+            if (leader) a.counters[sg.tile] = 0;
         }
         return;
     }
@@ -390,8 +567,14 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
     named_bar_sync(bar_id, nthr);
     const bool all_in = *fix_flag != 0;
     named_bar_sync(bar_id, nthr);
+#ifndef DEFCON_PROBE_TL_META
+    if (leader && stage_smem) TL(all_in ? 6 : 9);
+#endif
     if (all_in) {                          // fast path: partials + own TMEM accumulator
-        finish(true);
+        if (staged) finish_staged(stage_smem);
+        else finish(true);
+        if (leader) a.counters[sg.tile] = 0;
+        if (leader && stage_smem) TL(8);
         return;
     }
     write_partial(nct + blockIdx.x);       // slow path: publish own accumulator as well
@@ -403,6 +586,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const Segment&
     if (last) {
         __threadfence();
         finish(false);
+        if (leader) a.counters[sg.tile] = 0;
     }
 }
 
@@ -415,18 +599,20 @@ template <bool TEXW, int STAGES, int NTEX>
 __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
                                                 const uint32_t (&dst_lo)[ROWS], const uint32_t (&dst_hi)[ROWS],
                                                 const uint32_t (&mrow)[ROWS], uint32_t a_s, uint64_t* empty,
-                                                uint64_t* full_a, int t, int sub, int lane) {
+                                                uint64_t* full_a, int t, int sub, int lane, int next_m0) {
     using Smp = Sampler<TEXW>;
     const int m0 = (sg.tile / a.n_tiles_n) * BM;
     int chunk = sg.kb / a.KK;
     int tap = sg.kb - chunk * a.KK;
     int g = (chunk * BK) / a.Cg;
     named_bar_sync(1, NPT);          // previous table no longer read
-    for (int e = t; e < BM * a.KK; e += NPT) {
-        const int row = e / a.KK;
-        build_meta_entry(a, m0, row, e - row * a.KK, g, meta, ((row % (NPW * RPW)) / RPW) < NTEX);
-    }
+#ifdef DEFCON_PROBE_TL_META
+    if (t == 0) TL(9);
+#endif
+    build_meta_table<NTEX>(a, m0, g, meta, t);
     named_bar_sync(1, NPT);
+    prefetch_meta_l2(a, next_m0, t);
+    if (t == 0) TL(10 + (q ? 1 : 0));     // metadata table ready (first / later segment)
     // position of this thread's 16 channels: byte pointer (LDG) / texture layer (TEX)
     const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + sub * 16) * 2;
     int layer = chunk * (BK / 4) + sub * 4;
@@ -457,10 +643,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
 
         if (has_next && !prefetch) {          // offset group changes: new table
             named_bar_sync(1, NPT);
-            for (int e = t; e < BM * a.KK; e += NPT) {
-                const int row = e / a.KK;
-                build_meta_entry(a, m0, row, e - row * a.KK, ng, meta, ((row % (NPW * RPW)) / RPW) < NTEX);
-            }
+            build_meta_table<NTEX>(a, m0, ng, meta, t);
             named_bar_sync(1, NPT);
             g = ng;
 #pragma unroll
@@ -475,7 +658,8 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
 
 template <int BLOCK_N, int STAGES, int NTEX>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
-    dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const TcArgs a) {
+    dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const __grid_constant__ CUtensorMap ymap,
+                           const TcArgs a) {
     using Cfg = TcCfg<BLOCK_N>;
 
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -483,7 +667,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                                                ~uintptr_t(1023));
     uint8_t* sA = smem;
     uint8_t* sB = smem + STAGES * A_STAGE_BYTES;
-    uint8_t* meta = sB + STAGES * Cfg::B_STAGE_BYTES;
+    uint8_t* epi_scratch = sB + STAGES * Cfg::B_STAGE_BYTES;   // 4 epilogue warps x 4 KB
+    uint8_t* meta = epi_scratch + 4 * EPI_SCRATCH_PER_WARP;
     uint64_t* bars = reinterpret_cast<uint64_t*>(meta + BM * a.KK * META_ENTRY);
     uint64_t* full_a = bars;
     uint64_t* full_b = bars + STAGES;
@@ -492,6 +677,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     uint64_t* tmem_empty = tmem_full + Cfg::NBUF;
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty + Cfg::NBUF);
     int* fix_flag = reinterpret_cast<int*>(tmem_slot + 1);     // [0] epilogue, [1] producers
+    float* bias_s = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) +
+                                             bias_smem_offset(STAGES, Cfg::NBUF));
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -500,6 +687,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const long long it_begin = range_begin(T, nct, blockIdx.x);
     const long long it_end = range_begin(T, nct, blockIdx.x + 1);
     const int nseg = count_segments(a, it_begin, it_end);
+    if (threadIdx.x == 0) TL(0);
 
     if (warp == TMA_WARP && lane == 0) {
         for (int s = 0; s < STAGES; ++s) {
@@ -513,12 +701,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         fence_barrier_init();
         tma_prefetch_desc(&wmap);
+        tma_prefetch_desc(&ymap);
     }
     if (warp == MMA_WARP) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    // Everything above overlaps the previous kernel's tail (PDL); inputs are read and
+    // outputs / workspace written only after it has completed.
+    griddep_wait();
+    griddep_launch_dependents();
+    if (a.bias_in_smem)
+        for (int i = threadIdx.x; i < a.Cout; i += NUM_THREADS) bias_s[i] = a.bias ? __ldg(a.bias + i) : 0.f;
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    if (threadIdx.x == 0) TL(1);
 
     if (warp < NPW) {
         // ===================== A producers =====================
@@ -537,12 +733,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         int q = 0;                           // running k-iteration (stage) counter
         for (int o = 0; o < nseg; ++o) {
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
+            const int next_m0 = o + 1 < nseg
+                ? (segment_j(a, it_begin, it_end, seg_order(o + 1, nseg)).tile / a.n_tiles_n) * BM : -1;
+            if (t == 0 && o < 4) TL(2 + 2 * o);
             if (warp < NTEX)
                 produce_segment<true, STAGES, NTEX>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
-                                                    t, sub, lane);
+                                                    t, sub, lane, next_m0);
             else
                 produce_segment<false, STAGES, NTEX>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
-                                                     t, sub, lane);
+                                                     t, sub, lane, next_m0);
+            if (t == 0 && o < 4) TL(3 + 2 * o);
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
         // segment's epilogue, which would otherwise be exposed at the end of the CTA's range.
@@ -556,8 +756,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const int r = qd * 32 + lane;
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
             constexpr int SLICE = BLOCK_N / (NPW / 4);
-            epilogue_segment<BLOCK_N, SLICE>(a, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT, t == 0,
-                                             fix_flag + 1, T, nct);
+            if (t == 0) TL(12);
+            // idle pipeline buffers: A stages hold the per-warp store scratch, B stages the
+            // staged stream-K partials
+            epilogue_segment<BLOCK_N, SLICE>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT, t == 0,
+                                             fix_flag + 1, T, nct, a.bias_in_smem ? bias_s : nullptr,
+                                             sA + warp * EPI_SCRATCH_PER_WARP, sB,
+                                             (size_t)STAGES * Cfg::B_STAGE_BYTES, t);
+            if (t == 0) TL(13);
         }
     } else if (warp < EPI_WARP0 + 4) {
         // ===================== epilogue (all processed segments but the last) ============
@@ -569,8 +775,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             mbar_wait(&tmem_full[buf], (uint32_t)(o / Cfg::NBUF) & 1u);
             tc_fence_after();
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
-            epilogue_segment<BLOCK_N, BLOCK_N>(a, sg, tacc, r, 0, 2, 128, threadIdx.x == EPI_WARP0 * 32,
-                                               fix_flag, T, nct);
+            epilogue_segment<BLOCK_N, BLOCK_N>(a, &ymap, sg, tacc, r, 0, 2, 128, threadIdx.x == EPI_WARP0 * 32,
+                                               fix_flag, T, nct, a.bias_in_smem ? bias_s : nullptr,
+                                               epi_scratch + (warp - EPI_WARP0) * EPI_SCRATCH_PER_WARP);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&tmem_empty[buf]);
@@ -587,12 +794,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                     const int s = q % STAGES;
                     mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
+#ifdef DEFCON_PROBE_NO_B   // dev probe: weights never reloaded (stale smem B)
+                    mbar_arrive(&full_b[s]);
+                    (void)n0;
+#else
                     mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
                     const int kd = tap * a.Cin + chunk * BK;
 #pragma unroll
                     for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h)
                         tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + h * Cfg::TMA_BOX_N * 128, &wmap,
                                     &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+#endif
                     if (++tap == a.KK) { tap = 0; ++chunk; }
                 }
             }
@@ -631,6 +843,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 }
                 mma_commit(&tmem_full[buf]);
             }
+            TL(14);
         }
     }
 
@@ -641,6 +854,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         tc_fence_after();
         tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
     }
+    if (threadIdx.x == 0) TL(15);
 }
 
 int num_sms() {
@@ -719,6 +933,18 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
         *detail = "cuTensorMapEncodeTiled failed for the weight tensor";
         return cudaErrorInvalidValue;
     }
+    // y [M][Cout] bf16, stored by the epilogue in 32 x 32 boxes (64-byte swizzle)
+    CUtensorMap ymap;
+    cuuint64_t ydims[2] = {(cuuint64_t)g.Cout, (cuuint64_t)g.M};
+    cuuint64_t ystrides[1] = {(cuuint64_t)g.Cout * 2};
+    cuuint32_t ybox[2] = {(cuuint32_t)CS, 32u};
+    cr = encode(&ymap, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, p.y, ydims, ystrides, ybox, estr,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (cr != CUDA_SUCCESS) {
+        *detail = "cuTensorMapEncodeTiled failed for the output tensor";
+        return cudaErrorInvalidValue;
+    }
     TcArgs a;
     a.x = static_cast<const __nv_bfloat16*>(p.x);
     a.offset = p.offset;
@@ -735,28 +961,32 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.total_iters = plan.total;
     a.tex = tex ? tex_plan_texture(tex) : 0ull;
 
-    cudaError_t e = cudaMemsetAsync(a.counters, 0, plan.counters_bytes, stream);
-    if (e != cudaSuccess) {
-        *detail = "cudaMemsetAsync of the stream-K tile counters failed";
-        return e;
-    }
-    const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + (size_t)BM * g.KK * META_ENTRY +
-                        (3 * STAGES + 2 * Cfg::NBUF) * 8 + 32;
+    a.bias_in_smem = g.Cout <= BIAS_SMEM_MAX ? 1 : 0;
+    // Stream-K tile counters are NOT reset here: the workspace is zero-filled once by its
+    // owner and every launch leaves it zeroed (the finisher of each split tile resets it).
+    const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
+                        (size_t)BM * g.KK * META_ENTRY +
+                        bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0);
     auto kern = !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0>
                 : hybrid ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW / 2>
                          : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW>;
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) {
         *detail = "cudaFuncSetAttribute(MaxDynamicSharedMemorySize) failed";
         return e;
     }
-    kern<<<plan.grid, NUM_THREADS, smem, stream>>>(wmap, a);
-    e = cudaGetLastError();
+    e = launch_pdl(kern, dim3(plan.grid), dim3(NUM_THREADS), smem, stream, wmap, ymap, a);
     if (e != cudaSuccess) *detail = "dcn_fwd_bf16_tc_kernel launch failed";
     return e;
 }
 
 }  // namespace
+
+#ifdef DEFCON_PROBE_TIMELINE
+extern "C" int defcon_debug_timeline(unsigned long long* host) {
+    return (int)cudaMemcpyFromSymbol(host, g_tl, sizeof(g_tl));
+}
+#endif
 
 // Shared-memory budget: stages + metadata for up to 12 taps must fit in 227 KB.
 bool dcn_tc_bf16_supported(const DcnGeom& g) {
@@ -777,7 +1007,10 @@ cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, siz
                                const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
     if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
-    if (g.Cout <= 256) return launch_impl<256, 3>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+#ifndef DEFCON_STAGES_256
+#define DEFCON_STAGES_256 2
+#endif
+    if (g.Cout <= 256) return launch_impl<256, DEFCON_STAGES_256>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 }
 

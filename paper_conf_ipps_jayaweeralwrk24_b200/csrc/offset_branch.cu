@@ -68,6 +68,8 @@ template <bool BF16>
 __global__ void __launch_bounds__(DW_THREADS) dw_bn_relu_kernel(const BranchArgs a) {
     __shared__ __align__(16) float w_s[9 * DW_CH];     // [tap][half][vector][4]
     __shared__ __align__(16) float sc_s[DW_CH], sf_s[DW_CH];
+    griddep_wait();                        // PDL: the previous kernel's writes are visible
+    griddep_launch_dependents();
     const int tid = threadIdx.x;
     const int c0 = blockIdx.y * DW_CH;
     const int cn = min(DW_CH, a.C - c0);                // multiple of 8
@@ -195,6 +197,8 @@ __global__ void __launch_bounds__(PW_WARPS * 32) pw_sigmoid_kernel(const BranchA
     constexpr int OCP = 8 * NT;
     constexpr int STAGE = (PW_PIX + OCP) * PW_S;           // floats per stage
     extern __shared__ __align__(16) float sm[];
+    griddep_wait();                        // PDL: t from dw_bn_relu_kernel is complete
+    griddep_launch_dependents();
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
     const int g = lane >> 2, tq = lane & 3;
@@ -301,8 +305,7 @@ cudaError_t launch_pw(const BranchArgs& a, cudaStream_t stream) {
     auto kern = pw_sigmoid_kernel<NT>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    kern<<<(a.M + PW_PIX - 1) / PW_PIX, PW_WARPS * 32, smem, stream>>>(a);
-    return cudaGetLastError();
+    return launch_pdl(kern, dim3((a.M + PW_PIX - 1) / PW_PIX), dim3(PW_WARPS * 32), smem, stream, a);
 }
 
 }  // namespace
@@ -324,11 +327,8 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     a.OC = a.n_off + a.n_msk;
     if (a.OC > 256) return cudaErrorInvalidValue;   // api.cu maps this to DEFCON_ERR_LIMIT
     dim3 g1((a.M + DW_PIX - 1) / DW_PIX, (C + DW_CH - 1) / DW_CH);
-    if (x_bf16)
-        dw_bn_relu_kernel<true><<<g1, DW_THREADS, 0, stream>>>(a);
-    else
-        dw_bn_relu_kernel<false><<<g1, DW_THREADS, 0, stream>>>(a);
-    cudaError_t e = cudaGetLastError();
+    cudaError_t e = x_bf16 ? launch_pdl(dw_bn_relu_kernel<true>, g1, dim3(DW_THREADS), 0, stream, a)
+                           : launch_pdl(dw_bn_relu_kernel<false>, g1, dim3(DW_THREADS), 0, stream, a);
     if (e != cudaSuccess) return e;
     if (a.OC <= 32) return launch_pw<4>(a, stream);
     if (a.OC <= 64) return launch_pw<8>(a, stream);

@@ -120,6 +120,43 @@ def test_dcn_stream_k_partitions(oracle_mod, d, dev, monkeypatch, ctas):
     assert np.max(np.abs(y - y_default)) <= 2e-2 * np.max(np.abs(ref))
 
 
+@pytest.mark.parametrize("ctas", ["3", "37", "0"])
+def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas):
+    """The workspace is zero-filled once; every launch leaves the stream-K counters at zero
+    (no per-call memset), so repeated launches on one workspace -- plain and CUDA-graph
+    replayed -- give bit-identical y."""
+    c = small("wsclean", Cout=256, Cin=64)
+    L = inputs.gen_layer(c)
+    if ctas != "0":
+        monkeypatch.setenv("DEFCON_MAX_CTAS", ctas)
+    dt = TDT[c.dtype]
+    args = [to_dev(L["x"], dt, dev), to_dev(L["offset"], torch.float32, dev),
+            to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], dt, dev),
+            to_dev(L["bias"], torch.float32, dev)]
+    need = d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K, c.stride, c.pad, c.dil,
+                                       c.G, dt)
+    ws = torch.zeros(need, dtype=torch.uint8, device=dev)
+    y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), dtype=dt, device=dev)
+    fn = lambda: d.defcon_dcn_forward(*args, y=y, workspace=ws)
+    fn()
+    torch.cuda.synchronize()
+    y0 = y.clone()
+    n_tiles = ((c.M + 127) // 128) * ((c.Cout + 255) // 256)
+    assert int(ws[: n_tiles * 4].count_nonzero()) == 0
+    for _ in range(3):
+        fn()
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(4):
+            fn()
+    g.replay()
+    g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(y, y0)
+    assert int(ws[: n_tiles * 4].count_nonzero()) == 0
+
+
 def test_dcn_deterministic(d, dev):
     c = small("det")
     L = inputs.gen_layer(c)

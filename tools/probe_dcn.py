@@ -25,7 +25,7 @@ def time_cfg(c, sampler, reps=200):
     w = torch.from_numpy(L["weight"]).to(dev, dt)
     b = torch.from_numpy(L["bias"]).to(dev)
     y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
-    ws = torch.empty(max(16, d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K,
+    ws = torch.zeros(max(16, d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K,
                                                          c.stride, c.pad, c.dil, c.G, dt, sampler)),
                      dtype=torch.uint8, device=dev)
     plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler in ("tex", "hybrid") else None
