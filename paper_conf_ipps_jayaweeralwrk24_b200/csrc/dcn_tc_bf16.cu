@@ -121,7 +121,6 @@ struct MetaIn {
     float mk;     // mask (1 for DCNv1)
 };
 
-constexpr int META_MAX_PER_THREAD = 6;   // BM * KK / NPT for KK <= 12 (dcn_tc_bf16_supported)
 
 // Output pixel of tile row `row`: image n and the top-left tap position (R3).
 struct RowPos {

@@ -33,7 +33,14 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                  float* offset, float* mask, float* t_ws, cudaStream_t stream);
-size_t offset_branch_workspace(int M, int C);   // bytes of the fp32 t buffer
+size_t offset_branch_workspace(int M, int C);   // bytes of the fp32 t buffer (two-pass path)
+// single-launch branch: dw on CUDA cores -> t in smem -> 1x1 on tcgen05 (3xTF32)
+bool offset_branch_tc_supported(int C, int OC);
+cudaError_t launch_offset_branch_tc(const void* x, bool x_bf16, int N, int H, int W, int C,
+                                    const float* dw_w, const float* dw_scale, const float* dw_shift,
+                                    const float* pw_w, const float* pw_b, int n_off, int n_msk,
+                                    int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
+                                    float* offset, float* mask, cudaStream_t stream);
 
 // ---- step 2, CUDA-core anchor (dcn_simt.cu): fp32 math for fp32 or bf16 storage
 cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaStream_t stream);
