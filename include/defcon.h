@@ -153,6 +153,27 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin,
                        void* y, void* workspace, size_t workspace_bytes,
                        defcon_tex_plan_t tex_plan, void* stream);
 
+/*
+ * The sampling step alone -- the deformable im2col of the "two-step" formulation
+ * (P:69-76), Eq.3 with the mask (R6), zero outside the image:
+ *   columns[(n*Ho + ho)*Wo + wo][k*Cin + ci] = m[n][ho][wo][g][k] * X(n, ci, p_y, p_x)
+ * with k, g, p_y, p_x exactly as in defcon_dcn_forward below.  y = columns . W^T + bias
+ * (W viewed as [Cout][Kh*Kw*Cin]) is then the layer output: this is the unfused
+ * baseline's first step and the measurement of the sampling stage on its own.
+ * Arguments
+ *   x        [N][H][W][Cin], dtype `dtype` (DEFCON_BF16 or DEFCON_F32)
+ *   offset, mask  as in defcon_dcn_forward (mask may be NULL: DCNv1)
+ *   columns  [N*Ho*Wo][Kh*Kw*Cin], dtype `dtype` (written; bf16 rounded to nearest even
+ *            from the fp32 bilinear sum)
+ * Ownership: caller owns every buffer; asynchronous on `stream`; no workspace.
+ * Errors: as defcon_dcn_forward (INVALID_ARG, UNSUPPORTED for (Cin/G) % 16 (bf16) or % 8
+ *   (fp32) != 0 -- 32-byte gathers --, LIMIT when the column matrix has >= 2^31 elements,
+ *   MISALIGNED).
+ */
+int defcon_deform_columns(const void* x, int N, int H, int W, int Cin,
+                          const float* offset, const float* mask, int Kh, int Kw,
+                          defcon_conv_t cv, int dtype, void* columns, void* stream);
+
 /* Device workspace defcon_dcn_forward needs for these arguments (0 if none). */
 int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
                               defcon_conv_t cv, int dtype, int sampler, int fp32_mode,

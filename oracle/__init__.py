@@ -57,6 +57,8 @@ def _load():
         lib.oracle_dcn_pixels_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, i,
                                               i, i, i, i, i, i, i, i, i,
                                               ctypes.POINTER(ctypes.c_int64), i, dp]
+        lib.oracle_deform_columns_f64.argtypes = [dp, i, i, i, i, dp, dp, i, i, i, i, i, i, i, i, i,
+                                                  ctypes.POINTER(ctypes.c_int64), ctypes.c_long, dp]
         lib.oracle_offset_branch_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, dp,
                                                  i, i, i, i, i, i, dp, dp]
         lib.oracle_bilinear_f64.argtypes = [dp, i, i, ctypes.c_long, ctypes.c_double,
@@ -169,6 +171,34 @@ def dcn_pixels(x, offset, weight, pix_idx, bias=None, mask=None, stride=1, pad=1
         int(idx.size), _p(out))
     if rc:
         raise ValueError(f"oracle_dcn_pixels_f64 rc={rc}")
+    return out
+
+
+def deform_columns(x, offset, K, pix_idx=None, mask=None, stride=1, pad=1, dil=1, G=1):
+    """Sampling step alone (Eq.3 + mask): the deformable im2col rows.
+
+    Returns cols [n_pix, K*K*Cin] fp64 with cols[t, k*Cin + ci] = m_k * X(p_k) for the
+    flattened output pixels pix_idx (all pixels when None); K = (Kh, Kw) or int.
+    """
+    x, offset, mask = map(_f64, (x, offset, mask))
+    Kh, Kw = _pair(K)
+    N, H, W, Cin = x.shape
+    sh, sw = _pair(stride)
+    ph, pw = _pair(pad)
+    dh, dw = _pair(dil)
+    Ho, Wo = out_size(H, Kh, sh, ph, dh), out_size(W, Kw, sw, pw, dw)
+    if offset.shape != (N, Ho, Wo, G, Kh * Kw, 2):
+        raise ValueError("offset shape")
+    if pix_idx is None:
+        pix_idx = np.arange(N * Ho * Wo)
+    idx = np.ascontiguousarray(np.asarray(pix_idx, dtype=np.int64))
+    out = np.empty((idx.size, Kh * Kw * Cin), np.float64)
+    rc = _load().oracle_deform_columns_f64(_p(x), N, H, W, Cin, _p(offset), _p(mask), Kh, Kw, sh, sw,
+                                           ph, pw, dh, dw, G,
+                                           idx.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                           int(idx.size), _p(out))
+    if rc:
+        raise ValueError(f"oracle_deform_columns_f64 rc={rc}")
     return out
 
 

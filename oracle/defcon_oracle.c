@@ -138,12 +138,12 @@ int oracle_out_size(int in, int k, int stride, int pad, int dil) {
  * dp_k = (offset[..][g][k][0], offset[..][g][k][1]) = (dy, dx) (R4).
  * Built as col[k][ci] first, then one dot product per co.
  */
-static void dcn_one_pixel(const double *x, int H, int W, int Cin,
+/* The sampled column of one output pixel: col[k*Cin + ci] = m[g][k] * X(p_o + p_k + dp_k)
+ * (Eq.3 with the mask, R6); the deformable analogue of an im2col row ("two-step"). */
+static void dcn_pixel_col(const double *x, int H, int W, int Cin,
                           const double *off_px, const double *mask_px,
-                          const double *weight, const double *bias, int Cout,
                           int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
-                          int G, int n, int ho, int wo, int quant_mode,
-                          double *col, double *y_px) {
+                          int G, int n, int ho, int wo, int quant_mode, double *col) {
     const int KK = Kh * Kw;
     const int Cg = Cin / G;
     const double *img = x + (long)n * H * W * Cin;
@@ -164,6 +164,17 @@ static void dcn_one_pixel(const double *x, int H, int W, int Cin,
             }
         }
     }
+}
+
+static void dcn_one_pixel(const double *x, int H, int W, int Cin,
+                          const double *off_px, const double *mask_px,
+                          const double *weight, const double *bias, int Cout,
+                          int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
+                          int G, int n, int ho, int wo, int quant_mode,
+                          double *col, double *y_px) {
+    const int KK = Kh * Kw;
+    dcn_pixel_col(x, H, W, Cin, off_px, mask_px, Kh, Kw, sh, sw, ph, pw, dh, dw, G, n, ho, wo,
+                  quant_mode, col);
     for (int co = 0; co < Cout; ++co) {
         const double *wr = weight + (long)co * KK * Cin; /* [Kh][Kw][Cin] == [k][ci] */
         double acc = 0.0;
@@ -348,4 +359,30 @@ int oracle_offset_branch_f64(const double *x, int N, int H, int W, int C,
         free(t);
     }
     return fail ? 2 : 0;
+}
+
+/* Deformable columns (the sampling step alone, P:69-76 / Eq.3 + mask): for each flattened
+ * output pixel pix_idx[t] = (n*Ho + ho)*Wo + wo, cols[t][k*Cin + ci] as in dcn_pixel_col.
+ * Returns 0 on success, 1 on invalid arguments. */
+int oracle_deform_columns_f64(const double *x, int N, int H, int W, int Cin,
+                              const double *offset, const double *mask,
+                              int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
+                              int G, const int64_t *pix_idx, long n_pix, double *cols) {
+    int Ho = oracle_out_size(H, Kh, sh, ph, dh);
+    int Wo = oracle_out_size(W, Kw, sw, pw, dw);
+    if (dcn_check(N, H, W, Cin, 1, Kh, Kw, sh, sw, dh, dw, G, Ho, Wo)) return 1;
+    const long KKC = (long)Kh * Kw * Cin;
+    for (long t = 0; t < n_pix; ++t)
+        if (pix_idx[t] < 0 || pix_idx[t] >= (long)N * Ho * Wo) return 1;
+#pragma omp parallel for schedule(dynamic, 16)
+    for (long t = 0; t < n_pix; ++t) {
+        long pix = pix_idx[t];
+        int n = (int)(pix / ((long)Ho * Wo));
+        int rem = (int)(pix % ((long)Ho * Wo));
+        int ho = rem / Wo, wo = rem % Wo;
+        dcn_pixel_col(x, H, W, Cin, offset + pix * G * Kh * Kw * 2,
+                      mask ? mask + pix * G * Kh * Kw : NULL, Kh, Kw, sh, sw, ph, pw, dh, dw, G,
+                      n, ho, wo, 0, cols + t * KKC);
+    }
+    return 0;
 }

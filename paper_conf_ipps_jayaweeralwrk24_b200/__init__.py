@@ -9,6 +9,7 @@ from ._binding import (  # noqa: F401
     TexPlan,
     defcon_abi_version,
     defcon_dcn_forward,
+    defcon_deform_columns,
     defcon_dcn_workspace_size,
     defcon_layer_forward_host,
     defcon_layer_workspace_size,

@@ -24,7 +24,7 @@ DEFCON_FP32_3XTF32, DEFCON_FP32_SIMT = 0, 1
 # Every symbol include/defcon.h declares (checked by tests/test_abi.py).
 EXPORTED = (
     "defcon_offset_dw_conv", "defcon_offset_workspace_size", "defcon_dcn_forward",
-    "defcon_dcn_workspace_size",
+    "defcon_dcn_workspace_size", "defcon_deform_columns",
     "defcon_layer_forward_host", "defcon_layer_workspace_size", "defcon_tex_plan_create",
     "defcon_tex_plan_destroy", "defcon_tex_filter_probe", "defcon_status_string",
     "defcon_last_error_detail", "defcon_abi_version",
@@ -70,6 +70,7 @@ def load_library(path: str = None):
                                        sz, vp, vp]
     lib.defcon_dcn_workspace_size.argtypes = [i, i, i, i, i, i, i, conv, i, i, i,
                                               ctypes.POINTER(sz)]
+    lib.defcon_deform_columns.argtypes = [vp, i, i, i, i, fp, fp, i, i, conv, i, vp, vp]
     lib.defcon_layer_forward_host.argtypes = [vp, i, i, i, i, i, fp, fp, fp, fp, fp, vp, fp, i, i,
                                               conv, i, i, i, vp, vp, sz, vp]
     lib.defcon_layer_workspace_size.argtypes = [i, i, i, i, i, i, i, conv, i, i, i,
@@ -230,6 +231,30 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
                                 _stream_handle(stream))
     _check(rc, "defcon_dcn_forward")
     return y
+
+
+def defcon_deform_columns(x, offset, mask, K=3, stride=1, pad=1, dil=1, offset_groups=1, columns=None,
+                          stream=None):
+    """Sampling step alone (Eq.3 P:63-67 + mask, the "two-step" split P:69-76): returns the
+    deformable columns [N*Ho*Wo, K*K*Cin] in x's dtype."""
+    lib = load_library()
+    _dev_tensor(x, "x")
+    if x.dtype not in _DTYPES:
+        raise ValueError("x must be float32 or bfloat16")
+    N, H, W, Cin = x.shape
+    Kh, Kw = (K, K) if isinstance(K, int) else K
+    cv = _conv(stride, pad, dil, offset_groups)
+    Ho, Wo = _out(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w)
+    G = int(offset_groups)
+    _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
+    _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
+    if columns is None:
+        columns = torch.empty((N * Ho * Wo, Kh * Kw * Cin), device=x.device, dtype=x.dtype)
+    _dev_tensor(columns, "columns", x.dtype, (N * Ho * Wo, Kh * Kw * Cin))
+    rc = lib.defcon_deform_columns(_ptr(x), N, H, W, Cin, _ptr(offset), _ptr(mask), Kh, Kw, cv,
+                                   _DTYPES[x.dtype], _ptr(columns), _stream_handle(stream))
+    _check(rc, "defcon_deform_columns")
+    return columns
 
 
 def defcon_layer_workspace_size(N, H, W, Cin, Cout, K=3, stride=1, pad=1, dil=1, offset_groups=1,

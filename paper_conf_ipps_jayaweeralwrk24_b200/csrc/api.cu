@@ -253,6 +253,28 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     return DEFCON_OK;
 }
 
+int defcon_deform_columns(const void* x, int N, int H, int W, int Cin, const float* offset,
+                          const float* mask, int Kh, int Kw, defcon_conv_t cv, int dtype, void* columns,
+                          void* stream) {
+    g_detail[0] = 0;
+    DcnGeom g;
+    int rc = make_geom(N, H, W, Cin, 1, Kh, Kw, cv, dtype, &g);
+    if (rc) return rc;
+    if (!x || !offset || !columns) return fail(DEFCON_ERR_INVALID_ARG, "NULL tensor pointer");
+    const void* ptrs[] = {x, offset, mask, columns};
+    for (const void* p : ptrs)
+        if (p && !aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "tensor pointer not 16-byte aligned");
+    if ((long)g.M * g.KK * Cin >= (1L << 31))
+        return fail(DEFCON_ERR_LIMIT, "column matrix too large for 32-bit element indexing");
+    const int vec = dtype == DEFCON_BF16 ? 16 : 8;     // 32-byte pieces within one offset group
+    if (g.Cg % vec != 0)
+        return fail(DEFCON_ERR_UNSUPPORTED, "columns need Cin/G %% %d == 0 for this dtype", vec);
+    cudaError_t e = launch_deform_columns(g, x, offset, mask, dtype == DEFCON_BF16, columns,
+                                          static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "deform_columns launch");
+    return DEFCON_OK;
+}
+
 // ---------------------------------------------------------------- end-to-end host entry
 static size_t align_up(size_t v) { return (v + 255) & ~size_t(255); }
 

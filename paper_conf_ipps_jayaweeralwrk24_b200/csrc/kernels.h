@@ -42,6 +42,10 @@ cudaError_t launch_offset_branch_tc(const void* x, bool x_bf16, int N, int H, in
                                     int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                     float* offset, float* mask, cudaStream_t stream);
 
+// ---- sampling step alone: deformable columns [M][KK*Cin] (sampler.cu)
+cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* offset, const float* mask,
+                                  bool bf16, void* cols, cudaStream_t stream);
+
 // ---- step 2, CUDA-core anchor (dcn_simt.cu): fp32 math for fp32 or bf16 storage
 cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaStream_t stream);
 

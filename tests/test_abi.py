@@ -134,3 +134,20 @@ def test_product_never_imports_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "oracle" not in src.lower(), f
+
+
+def test_deform_columns_validation(lib):
+    """defcon_deform_columns rejects bad arguments before any launch (no GPU needed)."""
+    V = ctypes.c_void_p
+    lib.defcon_deform_columns.restype = ctypes.c_int
+
+    def call(x=FAKE, N=1, H=8, W=8, Cin=64, off=FAKE, mask=FAKE, K=3, cv=None, dtype=1, cols=FAKE):
+        return lib.defcon_deform_columns(V(x), N, H, W, Cin, V(off), V(mask), K, K, cv or _conv(), dtype,
+                                         V(cols), None)
+
+    assert call(N=0) == 1
+    assert call(x=0) == 1 and call(cols=0) == 1
+    assert call(cv=_conv(offset_groups=3)) == 1          # G does not divide Cin
+    assert call(cols=FAKE + 8) == 3                      # misaligned
+    assert call(cv=_conv(offset_groups=8)) == 2          # Cin/G = 8: 32-byte bf16 pieces need 16
+    assert call(dtype=5) == 1

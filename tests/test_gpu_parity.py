@@ -183,6 +183,32 @@ def test_dcn_full_size_sampled(oracle_mod, d, dev, c):
     assert normwise(y[idx], ref) < TOL[c.dtype]
 
 
+STACK = [l.replace(N=2) for l in configs.stack_layers(64) if l.name in ("stack_c3b0", "stack_c4b0", "stack_c4b3",
+                                                                      "stack_c5b0")]
+
+
+@pytest.mark.parametrize("c", STACK, ids=lambda c: c.name)
+def test_stack_layers_with_branch_sampled(oracle_mod, d, dev, c):
+    """Config 5 (interval-3 DCN stack): the stride-2 stage-entry layers and a stride-1 C4
+    layer, each fed by its own offset branch, at 2 images; sampled pixels vs the oracle
+    run on the oracle's own offsets (the branch itself is checked to 1e-5 elsewhere)."""
+    x = inputs.gen_x(c)
+    P, Pd = gen_branch_dev(c, dev)
+    w, b = inputs.gen_weight(c)
+    xd = to_dev(x, torch.bfloat16, dev)
+    off, msk = d.defcon_offset_dw_conv(xd, Pd["dw_w"], Pd["dw_scale"], Pd["dw_shift"], Pd["pw_w"], Pd["pw_b"],
+                                       K=c.K, stride=c.stride, pad=c.pad, dil=c.dil)
+    y = d.defcon_dcn_forward(xd, off, msk, to_dev(w, torch.bfloat16, dev), to_dev(b, torch.float32, dev),
+                             stride=c.stride, pad=c.pad, dil=c.dil)
+    torch.cuda.synchronize()
+    ro, rm = oracle_mod.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"], P["pw_b"],
+                                      K=c.K, stride=c.stride, pad=c.pad, dil=c.dil)
+    r = np.random.default_rng(11)
+    idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(c.M - 64, c.M), r.integers(0, c.M, 200)]))
+    ref = oracle_mod.dcn_pixels(x, ro, w, idx, b, mask=rm, stride=c.stride, pad=c.pad, dil=c.dil)
+    assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
+
+
 def gen_branch_dev(c, dev):
     P = inputs.gen_offset_branch(c)
     return P, {k: to_dev(v, torch.float32, dev) for k, v in P.items()}
@@ -284,3 +310,46 @@ def test_tex_sampler_parity(oracle_mod, d, dev, c, sampler):
     assert e_q < 1e-2
     assert e_x < 5e-3
     plan.close()
+
+
+# ------------------------------------------------------------------ sampling step alone
+@pytest.mark.parametrize("c", [small("cols_bf16", Cin=64), small("cols_f32_g4_s2", dtype="f32", Cin=32, G=4, stride=2),
+                               small("cols_v1_g2", Cin=64, G=2, modulated=False),
+                               configs.C5.replace(N=2)],
+                         ids=lambda c: c.name)
+def test_deform_columns_parity(oracle_mod, d, dev, c):
+    """defcon_deform_columns vs the oracle's columns, element by element on sampled rows:
+    bf16 = RNE of the fp32 bilinear sum (|err| <= 2^-8 |ref| + 1e-6 max|ref|), fp32 1e-5."""
+    L = inputs.gen_layer(c)
+    dt = TDT[c.dtype]
+    cols = d.defcon_deform_columns(to_dev(L["x"], dt, dev), to_dev(L["offset"], torch.float32, dev),
+                                   to_dev(L["mask"], torch.float32, dev), K=c.K, stride=c.stride, pad=c.pad,
+                                   dil=c.dil, offset_groups=c.G)
+    torch.cuda.synchronize()
+    rng_ = np.random.default_rng(7)
+    idx = np.unique(np.concatenate([[0, c.M - 1], rng_.integers(0, c.M, 300)]))
+    ref = oracle_mod.deform_columns(L["x"], L["offset"], c.K, pix_idx=idx, mask=L["mask"], stride=c.stride,
+                                    pad=c.pad, dil=c.dil, G=c.G)
+    g = cols.float().cpu().numpy()[idx]
+    scale = np.max(np.abs(ref))
+    if c.dtype == "bf16":
+        assert np.all(np.abs(g - ref) <= 2.0 ** -8 * np.abs(ref) + 1e-6 * scale)
+    else:
+        assert np.max(np.abs(g - ref)) <= 1e-5 * scale
+
+
+def test_unfused_columns_gemm_matches_fused(oracle_mod, d, dev):
+    """Two-step baseline (columns, then a library GEMM) and the fused kernel agree with the
+    oracle at the bf16 tolerance (the contraction itself is cuBLAS here: comparison only)."""
+    c = small("twostep", Cin=128, Cout=128)
+    L = inputs.gen_layer(c)
+    xd = to_dev(L["x"], torch.bfloat16, dev)
+    off, msk = to_dev(L["offset"], torch.float32, dev), to_dev(L["mask"], torch.float32, dev)
+    w = to_dev(L["weight"], torch.bfloat16, dev)
+    cols = d.defcon_deform_columns(xd, off, msk)
+    y2 = (cols.float() @ w.reshape(c.Cout, -1).float().t() + to_dev(L["bias"], torch.float32, dev))
+    y1 = d.defcon_dcn_forward(xd, off, msk, w, to_dev(L["bias"], torch.float32, dev))
+    torch.cuda.synchronize()
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"]).reshape(-1, c.Cout)
+    assert normwise(y2.cpu().numpy(), ref) < TOL["bf16"]
+    assert normwise(y1.float().cpu().numpy().reshape(-1, c.Cout), ref) < TOL["bf16"]

@@ -325,3 +325,29 @@ def test_inputs_are_seeded_per_image():
     assert np.array_equal(full[2:3], part)
     xb = inputs.gen_x(c)
     assert np.array_equal(inputs.round_to(xb, "bf16"), xb)
+
+
+# ------------------------------------------------------------------ deformable columns
+def test_columns_zero_offsets_equal_unfold(oracle_mod):
+    """Sampling step alone: zero offsets, no mask -> the regular im2col rows,
+    i.e. F.unfold of the zero-padded input (fp64), reordered to [pixel][tap][ci]."""
+    for stride, dil in ((1, 1), (2, 1), (1, 2)):
+        x, _, _, off, _, _, _ = rand_layer(N=2, H=7, W=9, Cin=6, stride=stride, pad=dil, dil=dil, seed=3)
+        off = np.zeros_like(off)
+        cols = oracle_mod.deform_columns(x, off, 3, stride=stride, pad=dil, dil=dil)
+        u = F.unfold(nchw(x), 3, dilation=dil, padding=dil, stride=stride)   # [N, Cin*9, L]
+        N, Cin = x.shape[0], x.shape[3]
+        ref = u.reshape(N, Cin, 9, -1).permute(0, 3, 2, 1).reshape(-1, 9 * Cin).numpy()
+        assert cols.shape == ref.shape
+        assert np.max(np.abs(cols - ref)) < 1e-14
+
+
+def test_columns_times_weight_is_dcn(oracle_mod):
+    """cols . W^T + b reproduces the (independently pinned) DCN forward, with mask and
+    offset groups -- the columns carry every sampled, modulated value of Eq.2."""
+    x, w, b, off, m, _, _ = rand_layer(N=2, H=6, W=8, Cin=8, Cout=5, G=2, seed=4)
+    y = oracle_mod.dcn_forward(x, off, w, b, mask=m, G=2)
+    idx = np.array([0, 5, 17, 33, 47, 95])
+    cols = oracle_mod.deform_columns(x, off, 3, pix_idx=idx, mask=m, G=2)
+    yy = cols @ w.reshape(w.shape[0], -1).T + b
+    assert np.max(np.abs(yy - y.reshape(-1, w.shape[0])[idx])) < 1e-12
