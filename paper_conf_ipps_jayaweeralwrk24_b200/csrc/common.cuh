@@ -115,6 +115,17 @@ DEFCON_DEVICE void tma_load_2d(void* smem_dst, const CUtensorMap* map, uint64_t*
         : "memory");
 }
 
+// 4-D tiled TMA load global -> shared (coordinates innermost first; out-of-bounds elements of the
+// box are zero-filled), completion signalled on `bar` (tx bytes = the full box).
+DEFCON_DEVICE void tma_load_4d(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                               int c2, int c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(smem_u32(smem_dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+}
+
 // 2-D tiled TMA store shared -> global (bulk async-group completion).  Elements of the box
 // outside the tensor are not written (row / column tails are clipped by the TMA unit).
 DEFCON_DEVICE void tma_store_2d(const CUtensorMap* map, const void* smem_src, int c0, int c1) {

@@ -15,6 +15,7 @@
 // bf16 x is widened exactly; all sums are fp32.
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -330,12 +331,18 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     a.n_msk = with_mask ? G * K * K : 0;
     a.OC = a.n_off + a.n_msk;
     if (a.OC > 256) return cudaErrorInvalidValue;   // api.cu maps this to DEFCON_ERR_LIMIT
-    // Two launches by default (measured fastest at the YOLACT++ shapes);
-    // DEFCON_OFFSET_TC=1 selects the single-launch tensor-core branch (offset_branch_tc.cu:
-    // t stays on chip, 1x1 on tcgen05 with 3xTF32).  Both paths are parity-tested.
-    if (getenv("DEFCON_OFFSET_TC") && offset_branch_tc_supported(C, a.OC))
+    // Two launches by default (measured fastest at the YOLACT++ shapes).
+    // DEFCON_OFFSET_IMPL=tc (or DEFCON_OFFSET_TC=1) selects the single-launch tcgen05 branch
+    // (offset_branch_tc.cu: t stays on chip), =row_tc the row-tile kernel with TMA-staged input
+    // (offset_branch_fused.cu).  All three are parity-tested.
+    const char* impl = getenv("DEFCON_OFFSET_IMPL");
+    if (((impl && !strcmp(impl, "tc")) || getenv("DEFCON_OFFSET_TC")) && offset_branch_tc_supported(C, a.OC))
         return launch_offset_branch_tc(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b, a.n_off,
                                        a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset, mask, stream);
+    if (impl && !strcmp(impl, "row_tc") && offset_branch_fused_supported(C, a.OC, Wo, s_w, d_w, d_h, x_bf16))
+        return launch_offset_branch_fused(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
+                                          a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
+                                          mask, stream);
     dim3 g1((a.M + DW_PIX - 1) / DW_PIX, (C + DW_CH - 1) / DW_CH);
     cudaError_t e = x_bf16 ? launch_pdl(dw_bn_relu_kernel<true>, g1, dim3(DW_THREADS), 0, stream, a)
                            : launch_pdl(dw_bn_relu_kernel<false>, g1, dim3(DW_THREADS), 0, stream, a);

@@ -214,16 +214,16 @@ def gen_branch_dev(c, dev):
     return P, {k: to_dev(v, torch.float32, dev) for k, v in P.items()}
 
 
-@pytest.mark.parametrize("path", ["tc", "two_pass"])
+@pytest.mark.parametrize("path", ["row_tc", "tc", "two_pass"])
 @pytest.mark.parametrize("c", [configs.C3.replace(N=2), configs.C4_G4.replace(N=2),
                                small("branch_s2_f32", dtype="f32", stride=2, Cin=48, modulated=False),
                                small("branch_d2", dil=2, pad=2, Cin=40, H=15, W=23),
                                configs.C5.replace(N=1), configs.C4],
                          ids=lambda c: c.name)
 def test_offset_branch_parity(oracle_mod, d, dev, monkeypatch, c, path):
-    """Single-launch tcgen05 branch (t kept on chip) and the two-launch path, vs the oracle."""
-    if path == "tc":
-        monkeypatch.setenv("DEFCON_OFFSET_TC", "1")
+    """All three branch kernels vs the oracle: the default two-launch path ("two_pass"), the
+    single-launch tcgen05 kernel ("tc") and the TMA-staged row-tile kernel ("row_tc")."""
+    monkeypatch.setenv("DEFCON_OFFSET_IMPL", path)
     x = inputs.gen_x(c)
     P, Pd = gen_branch_dev(c, dev)
     off, msk = d.defcon_offset_dw_conv(to_dev(x, TDT[c.dtype], dev), Pd["dw_w"], Pd["dw_scale"],

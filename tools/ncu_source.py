@@ -8,7 +8,8 @@ start = [i for i, l in enumerate(lines) if l.startswith('"Address"')]
 rows = list(csv.reader(lines[start[0]:]))
 h = rows[0]
 ix = {k: i for i, k in enumerate(h)}
-data = [r for r in rows[1:] if len(r) == len(h)]
+data = [r for r in rows[1:] if len(r) == len(h) and r[0] != "Address"]
+seen = set(); data = [r for r in data if not (r[0] in seen or seen.add(r[0]))]
 S = "Warp Stall Sampling (All Samples)"
 tot = sum(int(r[ix[S]] or 0) for r in data)
 stall_cols = [k for k in h if k.startswith("stall_") and "Not Issued" not in k]

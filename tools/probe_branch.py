@@ -1,8 +1,9 @@
 """Time the lightweight offset branch (defcon_offset_dw_conv) alone, graph-replayed, per config.
 
   python tools/probe_branch.py [config,...]
-Prints one JSON line per (config, path): single-launch tcgen05 kernel ("fused"), and the two-launch
-(dw, then 1x1) default path; DEFCON_OFFSET_TC=1 selects the tcgen05 kernel.
+Prints one JSON line per (config, path): the default two-launch path ("two_pass"), the
+single-launch tcgen05 kernel ("tc") and the TMA-staged row-tile kernel ("row_tc"), selected
+through DEFCON_OFFSET_IMPL.
 """
 import json
 import os
@@ -50,13 +51,10 @@ if __name__ == "__main__":
     d.load_library()
     for n in names:
         c = configs.SINGLE_LAYER[n]
-        for path in ("tc", "two_pass"):
-            if path == "tc":
-                os.environ["DEFCON_OFFSET_TC"] = "1"
-            else:
-                os.environ.pop("DEFCON_OFFSET_TC", None)
+        for path in ("row_tc", "tc", "two_pass"):
+            os.environ["DEFCON_OFFSET_IMPL"] = path
             us = time_branch(c)
             byt = configs.offset_branch_compulsory_bytes(c)
             print(json.dumps({"config": n, "path": path, "us": round(us, 2),
                               "GB/s(compulsory)": round(byt / (us * 1e-6) / 1e9, 1)}))
-    os.environ.pop("DEFCON_OFFSET_TC", None)
+    os.environ.pop("DEFCON_OFFSET_IMPL", None)
