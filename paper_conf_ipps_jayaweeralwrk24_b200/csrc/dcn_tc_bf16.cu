@@ -195,9 +195,12 @@ __device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& 
 // offset/mask loads of a pass are all issued before any arithmetic (one round trip per
 // pass).  Rows of warp w use the format of that warp's sampler.
 static_assert(NPT == 2 * BM, "metadata build assumes two producer threads per tile row");
+#ifndef DEFCON_META_PASS
+#define DEFCON_META_PASS 3
+#endif
 template <int NTEX>
 __device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t) {
-    constexpr int PASS = 3;          // taps in flight per thread (register budget)
+    constexpr int PASS = DEFCON_META_PASS;   // taps in flight per thread (register budget)
     const int row = t >> 1;
     const RowPos rp = row_pos(a, m0 + row);
     const bool tex_row = ((row % (NPW * RPW)) / RPW) < NTEX;

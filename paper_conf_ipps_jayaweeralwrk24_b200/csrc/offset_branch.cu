@@ -68,8 +68,11 @@ __device__ __forceinline__ void load8(const void* x, long idx, float (&v)[8]) {
 // loop needs no branches.
 __device__ __align__(32) const uint32_t g_zero32[8] = {0, 0, 0, 0, 0, 0, 0, 0};
 
+#ifndef DEFCON_DW_MINBLOCKS
+#define DEFCON_DW_MINBLOCKS 3   // <= 85 registers: 3 blocks per SM, C4 grid of 616 blocks in 2 rounds, not 3
+#endif
 template <bool BF16>
-__global__ void __launch_bounds__(DW_THREADS) dw_bn_relu_kernel(const BranchArgs a) {
+__global__ void __launch_bounds__(DW_THREADS, DEFCON_DW_MINBLOCKS) dw_bn_relu_kernel(const BranchArgs a) {
     __shared__ __align__(16) float w_s[9 * DW_CH];     // [tap][half][vector][4]
     __shared__ __align__(16) float sc_s[DW_CH], sf_s[DW_CH];
     griddep_wait();                        // PDL: the previous kernel's writes are visible
