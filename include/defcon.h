@@ -14,7 +14,8 @@
  *  - Every tensor pointer is a DEVICE pointer owned by the caller unless the
  *    parameter name ends in _host (pinned host memory, also caller-owned).
  *    The library never allocates on the call path; its only owned resources are
- *    texture plans (defcon_tex_plan_create / _destroy).
+ *    texture plans (defcon_tex_plan_create / _destroy) and the two streams the host
+ *    entry point pipelines on (created once, see defcon_layer_forward_host).
  *  - Tensors are dense, row-major, channel-last (NHWC), with the layouts given per
  *    argument.  Every tensor pointer must be 16-byte aligned (DEFCON_ERR_MISALIGNED).
  *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
@@ -181,11 +182,18 @@ int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, in
 
 /*
  * Whole layer with HOST buffers (the end-to-end entry point): copies x_host (pinned)
- * to the device, runs step 1 and step 2 on `stream`, copies y back to y_host and
- * synchronises `stream` before returning.  Parameters dw_* / pw_* / weight / bias are
- * device pointers (resident model weights), as in the two calls above.
+ * to the device, runs step 1 and step 2, copies y back to y_host and synchronises
+ * `stream` before returning.  Parameters dw_* / pw_* / weight / bias are device
+ * pointers (resident model weights), as in the two calls above.  Images are independent
+ * (P:58 is per output pixel), so the batch is cut into min(N, 2) image ranges
+ * (DEFCON_HOST_CHUNKS overrides) that flow H2D -> step 1 -> step 2 -> D2H on two
+ * internal streams ordered after the caller's prior work on `stream`: the copies of
+ * one range overlap the kernels of the other.  The internal streams / events are
+ * created once per process on first use; concurrent calls are serialised.
  * dev_workspace must hold defcon_layer_workspace_size() bytes (x, offsets, mask, y and
- * the step-2 workspace are carved out of it).  modulated != 0 selects DCNv2.
+ * two step-1 / step-2 workspaces are carved out of it).  modulated != 0 selects DCNv2.
+ * Per-image results equal defcon_dcn_forward on the same images up to the fp32
+ * summation order of the stream-K partition, which depends on the batch size.
  */
 int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, int dtype,
                               const float* dw_w, const float* dw_scale, const float* dw_shift,

@@ -5,6 +5,9 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
+#include <algorithm>
+#include <cstdlib>
 
 #include "../../include/defcon.h"
 #include "common.cuh"
@@ -114,6 +117,9 @@ static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, 
 
 static size_t path_workspace(const DcnGeom& g, Path path) {
     return path == Path::TC_BF16 ? dcn_tc_bf16_workspace(g) : 0;
+}
+static size_t path_workspace_zeroed(const DcnGeom& g, Path path) {
+    return path == Path::TC_BF16 ? dcn_tc_bf16_workspace_zeroed(g) : 0;
 }
 
 }  // namespace defcon
@@ -278,8 +284,27 @@ int defcon_deform_columns(const void* x, int N, int H, int W, int Cin, const flo
 // ---------------------------------------------------------------- end-to-end host entry
 static size_t align_up(size_t v) { return (v + 255) & ~size_t(255); }
 
+// The host entry point pipelines the batch: images are independent, so the batch
+// is cut into nchunk image ranges that flow H2D -> step 1 -> step 2 -> D2H on two internal
+// streams, and the copy engines (one per direction) overlap with the kernels of the other
+// chunk.  Device workspace: x and y for the whole batch (image slices stay 16-byte aligned),
+// offsets / mask per chunk (their per-image size is not a 16-byte multiple), and one step-2
+// workspace + one offset-branch workspace per internal stream.
+constexpr int HOST_PIPE_STREAMS = 2;
+
+static int host_chunks(int N) {
+    int k = N < 2 ? N : 2;
+    if (const char* env = getenv("DEFCON_HOST_CHUNKS")) {
+        const int v = atoi(env);
+        if (v > 0) k = v < N ? v : N;
+    }
+    return k > 0 ? k : 1;
+}
+
 struct LayerCarve {
-    size_t x, off, msk, y, ws, tws, total;
+    int nchunk, per;                    // chunks, images per chunk (last may be short)
+    size_t x, y, offm, ws, tws, total;  // offm = all per-chunk offset + mask regions
+    size_t ws_zero;                     // leading step-2 workspace bytes that must start at zero
 };
 
 static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
@@ -291,13 +316,23 @@ static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
     rc = select_path(*g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
     const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
+    c->nchunk = host_chunks(N);
+    c->per = (N + c->nchunk - 1) / c->nchunk;
+    c->nchunk = (N + c->per - 1) / c->per;
+    const size_t hw = (size_t)g->Ho * g->Wo;
     c->x = align_up((size_t)N * H * W * Cin * es);
-    c->off = align_up((size_t)g->M * g->G * g->KK * 2 * sizeof(float));
-    c->msk = modulated ? align_up((size_t)g->M * g->G * g->KK * sizeof(float)) : 0;
     c->y = align_up((size_t)g->M * Cout * es);
+    c->offm = 0;
+    for (int k = 0; k < c->nchunk; ++k) {
+        const size_t nc = (size_t)std::min(c->per, N - k * c->per);
+        c->offm += align_up(nc * hw * g->G * g->KK * 2 * sizeof(float));
+        if (modulated) c->offm += align_up(nc * hw * g->G * g->KK * sizeof(float));
+    }
+    // step-2 / branch workspaces sized for the full batch cover every chunk
     c->ws = align_up(path_workspace(*g, path));
+    c->ws_zero = path_workspace_zeroed(*g, path);
     c->tws = align_up(offset_branch_workspace(g->M, Cin));
-    c->total = c->x + c->off + c->msk + c->y + c->ws + c->tws;
+    c->total = c->x + c->y + c->offm + HOST_PIPE_STREAMS * (c->ws + c->tws);
     return DEFCON_OK;
 }
 
@@ -314,6 +349,32 @@ int defcon_layer_workspace_size(int N, int H, int W, int Cin, int dtype, int Cou
     return DEFCON_OK;
 }
 
+// Two internal streams and their completion events, created once per process on first use
+// (the only resources the host entry point keeps); calls are serialised by a mutex.
+struct HostPipe {
+    int dev = -1;
+    cudaStream_t s[HOST_PIPE_STREAMS] = {};
+    cudaEvent_t start = nullptr, done[HOST_PIPE_STREAMS] = {};
+};
+static std::mutex g_pipe_mu;
+static HostPipe g_pipe;
+
+static cudaError_t host_pipe_ready() {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (g_pipe.dev == dev) return cudaSuccess;
+    HostPipe p;
+    p.dev = dev;
+    for (int i = 0; i < HOST_PIPE_STREAMS; ++i) {
+        if ((e = cudaStreamCreateWithFlags(&p.s[i], cudaStreamNonBlocking)) != cudaSuccess) return e;
+        if ((e = cudaEventCreateWithFlags(&p.done[i], cudaEventDisableTiming)) != cudaSuccess) return e;
+    }
+    if ((e = cudaEventCreateWithFlags(&p.start, cudaEventDisableTiming)) != cudaSuccess) return e;
+    g_pipe = p;   // a previous device's objects are left to process teardown
+    return cudaSuccess;
+}
+
 int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, int dtype,
                               const float* dw_w, const float* dw_scale, const float* dw_shift,
                               const float* pw_w, const float* pw_b, const void* weight,
@@ -328,32 +389,63 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
     if (rc) return rc;
     if (dev_workspace_bytes < c.total)
         return fail(DEFCON_ERR_LIMIT, "device workspace %zu < required %zu", dev_workspace_bytes, c.total);
-    uint8_t* base = static_cast<uint8_t*>(dev_workspace);
-    void* xd = base;
-    float* offd = reinterpret_cast<float*>(base + c.x);
-    float* mskd = modulated ? reinterpret_cast<float*>(base + c.x + c.off) : nullptr;
-    void* yd = base + c.x + c.off + c.msk;
-    void* wsd = c.ws ? base + c.x + c.off + c.msk + c.y : nullptr;
-    void* twsd = base + c.x + c.off + c.msk + c.y + c.ws;
-    cudaStream_t st = static_cast<cudaStream_t>(stream);
-    const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
-    cudaError_t e = cudaMemcpyAsync(xd, x_host, (size_t)N * H * W * Cin * es, cudaMemcpyHostToDevice, st);
-    if (e != cudaSuccess) return cuda_fail(e, "H2D copy of x");
-    rc = defcon_offset_dw_conv(xd, N, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
-                               offd, mskd, twsd, c.tws, stream);
-    if (rc) return rc;
     if (out_size(H, 3, cv.stride_h, cv.pad_h, cv.dil_h) != g.Ho ||
         out_size(W, 3, cv.stride_w, cv.pad_w, cv.dil_w) != g.Wo)
         return fail(DEFCON_ERR_INVALID_ARG, "offset-branch grid differs from the DCN grid");
-    if (wsd) {   // the caller's dev_workspace carries no zero-fill guarantee: clear step 2's scratch
-        e = cudaMemsetAsync(wsd, 0, c.ws, st);
-        if (e != cudaSuccess) return cuda_fail(e, "workspace clear");
+    std::lock_guard<std::mutex> lock(g_pipe_mu);
+    cudaError_t e = host_pipe_ready();
+    if (e != cudaSuccess) return cuda_fail(e, "host pipeline streams");
+    uint8_t* base = static_cast<uint8_t*>(dev_workspace);
+    uint8_t* xd = base;
+    uint8_t* yd = base + c.x;
+    uint8_t* offm = yd + c.y;
+    uint8_t* wsbase = offm + c.offm;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
+    const size_t hw = (size_t)g.Ho * g.Wo;
+    const size_t x_img = (size_t)H * W * Cin * es, y_img = hw * Cout * es;
+    // order the pipeline after the caller's prior work on `stream`
+    if ((e = cudaEventRecord(g_pipe.start, st)) != cudaSuccess) return cuda_fail(e, "event record");
+    for (int i = 0; i < HOST_PIPE_STREAMS; ++i)
+        if ((e = cudaStreamWaitEvent(g_pipe.s[i], g_pipe.start, 0)) != cudaSuccess) return cuda_fail(e, "event wait");
+    bool cleared[HOST_PIPE_STREAMS] = {};
+    for (int k = 0; k < c.nchunk; ++k) {
+        const int si = k % HOST_PIPE_STREAMS;
+        cudaStream_t s = g_pipe.s[si];
+        const int n0 = k * c.per, nc = std::min(c.per, N - n0);
+        float* offd = reinterpret_cast<float*>(offm);
+        offm += align_up((size_t)nc * hw * g.G * g.KK * 2 * sizeof(float));
+        float* mskd = nullptr;
+        if (modulated) {
+            mskd = reinterpret_cast<float*>(offm);
+            offm += align_up((size_t)nc * hw * g.G * g.KK * sizeof(float));
+        }
+        void* wsd = c.ws ? wsbase + si * (c.ws + c.tws) : nullptr;
+        void* twsd = wsbase + si * (c.ws + c.tws) + c.ws;
+        uint8_t* xk = xd + n0 * x_img;
+        uint8_t* yk = yd + n0 * y_img;
+        e = cudaMemcpyAsync(xk, static_cast<const uint8_t*>(x_host) + n0 * x_img, nc * x_img,
+                            cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) return cuda_fail(e, "H2D copy of x");
+        rc = defcon_offset_dw_conv(xk, nc, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
+                                   offd, mskd, twsd, c.tws, s);
+        if (rc) return rc;
+        if (wsd && c.ws_zero && !cleared[si]) {   // the caller's workspace carries no zero-fill
+            cleared[si] = true;      // guarantee: clear step 2's tile counters once (self-cleaning after)
+            e = cudaMemsetAsync(wsd, 0, c.ws_zero, s);
+            if (e != cudaSuccess) return cuda_fail(e, "workspace clear");
+        }
+        rc = defcon_dcn_forward(xk, nc, H, W, Cin, offd, mskd, weight, bias, Cout, K, K, cv, dtype,
+                                sampler, fp32_mode, yk, wsd, c.ws, nullptr, s);
+        if (rc) return rc;
+        e = cudaMemcpyAsync(static_cast<uint8_t*>(y_host) + n0 * y_img, yk, nc * y_img,
+                            cudaMemcpyDeviceToHost, s);
+        if (e != cudaSuccess) return cuda_fail(e, "D2H copy of y");
     }
-    rc = defcon_dcn_forward(xd, N, H, W, Cin, offd, mskd, weight, bias, Cout, K, K, cv, dtype,
-                            sampler, fp32_mode, yd, wsd, c.ws, nullptr, stream);
-    if (rc) return rc;
-    e = cudaMemcpyAsync(y_host, yd, (size_t)g.M * Cout * es, cudaMemcpyDeviceToHost, st);
-    if (e != cudaSuccess) return cuda_fail(e, "D2H copy of y");
+    for (int i = 0; i < HOST_PIPE_STREAMS; ++i) {
+        if ((e = cudaEventRecord(g_pipe.done[i], g_pipe.s[i])) != cudaSuccess) return cuda_fail(e, "event record");
+        if ((e = cudaStreamWaitEvent(st, g_pipe.done[i], 0)) != cudaSuccess) return cuda_fail(e, "event wait");
+    }
     e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) return cuda_fail(e, "stream synchronize");
     return DEFCON_OK;

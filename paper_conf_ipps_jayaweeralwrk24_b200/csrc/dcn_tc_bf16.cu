@@ -998,6 +998,15 @@ bool dcn_tc_bf16_supported(const DcnGeom& g) {
     return true;
 }
 
+// Leading bytes of the workspace that must be zero before the first launch (the stream-K tile
+// counters; every launch leaves them zero again).  The fp32 partials need no initialisation.
+size_t dcn_tc_bf16_workspace_zeroed(const DcnGeom& g) {
+    if (g.Cout <= 64) return make_plan<64>(g).counters_bytes;
+    if (g.Cout <= 128) return make_plan<128>(g).counters_bytes;
+    if (g.Cout <= 256) return make_plan<256>(g).counters_bytes;
+    return make_plan<512>(g).counters_bytes;
+}
+
 size_t dcn_tc_bf16_workspace(const DcnGeom& g) {
     if (g.Cout <= 64) return workspace_impl<64>(g);
     if (g.Cout <= 128) return workspace_impl<128>(g);
