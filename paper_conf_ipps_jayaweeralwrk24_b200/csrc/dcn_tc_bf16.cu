@@ -24,6 +24,7 @@
 // sampling metadata (4 corner offsets, 4 mask-scaled weights) is built once per
 // (tile, offset group) into shared memory and reused by every chunk of that group.
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -74,6 +75,7 @@ struct TcArgs {
     long long total_iters; // num_tiles * ipt
     unsigned long long tex;          // DEFCON_SAMPLER_TEX: stacked-image texture object, else 0
     int bias_in_smem;      // Cout <= BIAS_SMEM_MAX: bias (or zeros) staged in shared memory
+    int pair;              // 1: CTA pairs (cta_group::2, M = 256 per MMA), tiles of 2 x BM rows
 };
 
 constexpr int BIAS_SMEM_MAX = 1024;
@@ -83,16 +85,25 @@ __host__ __device__ constexpr int bias_smem_offset(int stages, int nbuf) {
     return (((3 * stages + 2 * nbuf) * 8 + 12) + 15) & ~15;
 }
 
-template <int BLOCK_N>
+template <int BLOCK_N, bool PAIR = false>
 struct TcCfg {
     static constexpr int UMMA_N = BLOCK_N > 256 ? 256 : BLOCK_N;
     static constexpr int N_MMA = BLOCK_N / UMMA_N;
-    static constexpr int B_STAGE_BYTES = BLOCK_N * BK * 2;
+    static constexpr int B_ROWS = PAIR ? BLOCK_N / 2 : BLOCK_N;   // B rows staged by this CTA
+    static constexpr int B_STAGE_BYTES = B_ROWS * BK * 2;
     static constexpr int STAGE_BYTES = A_STAGE_BYTES + B_STAGE_BYTES;
     static constexpr int NBUF = BLOCK_N <= 256 ? 2 : 1;      // TMEM accumulator buffers
     static constexpr int TMEM_COLS = (BLOCK_N * NBUF) < 32 ? 32 : BLOCK_N * NBUF;
-    static constexpr int TMA_BOX_N = BLOCK_N > 256 ? 256 : BLOCK_N;
+    static constexpr int TMA_BOX_N = B_ROWS > 256 ? 256 : B_ROWS;
 };
+
+// First output row of `tile` for this CTA: tiles are BM rows, or 2 x BM rows split between
+// the two CTAs of a pair (rank r owns rows r*BM .. r*BM + BM - 1).
+template <bool PAIR>
+__device__ __forceinline__ int tile_m0(const TcArgs& a, int tile) {
+    if (!PAIR) return (tile / a.n_tiles_n) * BM;
+    return (tile / a.n_tiles_n) * (2 * BM) + (int)cluster_ctarank() * BM;
+}
 
 // Static stream-K partition: CTA b owns global iterations [it0(b), it0(b+1)).
 __device__ __forceinline__ long long range_begin(long long T, int G, int b) {
@@ -417,7 +428,7 @@ __device__ __forceinline__ void store_group_tma(const CUtensorMap* ymap, uint8_t
     }
 }
 
-template <int BLOCK_N, int NCOLS>
+template <int BLOCK_N, int NCOLS, bool PAIR>
 __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensorMap* ymap, const Segment& sg,
                                                  uint32_t tacc, int r, int col0, int bar_id, int nthr,
                                                  bool leader, int* fix_flag, long long T, int nct,
@@ -426,8 +437,13 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
                                                  int sid = 0) {
     constexpr int CH = 16;     // columns per partial write
     const int lane = threadIdx.x & 31;
-    const int m0 = (sg.tile / a.n_tiles_n) * BM;
+    const int m0 = tile_m0<PAIR>(a, sg.tile);
     const int n0 = (sg.tile % a.n_tiles_n) * BLOCK_N;
+    // pair mode: contributors are CTA pairs; this CTA's half of a tile has its own counter and
+    // partial slots (slot of unit b = 2b + rank, i.e. the contributing CTA's index)
+    const int rk = PAIR ? (int)cluster_ctarank() : 0;
+    const int ctr = PAIR ? 2 * sg.tile + rk : sg.tile;
+    auto slot_of = [&](int b) { return PAIR ? 2 * b + rk : b; };
     const int row = m0 + r;
     const int row0 = m0 + (r & ~31);
     const bool row_ok = row < a.M;
@@ -473,7 +489,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
         if (row_ok) {
 #pragma unroll 1
             for (int j = 0; j < nslab; ++j) {
-                const int slot = b_lo + j < b_hi ? b_lo + j : nct + b_hi;
+                const int slot = b_lo + j < b_hi ? slot_of(b_lo + j) : (int)gridDim.x + slot_of(b_hi);
                 float4 f[CS / 4];
 #pragma unroll
                 for (int u = 0; u < CS / 4; ++u)
@@ -525,7 +541,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
         for (int p0 = col0; p0 < col0 + NCOLS; p0 += pwc) {
             if (row_ok) {
                 for (int j = 0; j < nslab_fast; ++j) {
-                    const float4* src = parts + (size_t)(b_lo + j) * (slot_elems / 4) + (size_t)(p0 >> 2) * BM + r;
+                    const float4* src = parts + (size_t)slot_of(b_lo + j) * (slot_elems / 4) + (size_t)(p0 >> 2) * BM + r;
 #pragma unroll 4
                     for (int u = 0; u < pwc / 4; ++u)
                         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(
@@ -553,19 +569,19 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
     if (!owner) {                          // non-owner contributor: publish, count
         write_partial(blockIdx.x);
         named_bar_sync(bar_id, nthr);
-        if (leader) *fix_flag = (atomicAdd(a.counters + sg.tile, 1) == ncontrib) ? 1 : 0;
+        if (leader) *fix_flag = (atomicAdd(a.counters + ctr, 1) == ncontrib) ? 1 : 0;
         named_bar_sync(bar_id, nthr);
         const bool last = *fix_flag != 0;
         named_bar_sync(bar_id, nthr);      // fix_flag reused by the next segment
         if (last) {                        // owner took the slow path: finish from partials
             __threadfence();
             finish(false);
-            if (leader) a.counters[sg.tile] = 0;
+            if (leader) a.counters[ctr] = 0;
         }
         return;
     }
     // owner of a split tile
-    if (leader) *fix_flag = (ld_acquire_gpu(a.counters + sg.tile) == ncontrib) ? 1 : 0;
+    if (leader) *fix_flag = (ld_acquire_gpu(a.counters + ctr) == ncontrib) ? 1 : 0;
     named_bar_sync(bar_id, nthr);
     const bool all_in = *fix_flag != 0;
     named_bar_sync(bar_id, nthr);
@@ -575,20 +591,20 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
     if (all_in) {                          // fast path: partials + own TMEM accumulator
         if (staged) finish_staged(stage_smem);
         else finish(true);
-        if (leader) a.counters[sg.tile] = 0;
+        if (leader) a.counters[ctr] = 0;
         if (leader && stage_smem) TL(8);
         return;
     }
-    write_partial(nct + blockIdx.x);       // slow path: publish own accumulator as well
+    write_partial((int)gridDim.x + blockIdx.x);   // slow path: publish own accumulator as well
     named_bar_sync(bar_id, nthr);
-    if (leader) *fix_flag = (atomicAdd(a.counters + sg.tile, 1) == ncontrib) ? 1 : 0;
+    if (leader) *fix_flag = (atomicAdd(a.counters + ctr, 1) == ncontrib) ? 1 : 0;
     named_bar_sync(bar_id, nthr);
     const bool last = *fix_flag != 0;
     named_bar_sync(bar_id, nthr);
     if (last) {
         __threadfence();
         finish(false);
-        if (leader) a.counters[sg.tile] = 0;
+        if (leader) a.counters[ctr] = 0;
     }
 }
 
@@ -597,13 +613,13 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
 // soon as the row's registers are free (rolling prefetch).  Warps with TEXW use the texture
 // sampler, the others LDG gathers + software lerp; the metadata table holds each row in the
 // format its warp consumes (warp of row r = (r mod 64) / 8).
-template <bool TEXW, int STAGES, int NTEX>
+template <bool TEXW, int STAGES, int NTEX, bool PAIR>
 __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
                                                 const uint32_t (&dst_lo)[ROWS], const uint32_t (&dst_hi)[ROWS],
                                                 const uint32_t (&mrow)[ROWS], uint32_t a_s, uint64_t* empty,
                                                 uint64_t* full_a, int t, int sub, int lane, int next_m0) {
     using Smp = Sampler<TEXW>;
-    const int m0 = (sg.tile / a.n_tiles_n) * BM;
+    const int m0 = tile_m0<PAIR>(a, sg.tile);
     int chunk = sg.kb / a.KK;
     int tap = sg.kb - chunk * a.KK;
     int g = (chunk * BK) / a.Cg;
@@ -641,7 +657,10 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         }
         fence_proxy_async_smem();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&full_a[s]);
+        if (lane == 0) {
+            if (PAIR) mbar_arrive_cluster(&full_a[s], 0);   // the pair's MMA issuer is rank 0
+            else mbar_arrive(&full_a[s]);
+        }
 
         if (has_next && !prefetch) {          // offset group changes: new table
             named_bar_sync(1, NPT);
@@ -658,11 +677,11 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     }
 }
 
-template <int BLOCK_N, int STAGES, int NTEX>
+template <int BLOCK_N, int STAGES, int NTEX, bool PAIR>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const __grid_constant__ CUtensorMap ymap,
                            const TcArgs a) {
-    using Cfg = TcCfg<BLOCK_N>;
+    using Cfg = TcCfg<BLOCK_N, PAIR>;
 
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -685,27 +704,33 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
     const long long T = a.total_iters;
-    const int nct = gridDim.x;
-    const long long it_begin = range_begin(T, nct, blockIdx.x);
-    const long long it_end = range_begin(T, nct, blockIdx.x + 1);
+    // stream-K units: CTAs, or CTA pairs (both CTAs of a pair walk the same range)
+    const int rank = PAIR ? (int)cluster_ctarank() : 0;
+    const int nct = PAIR ? (int)gridDim.x / 2 : (int)gridDim.x;
+    const int unit = PAIR ? (int)blockIdx.x / 2 : (int)blockIdx.x;
+    const long long it_begin = range_begin(T, nct, unit);
+    const long long it_end = range_begin(T, nct, unit + 1);
     const int nseg = count_segments(a, it_begin, it_end);
     if (threadIdx.x == 0) TL(0);
 
     if (warp == TMA_WARP && lane == 0) {
         for (int s = 0; s < STAGES; ++s) {
-            mbar_init(&full_a[s], NPW);
+            mbar_init(&full_a[s], PAIR ? 2 * NPW : NPW);   // pair: both CTAs' producers
             mbar_init(&full_b[s], 1);
             mbar_init(&empty[s], 1);
         }
         for (int b = 0; b < Cfg::NBUF; ++b) {
             mbar_init(&tmem_full[b], 1);
-            mbar_init(&tmem_empty[b], 4);
+            mbar_init(&tmem_empty[b], PAIR ? 8 : 4);       // pair: both CTAs' epilogue warps
         }
         fence_barrier_init();
         tma_prefetch_desc(&wmap);
         tma_prefetch_desc(&ymap);
     }
-    if (warp == MMA_WARP) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    if (warp == MMA_WARP) {
+        if (PAIR) tmem_alloc_pair<Cfg::TMEM_COLS>(tmem_slot);
+        else tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    }
     // Everything above overlaps the previous kernel's tail (PDL); inputs are read and
     // outputs / workspace written only after it has completed.
     griddep_wait();
@@ -714,6 +739,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int i = threadIdx.x; i < a.Cout; i += NUM_THREADS) bias_s[i] = a.bias ? __ldg(a.bias + i) : 0.f;
     tc_fence_before();
     __syncthreads();
+    if (PAIR) cluster_sync_all();      // the peer's barriers are initialised before any remote arrive
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
     if (threadIdx.x == 0) TL(1);
@@ -736,13 +762,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int o = 0; o < nseg; ++o) {
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
             const int next_m0 = o + 1 < nseg
-                ? (segment_j(a, it_begin, it_end, seg_order(o + 1, nseg)).tile / a.n_tiles_n) * BM : -1;
+                ? tile_m0<PAIR>(a, segment_j(a, it_begin, it_end, seg_order(o + 1, nseg)).tile) : -1;
             if (t == 0 && o < 4) TL(2 + 2 * o);
             if (warp < NTEX)
-                produce_segment<true, STAGES, NTEX>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
+                produce_segment<true, STAGES, NTEX, PAIR>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
                                                     t, sub, lane, next_m0);
             else
-                produce_segment<false, STAGES, NTEX>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
+                produce_segment<false, STAGES, NTEX, PAIR>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
                                                      t, sub, lane, next_m0);
             if (t == 0 && o < 4) TL(3 + 2 * o);
         }
@@ -761,7 +787,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (t == 0) TL(12);
             // idle pipeline buffers: A stages hold the per-warp store scratch, B stages the
             // staged stream-K partials
-            epilogue_segment<BLOCK_N, SLICE>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT, t == 0,
+            epilogue_segment<BLOCK_N, SLICE, PAIR>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT, t == 0,
                                              fix_flag + 1, T, nct, a.bias_in_smem ? bias_s : nullptr,
                                              sA + warp * EPI_SCRATCH_PER_WARP, sB,
                                              (size_t)STAGES * Cfg::B_STAGE_BYTES, t);
@@ -777,12 +803,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             mbar_wait(&tmem_full[buf], (uint32_t)(o / Cfg::NBUF) & 1u);
             tc_fence_after();
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
-            epilogue_segment<BLOCK_N, BLOCK_N>(a, &ymap, sg, tacc, r, 0, 2, 128, threadIdx.x == EPI_WARP0 * 32,
+            epilogue_segment<BLOCK_N, BLOCK_N, PAIR>(a, &ymap, sg, tacc, r, 0, 2, 128, threadIdx.x == EPI_WARP0 * 32,
                                                fix_flag, T, nct, a.bias_in_smem ? bias_s : nullptr,
                                                epi_scratch + (warp - EPI_WARP0) * EPI_SCRATCH_PER_WARP);
             tc_fence_before();
             __syncwarp();
-            if (lane == 0) mbar_arrive(&tmem_empty[buf]);
+            if (lane == 0) {
+                if (PAIR) mbar_arrive_cluster(&tmem_empty[buf], 0);
+                else mbar_arrive(&tmem_empty[buf]);
+            }
         }
     } else if (warp == TMA_WARP) {
         // ===================== TMA producer (weights) =====================
@@ -800,33 +829,45 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     mbar_arrive(&full_b[s]);
                     (void)n0;
 #else
-                    mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
                     const int kd = tap * a.Cin + chunk * BK;
+                    if (PAIR) {   // this CTA's half of B; both halves complete on rank 0's barrier
+                        if (rank == 0) mbar_arrive_expect_tx(&full_b[s], 2 * Cfg::B_STAGE_BYTES);
+                        tma_load_2d_pair(sB + s * Cfg::B_STAGE_BYTES, &wmap, &full_b[s], kd,
+                                         n0 + rank * Cfg::B_ROWS);
+                    } else {
+                        mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
 #pragma unroll
-                    for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h)
-                        tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + h * Cfg::TMA_BOX_N * 128, &wmap,
-                                    &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+                        for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h)
+                            tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + h * Cfg::TMA_BOX_N * 128, &wmap,
+                                        &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+                    }
 #endif
                     if (++tap == a.KK) { tap = 0; ++chunk; }
                 }
             }
         }
     } else {
-        // ===================== MMA issuer =====================
-        if (lane == 0) {
-            constexpr uint32_t idesc = make_idesc(1u /*BF16*/, BM, Cfg::UMMA_N);
+        // ===================== MMA issuer (pair: rank 0 only) =====================
+        if (lane == 0 && (!PAIR || rank == 0)) {
+            constexpr uint32_t idesc = make_idesc(1u /*BF16*/, PAIR ? 2 * BM : BM, Cfg::UMMA_N);
             int q = 0;
             for (int o = 0; o < nseg; ++o) {
                 const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
                 const int buf = o % Cfg::NBUF;
-                mbar_wait(&tmem_empty[buf], ((uint32_t)(o / Cfg::NBUF) & 1u) ^ 1u);
+                if (PAIR) mbar_wait_cluster(&tmem_empty[buf], ((uint32_t)(o / Cfg::NBUF) & 1u) ^ 1u);
+                else mbar_wait(&tmem_empty[buf], ((uint32_t)(o / Cfg::NBUF) & 1u) ^ 1u);
                 tc_fence_after();
                 const uint32_t d_base = tmem_base + (uint32_t)(buf * BLOCK_N);
                 for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                     const int s = q % STAGES;
                     const uint32_t ph = (uint32_t)(q / STAGES) & 1u;
-                    mbar_wait(&full_a[s], ph);
-                    mbar_wait(&full_b[s], ph);
+                    if (PAIR) {
+                        mbar_wait_cluster(&full_a[s], ph);
+                        mbar_wait_cluster(&full_b[s], ph);
+                    } else {
+                        mbar_wait(&full_a[s], ph);
+                        mbar_wait(&full_b[s], ph);
+                    }
                     tc_fence_after();
                     const uint32_t a_addr = smem_u32(sA + s * A_STAGE_BYTES);
                     const uint32_t b_addr = smem_u32(sB + s * Cfg::B_STAGE_BYTES);
@@ -837,13 +878,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         for (int h = 0; h < Cfg::N_MMA; ++h) {
                             const uint64_t bdesc =
                                 make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
-                            mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
-                                        (kt != sg.kb || kk != 0) ? 1u : 0u);
+                            if (PAIR)
+                                mma_bf16_ss_pair(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
+                                                 (kt != sg.kb || kk != 0) ? 1u : 0u);
+                            else
+                                mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
+                                            (kt != sg.kb || kk != 0) ? 1u : 0u);
                         }
                     }
-                    mma_commit(&empty[s]);
+                    if (PAIR) mma_commit_pair(&empty[s], 0x3);
+                    else mma_commit(&empty[s]);
                 }
-                mma_commit(&tmem_full[buf]);
+                if (PAIR) mma_commit_pair(&tmem_full[buf], 0x3);
+                else mma_commit(&tmem_full[buf]);
             }
             TL(14);
         }
@@ -852,9 +899,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     __syncwarp();
     tc_fence_before();
     __syncthreads();
+    if (PAIR) cluster_sync_all();      // no CTA leaves while its peer may still touch its smem / TMEM
     if (warp == MMA_WARP) {
         tc_fence_after();
-        tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+        if (PAIR) tmem_dealloc_pair<Cfg::TMEM_COLS>(tmem_base);
+        else tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
     }
     if (threadIdx.x == 0) TL(15);
 }
@@ -881,37 +930,84 @@ struct Plan {
     size_t partial_bytes;
 };
 
+// Pair mode (CTA pairs, cta_group::2): tiles of 2 x BM rows, stream-K over pairs.
+// Co-resident 2-CTA clusters of the pair kernel (GPCs with an odd number of usable SMs leave
+// one SM unpaired), set by the pair launcher from cudaOccupancyMaxActiveClusters.
+static int g_pair_units = 0;
+
 template <int BLOCK_N>
-Plan<BLOCK_N> make_plan(const DcnGeom& g) {
+Plan<BLOCK_N> make_plan(const DcnGeom& g, bool pair = false) {
     Plan<BLOCK_N> p;
+    const int rows = pair ? 2 * BM : BM;
     p.n_tiles_n = (g.Cout + BLOCK_N - 1) / BLOCK_N;
-    p.n_tiles = ((g.M + BM - 1) / BM) * p.n_tiles_n;
+    p.n_tiles = ((g.M + rows - 1) / rows) * p.n_tiles_n;
     p.ipt = (g.Cin / BK) * g.KK;
     p.total = (long long)p.n_tiles * p.ipt;
-    // At least 4 k-iterations per CTA; DEFCON_MAX_CTAS caps the grid (tests use it to
+    // At least 4 k-iterations per CTA (pair); DEFCON_MAX_CTAS caps the grid (tests use it to
     // force long persistent ranges and many whole tiles per CTA).
-    long long grid = std::min<long long>(num_sms(), (p.total + 3) / 4);
+    const int per = pair ? 2 : 1;
+    const int max_units = pair && g_pair_units > 0 ? g_pair_units : num_sms() / per;
+    long long units = std::min<long long>(max_units, (p.total + 3) / 4);
     if (const char* env = getenv("DEFCON_MAX_CTAS")) {
         const long long cap = atoll(env);
-        if (cap > 0) grid = std::min(grid, cap);
+        if (cap > 0) units = std::min(units, std::max<long long>(cap / per, 1));
     }
-    p.grid = (int)std::max<long long>(grid, 1);
-    p.counters_bytes = ((size_t)p.n_tiles * sizeof(int) + 255) & ~size_t(255);
+    p.grid = (int)std::max<long long>(units, 1) * per;
+    // counters: one per tile (per tile half in pair mode); sized for both modes so a workspace
+    // from defcon_dcn_workspace_size fits either
+    const size_t ctrs = std::max<size_t>((size_t)(((g.M + BM - 1) / BM) * p.n_tiles_n),
+                                         (size_t)(2 * ((g.M + 2 * BM - 1) / (2 * BM)) * p.n_tiles_n));
+    p.counters_bytes = (ctrs * sizeof(int) + 255) & ~size_t(255);
     p.partial_bytes = (size_t)2 * p.grid * BLOCK_N * BM * sizeof(float);
     return p;
 }
 
 template <int BLOCK_N>
 size_t workspace_impl(const DcnGeom& g) {
-    auto p = make_plan<BLOCK_N>(g);
-    return p.counters_bytes + p.partial_bytes;
+    auto p = make_plan<BLOCK_N>(g, false);
+    auto q = make_plan<BLOCK_N>(g, true);
+    return p.counters_bytes + std::max(p.partial_bytes, q.partial_bytes);
 }
 
-template <int BLOCK_N, int STAGES>
+#ifndef DEFCON_PAIR_DEFAULT
+#define DEFCON_PAIR_DEFAULT 0
+#endif
+// DEFCON_DCN_PAIR=0 / 1 forces the single-CTA / CTA-pair schedule of the N = 256 kernel.
+bool use_pair(const DcnGeom& g, const TexPlan* tex) {
+    if (tex || g.Cout > 256 || g.Cout <= 128) return false;
+    if (const char* env = getenv("DEFCON_DCN_PAIR")) return atoi(env) != 0;
+    return DEFCON_PAIR_DEFAULT != 0;
+}
+
+template <int BLOCK_N, int STAGES, bool PAIR = false>
 cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
                         const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
-    using Cfg = TcCfg<BLOCK_N>;
-    auto plan = make_plan<BLOCK_N>(g);
+    using Cfg = TcCfg<BLOCK_N, PAIR>;
+    if (PAIR && g_pair_units == 0) {   // how many pairs fit at once (one CTA per SM)
+        auto kp = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR>;
+        const size_t smem_q = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
+                              (size_t)BM * g.KK * META_ENTRY + bias_smem_offset(STAGES, Cfg::NBUF) +
+                              (size_t)BIAS_SMEM_MAX * 4;
+        cudaFuncSetAttribute(kp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_q);
+        cudaLaunchConfig_t qc = {};
+        qc.gridDim = dim3(num_sms());
+        qc.blockDim = dim3(NUM_THREADS);
+        qc.dynamicSmemBytes = smem_q;
+        cudaLaunchAttribute qa[1];
+        qa[0].id = cudaLaunchAttributeClusterDimension;
+        qa[0].val.clusterDim.x = 2;
+        qa[0].val.clusterDim.y = 1;
+        qa[0].val.clusterDim.z = 1;
+        qc.attrs = qa;
+        qc.numAttrs = 1;
+        int nclusters = 0;
+        if (cudaOccupancyMaxActiveClusters(&nclusters, kp, &qc) != cudaSuccess || nclusters <= 0)
+            nclusters = num_sms() / 2;
+        cudaGetLastError();
+        g_pair_units = std::min(nclusters, num_sms() / 2);
+        if (getenv("DEFCON_DEBUG")) fprintf(stderr, "defcon: %d co-resident 2-CTA clusters\n", nclusters);
+    }
+    auto plan = make_plan<BLOCK_N>(g, PAIR);
     if (ws_bytes < plan.counters_bytes + plan.partial_bytes || ws == nullptr) {
         *detail = "workspace too small for the stream-K partials";
         return cudaErrorInvalidValue;
@@ -964,20 +1060,41 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.tex = tex ? tex_plan_texture(tex) : 0ull;
 
     a.bias_in_smem = g.Cout <= BIAS_SMEM_MAX ? 1 : 0;
+    a.pair = PAIR ? 1 : 0;
     // Stream-K tile counters are NOT reset here: the workspace is zero-filled once by its
     // owner and every launch leaves it zeroed (the finisher of each split tile resets it).
     const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
                         (size_t)BM * g.KK * META_ENTRY +
                         bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0);
-    auto kern = !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0>
-                : hybrid ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW / 2>
-                         : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW>;
+    auto kern = PAIR ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR>
+                : !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false>
+                : hybrid ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW / 2, false>
+                         : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) {
         *detail = "cudaFuncSetAttribute(MaxDynamicSharedMemorySize) failed";
         return e;
     }
-    e = launch_pdl(kern, dim3(plan.grid), dim3(NUM_THREADS), smem, stream, wmap, ymap, a);
+    if (PAIR) {   // 2-CTA clusters (the pair shares one M = 256 MMA) + PDL
+        e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 0);
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(plan.grid);
+        cfg.blockDim = dim3(NUM_THREADS);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = stream;
+        cudaLaunchAttribute attr[2];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = 2;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[1].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 2;
+        e = cudaLaunchKernelEx(&cfg, kern, wmap, ymap, a);
+    } else {
+        e = launch_pdl(kern, dim3(plan.grid), dim3(NUM_THREADS), smem, stream, wmap, ymap, a);
+    }
     if (e != cudaSuccess) *detail = "dcn_fwd_bf16_tc_kernel launch failed";
     return e;
 }
@@ -1021,6 +1138,11 @@ cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, siz
 #ifndef DEFCON_STAGES_256
 #define DEFCON_STAGES_256 2
 #endif
+#ifndef DEFCON_STAGES_PAIR
+#define DEFCON_STAGES_PAIR 4
+#endif
+    if (g.Cout <= 256 && use_pair(g, tex))
+        return launch_impl<256, DEFCON_STAGES_PAIR, true>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     if (g.Cout <= 256) return launch_impl<256, DEFCON_STAGES_256>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 }

@@ -105,10 +105,14 @@ def test_dcn_special_offsets(oracle_mod, d, dev, dist, dtype):
         assert normwise(y, ref) < TOL[dtype] / (2 if dtype == "bf16" else 1)
 
 
+@pytest.mark.parametrize("pair", ["0", "1"])
 @pytest.mark.parametrize("ctas", ["1", "3", "37"])
-def test_dcn_stream_k_partitions(oracle_mod, d, dev, monkeypatch, ctas):
+def test_dcn_stream_k_partitions(oracle_mod, d, dev, monkeypatch, ctas, pair):
     """Same result for any persistent grid: 1 CTA (every tile whole, TMEM double buffer
-    cycles many times), 3 and 37 CTAs (tiles split across CTAs, stream-K fixup)."""
+    cycles many times), 3 and 37 CTAs (tiles split across CTAs, stream-K fixup); single CTAs
+    and CTA pairs (cta_group::2, M = 256 per MMA, DEFCON_DCN_PAIR=1: the cap is rounded to
+    whole pairs)."""
+    monkeypatch.setenv("DEFCON_DCN_PAIR", pair)
     c = small("streamk", Cout=256, Cin=64)
     L = inputs.gen_layer(c)
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
@@ -120,11 +124,13 @@ def test_dcn_stream_k_partitions(oracle_mod, d, dev, monkeypatch, ctas):
     assert np.max(np.abs(y - y_default)) <= 2e-2 * np.max(np.abs(ref))
 
 
+@pytest.mark.parametrize("pair", ["0", "1"])
 @pytest.mark.parametrize("ctas", ["3", "37", "0"])
-def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas):
+def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas, pair):
     """The workspace is zero-filled once; every launch leaves the stream-K counters at zero
     (no per-call memset), so repeated launches on one workspace -- plain and CUDA-graph
-    replayed -- give bit-identical y."""
+    replayed -- give bit-identical y (single CTAs and CTA pairs)."""
+    monkeypatch.setenv("DEFCON_DCN_PAIR", pair)
     c = small("wsclean", Cout=256, Cin=64)
     L = inputs.gen_layer(c)
     if ctas != "0":
@@ -141,7 +147,7 @@ def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas):
     fn()
     torch.cuda.synchronize()
     y0 = y.clone()
-    n_tiles = ((c.M + 127) // 128) * ((c.Cout + 255) // 256)
+    n_tiles = ((c.M + 127) // 128 + 1) * ((c.Cout + 255) // 256)
     assert int(ws[: n_tiles * 4].count_nonzero()) == 0
     for _ in range(3):
         fn()
@@ -155,6 +161,21 @@ def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas):
     torch.cuda.synchronize()
     assert torch.equal(y, y0)
     assert int(ws[: n_tiles * 4].count_nonzero()) == 0
+
+
+@pytest.mark.parametrize("c", [configs.C4, configs.C4_G4], ids=lambda c: c.name)
+def test_dcn_pair_full_size_sampled(oracle_mod, d, dev, monkeypatch, c):
+    """The CTA-pair schedule (DEFCON_DCN_PAIR=1) at the full YOLACT++ C4 shapes, sampled
+    against the oracle, and within bf16 rounding of the single-CTA schedule."""
+    L = inputs.gen_layer(c)
+    y1 = run_dcn(d, dev, c, L)
+    monkeypatch.setenv("DEFCON_DCN_PAIR", "1")
+    y2 = run_dcn(d, dev, c, L)
+    r = np.random.default_rng(5)
+    idx = np.unique(np.concatenate([np.arange(0, 300), np.arange(c.M - 300, c.M), r.integers(0, c.M, 400)]))
+    ref = oracle_mod.dcn_pixels(L["x"], L["offset"], L["weight"], idx, L["bias"], mask=L["mask"], G=c.G)
+    assert normwise(y2.reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
+    assert np.max(np.abs(y2 - y1)) <= 2e-2 * np.max(np.abs(ref))
 
 
 def test_dcn_deterministic(d, dev):
