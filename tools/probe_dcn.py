@@ -21,7 +21,7 @@ def time_cfg(c, sampler, reps=200):
     dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
     x = torch.from_numpy(L["x"]).to(dev, dt)
     off = torch.from_numpy(L["offset"]).to(dev)
-    msk = torch.from_numpy(L["mask"]).to(dev)
+    msk = torch.from_numpy(L["mask"]).to(dev) if L["mask"] is not None else None
     w = torch.from_numpy(L["weight"]).to(dev, dt)
     b = torch.from_numpy(L["bias"]).to(dev)
     y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
