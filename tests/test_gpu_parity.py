@@ -71,8 +71,10 @@ SMALL = [
     small("bf16_tc_cout512", Cout=512, Cin=64, H=9, W=11),
     small("bf16_tc_cout48", Cout=48),               # N tile not full (TMA zero-fill)
     small("bf16_simt_cg32", Cin=64, G=2),           # Cin/G = 32: CUDA-core fallback
-    small("f32_simt_g1", dtype="f32", Cin=32, Cout=40),
-    small("f32_simt_g4_s2", dtype="f32", Cin=32, Cout=24, G=4, stride=2),
+    small("f32_simt_g1", dtype="f32", Cin=32, Cout=40),              # register-tiled fp32 kernel
+    small("f32_simt_g4_s2", dtype="f32", Cin=32, Cout=24, G=4, stride=2),   # Cg = 8: anchor kernel
+    small("f32_tiled_cout264", dtype="f32", Cin=48, Cout=264, H=11, W=9),   # 2 channel tiles, ragged M
+    small("f32_tiled_g3_dil2", dtype="f32", Cin=48, Cout=36, G=3, dil=2, pad=2),
     configs.TINY,
 ]
 
@@ -87,6 +89,18 @@ def test_dcn_small_parity(oracle_mod, d, dev, c):
     assert err < TOL[c.dtype], err
     if c.dtype == "f32":
         assert err < 1e-5
+
+
+def test_dcn_f32_anchor_matches_tiled(oracle_mod, d, dev, monkeypatch):
+    """The simple fp32 anchor kernel (DEFCON_F32_ANCHOR=1) and the register-tiled fp32 kernel
+    both reach fp32 accuracy against the oracle on the same inputs."""
+    c = small("f32_anchor", dtype="f32", Cin=32, Cout=40)
+    L = inputs.gen_layer(c)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
+    y_tiled = run_dcn(d, dev, c, L)
+    monkeypatch.setenv("DEFCON_F32_ANCHOR", "1")
+    y_anchor = run_dcn(d, dev, c, L)
+    assert normwise(y_tiled, ref) < 1e-5 and normwise(y_anchor, ref) < 1e-5
 
 
 @pytest.mark.parametrize("dist", ["zeros", "integer", "half", "far", "border", "local"])
