@@ -30,7 +30,11 @@ struct BranchArgs {
     const float* dw_shift;
     const float* pw_w;
     const float* pw_b;
-    float* t;          // workspace [M][C]
+    float* t;          // workspace [M][C] (t, or its tf32-hi plane when t_lo is set)
+    float* t_lo;       // [M][C] tf32-lo plane (t - hi) for the tcgen05 1x1, or null
+    float* w_hi;       // [OCN][C] W2 tf32-hi plane (rows >= OC zero), written by the dw kernel
+    float* w_lo;       // [OCN][C] W2 tf32-lo plane
+    int OCN;           // OC rounded up to the 1x1's MMA N
     float* offset;
     float* mask;
     int N, H, W, C, Ho, Wo, M;
@@ -90,6 +94,17 @@ __global__ void __launch_bounds__(DW_THREADS, DEFCON_DW_MINBLOCKS) dw_bn_relu_ke
         sf_s[e] = __ldg(a.dw_shift + c0 + e);
     }
     __syncthreads();
+    if (a.w_hi) {   // split W2 into tf32 hi / lo planes for the tcgen05 1x1 (grid-stride, tiny)
+        const long nw = (long)a.OCN * a.C;
+        const long nthr = (long)gridDim.x * gridDim.y * DW_THREADS;
+        for (long e = ((long)blockIdx.y * gridDim.x + blockIdx.x) * DW_THREADS + tid; e < nw; e += nthr) {
+            const int o = (int)(e / a.C);
+            const float wv = o < a.OC ? __ldg(a.pw_w + e) : 0.f;
+            const float h = __uint_as_float(__float_as_uint(wv) & 0xFFFFE000u);
+            a.w_hi[e] = h;
+            a.w_lo[e] = wv - h;
+        }
+    }
     const int v = tid & 7;                 // 8-channel vector within the 64-channel slice
     const int lane_p = tid >> 3;           // pixel lane
     if (v * 8 >= cn) return;
@@ -163,8 +178,22 @@ __global__ void __launch_bounds__(DW_THREADS, DEFCON_DW_MINBLOCKS) dw_bn_relu_ke
 #pragma unroll
         for (int u = 0; u < 8; ++u) r[u] = fmaxf(fmaf(sc_s[v * 8 + u], r[u], sf_s[v * 8 + u]), 0.f);
         float4* dst = reinterpret_cast<float4*>(a.t + (long)m * a.C + c0 + v * 8);
-        dst[0] = make_float4(r[0], r[1], r[2], r[3]);
-        dst[1] = make_float4(r[4], r[5], r[6], r[7]);
+        if (a.t_lo) {   // t = hi + lo exactly: hi = t with the low 13 mantissa bits cleared (tf32)
+            float h[8], l[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                h[u] = __uint_as_float(__float_as_uint(r[u]) & 0xFFFFE000u);
+                l[u] = r[u] - h[u];
+            }
+            float4* dlo = reinterpret_cast<float4*>(a.t_lo + (long)m * a.C + c0 + v * 8);
+            dst[0] = make_float4(h[0], h[1], h[2], h[3]);
+            dst[1] = make_float4(h[4], h[5], h[6], h[7]);
+            dlo[0] = make_float4(l[0], l[1], l[2], l[3]);
+            dlo[1] = make_float4(l[4], l[5], l[6], l[7]);
+        } else {
+            dst[0] = make_float4(r[0], r[1], r[2], r[3]);
+            dst[1] = make_float4(r[4], r[5], r[6], r[7]);
+        }
     }
 }
 
@@ -316,9 +345,159 @@ cudaError_t launch_pw(const BranchArgs& a, cudaStream_t stream) {
 }
 
 
+// ------------------------------------------------------------------ 1x1 + sigmoid on tcgen05
+// [M x C] x [C x OC] with t already split into tf32 hi / lo planes by the dw kernel, so the
+// operand tiles come straight from L2 by TMA in the canonical K-major SWIZZLE_128B layout (no
+// producer arithmetic): CTA = 128 pixels (the UMMA M), 32-channel chunks (one 128-byte row),
+// 3 MMAs per 8-channel k-step (lo*hi + hi*lo + hi*hi, kind::tf32, fp32-level accuracy), fp32
+// accumulators in TMEM.  Legacy mma.sync TF32 issues at about FFMA rate on sm_100a; tcgen05
+// does not.  Warps 0-3: W2 chunk split + staging, then the epilogue (TMEM lane quarters);
+// warp 4: TMA; warp 5: TMEM allocation + MMA issue.
+constexpr int PT_THREADS = 6 * 32;
+constexpr int PT_KC = 32;
+
+template <int OCN, int STAGES>
+__global__ void __launch_bounds__(PT_THREADS, 2)
+    pw_tc_kernel(const __grid_constant__ CUtensorMap thi, const __grid_constant__ CUtensorMap tlo,
+                 const __grid_constant__ CUtensorMap whi, const __grid_constant__ CUtensorMap wlo, const BranchArgs a) {
+    constexpr int A_BYTES = 128 * 128;               // one plane: 128 rows x 128 bytes
+    constexpr int B_BYTES = OCN * 128;
+    constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+    constexpr uint32_t TCOLS = OCN <= 32 ? 32 : OCN <= 64 ? 64 : OCN <= 128 ? 128 : 256;
+    extern __shared__ __align__(1024) uint8_t pt_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(pt_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE);
+    uint64_t* full = bars;                   // [STAGES] TMA tx (t and W2 planes)
+    uint64_t* empty = bars + STAGES;         // [STAGES] MMA commit
+    uint64_t* tmem_full = bars + 2 * STAGES;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int m0 = blockIdx.x * 128;
+    const int nch = (a.C + PT_KC - 1) / PT_KC;
+    if (tid == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        mbar_init(tmem_full, 1);
+        fence_barrier_init();
+        tma_prefetch_desc(&thi);
+        tma_prefetch_desc(&tlo);
+        tma_prefetch_desc(&whi);
+        tma_prefetch_desc(&wlo);
+    }
+    if (warp == 5) tmem_alloc<TCOLS>(tmem_slot);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    griddep_wait();                          // PDL: t and the W2 planes from the dw kernel are complete
+    const uint32_t st0 = smem_u32(smem);
+    if (warp < 4) {
+        // ---- epilogue: TMEM lane = pixel of the tile
+        mbar_wait(tmem_full, 0);
+        tc_fence_after();
+        const int row = warp * 32 + lane;
+        const int m = m0 + row;
+#pragma unroll 1
+        for (int c0 = 0; c0 < OCN; c0 += 16) {
+            uint32_t vv[16];
+            tmem_ld_32x32b_x16(tmem + ((uint32_t)(warp * 32) << 16) + c0, vv);
+            tmem_ld_wait();
+            if (m < a.M) {
+#pragma unroll
+                for (int u = 0; u < 16; ++u) {
+                    const int o = c0 + u;
+                    if (o >= a.OC) break;
+                    const float val = __uint_as_float(vv[u]) + (a.pw_b ? __ldg(a.pw_b + o) : 0.f);
+                    if (o < a.n_off)
+                        a.offset[(long)m * a.n_off + o] = val;
+                    else
+                        a.mask[(long)m * a.n_msk + (o - a.n_off)] = 1.f / (1.f + __expf(-val));
+                }
+            }
+        }
+    } else if (warp == 4) {
+        if (lane == 0) {                     // ---- TMA: t and W2 hi / lo chunks (rows past M zero)
+            for (int ch = 0; ch < nch; ++ch) {
+                const int s = ch % STAGES;
+                mbar_wait(&empty[s], ((uint32_t)(ch / STAGES) & 1u) ^ 1u);
+                mbar_arrive_expect_tx(&full[s], STAGE);
+                uint8_t* st = smem + s * STAGE;
+                tma_load_2d(st, &thi, &full[s], ch * PT_KC, m0);
+                tma_load_2d(st + A_BYTES, &tlo, &full[s], ch * PT_KC, m0);
+                tma_load_2d(st + 2 * A_BYTES, &whi, &full[s], ch * PT_KC, 0);
+                tma_load_2d(st + 2 * A_BYTES + B_BYTES, &wlo, &full[s], ch * PT_KC, 0);
+            }
+        }
+    } else if (lane == 0) {                  // ---- MMA issuer
+        constexpr uint32_t idesc = make_idesc(2u /*TF32*/, 128, OCN);
+        for (int ch = 0; ch < nch; ++ch) {
+            const int s = ch % STAGES;
+            mbar_wait(&full[s], (uint32_t)(ch / STAGES) & 1u);
+            tc_fence_after();
+            const uint32_t ah = st0 + s * STAGE, al = ah + A_BYTES, bh = al + A_BYTES, bl = bh + B_BYTES;
+#pragma unroll
+            for (int kk = 0; kk < PT_KC / 8; ++kk) {
+                const uint64_t dah = make_sw128_desc(ah + kk * 32), dal = make_sw128_desc(al + kk * 32);
+                const uint64_t dbh = make_sw128_desc(bh + kk * 32), dbl = make_sw128_desc(bl + kk * 32);
+                mma_tf32_ss(tmem, dal, dbh, idesc, (ch | kk) != 0 ? 1u : 0u);
+                mma_tf32_ss(tmem, dah, dbl, idesc, 1u);
+                mma_tf32_ss(tmem, dah, dbh, idesc, 1u);
+            }
+            mma_commit(&empty[s]);
+        }
+        mma_commit(tmem_full);
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 5) {
+        tc_fence_after();
+        tmem_dealloc<TCOLS>(tmem);
+    }
+}
+
+template <int OCN, int STAGES>
+cudaError_t launch_pw_tc(const BranchArgs& a, cudaStream_t stream) {
+    PFN_encodeTiled encode = get_encode_tiled();
+    if (!encode) return cudaErrorNotSupported;
+    CUtensorMap maps[4];
+    for (int p = 0; p < 4; ++p) {
+        const bool t = p < 2;
+        cuuint64_t dims[2] = {(cuuint64_t)a.C, (cuuint64_t)(t ? a.M : OCN)};
+        cuuint64_t strides[1] = {(cuuint64_t)a.C * 4};
+        cuuint32_t box[2] = {(cuuint32_t)PT_KC, t ? 128u : (cuuint32_t)OCN};
+        cuuint32_t estr[2] = {1, 1};
+        float* base = p == 0 ? a.t : p == 1 ? a.t_lo : p == 2 ? a.w_hi : a.w_lo;
+        CUresult cr = encode(&maps[p], CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, base, dims, strides, box, estr,
+                             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (cr != CUDA_SUCCESS) return cudaErrorInvalidValue;
+    }
+    constexpr int STAGE = 2 * 128 * 128 + 2 * OCN * 128;
+    const size_t smem = 1024 + (size_t)STAGES * STAGE + (2 * STAGES + 1) * 8 + 16;
+    auto kern = pw_tc_kernel<OCN, STAGES>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    return launch_pdl(kern, dim3((a.M + 127) / 128), dim3(PT_THREADS), smem, stream, maps[0], maps[1], maps[2],
+                      maps[3], a);
+}
+
+int pw_tc_ocn(int OC) { return OC <= 32 ? 32 : OC <= 64 ? 64 : OC <= 128 ? 128 : 256; }
+
+cudaError_t launch_pw_tc_any(const BranchArgs& a, cudaStream_t stream) {
+    // 2 stages keep two CTAs per SM for N <= 64 (the C4 grid of 154 tiles in one round)
+    if (a.OCN == 32) return launch_pw_tc<32, 2>(a, stream);
+    if (a.OCN == 64) return launch_pw_tc<64, 2>(a, stream);
+    if (a.OCN == 128) return launch_pw_tc<128, 2>(a, stream);
+    return launch_pw_tc<256, 2>(a, stream);
+}
+
 }  // namespace
 
-size_t offset_branch_workspace(int M, int C) { return (size_t)M * C * sizeof(float); }
+// t as two fp32 planes (tf32 hi / lo) for the tcgen05 1x1 (or plain t in the first plane), then
+// the W2 hi / lo planes padded to 256 rows
+size_t offset_branch_workspace(int M, int C) { return (2 * (size_t)M * C + 2 * (size_t)256 * C) * sizeof(float); }
 
 cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W, int C,
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
@@ -327,7 +506,8 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  float* offset, float* mask, float* t_ws, cudaStream_t stream) {
     BranchArgs a;
     a.x = x; a.dw_w = dw_w; a.dw_scale = dw_scale; a.dw_shift = dw_shift;
-    a.pw_w = pw_w; a.pw_b = pw_b; a.t = t_ws; a.offset = offset; a.mask = mask;
+    a.pw_w = pw_w; a.pw_b = pw_b; a.t = t_ws; a.t_lo = nullptr; a.w_hi = nullptr; a.w_lo = nullptr;
+    a.offset = offset; a.mask = mask;
     a.N = N; a.H = H; a.W = W; a.C = C; a.Ho = Ho; a.Wo = Wo; a.M = N * Ho * Wo;
     a.sh = s_h; a.sw = s_w; a.ph = p_h; a.pw = p_w; a.dh = d_h; a.dw = d_w;
     a.n_off = 2 * G * K * K;
@@ -346,10 +526,34 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
         return launch_offset_branch_fused(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
                                           a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
                                           mask, stream);
+    // 1x1 on tcgen05 from TMA-loaded hi / lo planes, or the mma.sync 3xTF32 kernel (t in one
+    // plane; DEFCON_PW_MMA=1 or DEFCON_PW_IMPL=mma forces it)
+    // The tcgen05 kernel runs one 128-pixel tile per CTA, two CTAs per SM, each CTA a latency
+    // chain over the channel chunks: it wins when its tiles fill whole rounds of CTAs, so a grid
+    // whose last round would hold a few stragglers (C3: 298 tiles for 296 slots) keeps mma.sync.
+    int sms = 148;
+    {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    const int pw_tiles = (a.M + 127) / 128, pw_slots = 2 * sms;
+    const int pw_rounds = (pw_tiles + pw_slots - 1) / pw_slots;
+    const bool pw_fill = pw_rounds == 1 || pw_tiles - (pw_rounds - 1) * pw_slots >= pw_slots / 2;
+    const char* pw_env = getenv("DEFCON_PW_IMPL");   // "mma" / "tc" force a kernel
+    const bool pw_tc = C % 4 == 0 && get_encode_tiled() != nullptr && !getenv("DEFCON_PW_MMA") &&
+                       (pw_env ? !strcmp(pw_env, "tc") : pw_fill);
+    a.OCN = pw_tc_ocn(a.OC);
+    if (pw_tc) {
+        a.t_lo = t_ws + (size_t)a.M * C;
+        a.w_hi = t_ws + 2 * (size_t)a.M * C;
+        a.w_lo = a.w_hi + (size_t)256 * C;
+    }
     dim3 g1((a.M + DW_PIX - 1) / DW_PIX, (C + DW_CH - 1) / DW_CH);
     cudaError_t e = x_bf16 ? launch_pdl(dw_bn_relu_kernel<true>, g1, dim3(DW_THREADS), 0, stream, a)
                            : launch_pdl(dw_bn_relu_kernel<false>, g1, dim3(DW_THREADS), 0, stream, a);
     if (e != cudaSuccess) return e;
+    if (pw_tc) return launch_pw_tc_any(a, stream);
     if (a.OC <= 32) return launch_pw<4>(a, stream);
     if (a.OC <= 64) return launch_pw<8>(a, stream);
     if (a.OC <= 128) return launch_pw<16>(a, stream);

@@ -249,7 +249,7 @@ def gen_branch_dev(c, dev):
     return P, {k: to_dev(v, torch.float32, dev) for k, v in P.items()}
 
 
-@pytest.mark.parametrize("path", ["row_tc", "tc", "two_pass"])
+@pytest.mark.parametrize("path", ["row_tc", "tc", "two_pass", "two_pass_pw_tc", "two_pass_pw_mma"])
 @pytest.mark.parametrize("c", [configs.C3.replace(N=2), configs.C4_G4.replace(N=2),
                                small("branch_s2_f32", dtype="f32", stride=2, Cin=48, modulated=False),
                                small("branch_d2", dil=2, pad=2, Cin=40, H=15, W=23),
@@ -258,7 +258,9 @@ def gen_branch_dev(c, dev):
 def test_offset_branch_parity(oracle_mod, d, dev, monkeypatch, c, path):
     """All three branch kernels vs the oracle: the default two-launch path ("two_pass"), the
     single-launch tcgen05 kernel ("tc") and the TMA-staged row-tile kernel ("row_tc")."""
-    monkeypatch.setenv("DEFCON_OFFSET_IMPL", path)
+    monkeypatch.setenv("DEFCON_OFFSET_IMPL", path.split("_pw_")[0])
+    if "_pw_" in path:   # the two-launch path's 1x1: tcgen05 from hi / lo planes, or mma.sync
+        monkeypatch.setenv("DEFCON_PW_IMPL", path.split("_pw_")[1])
     x = inputs.gen_x(c)
     P, Pd = gen_branch_dev(c, dev)
     off, msk = d.defcon_offset_dw_conv(to_dev(x, TDT[c.dtype], dev), Pd["dw_w"], Pd["dw_scale"],
