@@ -19,7 +19,7 @@ for r in rows:
     if hdr and len(r) == len(hdr):
         d = dict(zip(hdr, r))
         launch.append((d["Kernel Name"].split("(")[0].replace("void ", ""), float(d["Metric Value"])))
-ours = [(k, v) for k, v in launch if any(s in k for s in ("dcn_fwd", "dw_bn", "pw_sig", "tex_stage"))]
+ours = [(k, v) for k, v in launch if any(s in k for s in ("dcn_fwd", "dw_bn", "pw_", "tex_stage"))]
 tot = {}
 for k, v in ours:
     tot.setdefault(k, []).append(v)
