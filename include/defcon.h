@@ -111,7 +111,8 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
                           float* offset, float* mask, void* workspace, size_t workspace_bytes,
                           void* stream);
 
-/* Device workspace defcon_offset_dw_conv needs: the fp32 intermediate t, N*Ho*Wo*C*4 bytes. */
+/* Device workspace defcon_offset_dw_conv needs: the fp32 intermediate t as two planes (tf32 hi /
+ * lo, 2*N*Ho*Wo*C*4 bytes) and the pointwise weights likewise (2*256*C*4 bytes). */
 int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_t cv,
                                  size_t* bytes);
 

@@ -3,8 +3,10 @@ from __future__ import annotations
 
 import glob
 import os
+import shutil
 import subprocess
 import sys
+from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
@@ -34,18 +36,38 @@ def _stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile every csrc/*.cu to an object in parallel (nvcc, sm_100a), then link libdefcon.so."""
     if not force and not _stale():
         return LIB
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc, *NVCC_FLAGS, "-I", INCLUDE, "-o", tmp, *sources(), "-lcudart"]
-    r = subprocess.run(cmd, capture_output=True, text=True)
-    if verbose or r.returncode != 0:
-        sys.stderr.write(r.stdout + r.stderr)
-    if r.returncode != 0:
+    tag = f".tmp{os.getpid()}"
+    objdir = os.path.join(HERE, "build" + tag)
+    os.makedirs(objdir, exist_ok=True)
+    compile_flags = [f for f in NVCC_FLAGS if f != "-shared"]
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        cmd = [nvcc, *compile_flags, "-c", "-I", INCLUDE, "-o", obj, src]
+        return obj, subprocess.run(cmd, capture_output=True, text=True)
+
+    with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
+        results = list(ex.map(compile_one, sources()))
+    report = "".join(r.stdout + r.stderr for _, r in results)
+    failed = [r for _, r in results if r.returncode != 0]
+    if verbose or failed:
+        sys.stderr.write(report)
+    if failed:
+        shutil.rmtree(objdir, ignore_errors=True)
         raise RuntimeError("nvcc failed building libdefcon.so")
+    tmp = LIB + tag
+    link = subprocess.run([nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp,
+                           *[o for o, _ in results], "-lcudart"], capture_output=True, text=True)
+    shutil.rmtree(objdir, ignore_errors=True)
+    if link.returncode != 0:
+        sys.stderr.write(link.stdout + link.stderr)
+        raise RuntimeError("nvcc failed linking libdefcon.so")
     with open(os.path.join(HERE, "ptxas_report.txt"), "w") as f:
-        f.write(r.stderr)
+        f.write(report)
     os.replace(tmp, LIB)
     return LIB
 

@@ -100,7 +100,8 @@ def test_offset_branch_validation(lib):
     assert lib.defcon_offset_dw_conv(*bad, _conv(), V(FAKE), V(FAKE), V(FAKE), big, None) == 1
     out = ctypes.c_size_t(0)
     assert lib.defcon_offset_workspace_size(1, 8, 8, 16, 3, _conv(), ctypes.byref(out)) == 0
-    assert out.value == 8 * 8 * 16 * 4
+    # t as tf32 hi / lo planes (2 x M x C fp32) + the W2 hi / lo planes padded to 256 rows
+    assert out.value == (2 * 8 * 8 * 16 + 2 * 256 * 16) * 4
 
 
 def test_workspace_size_and_layer_size(lib):
