@@ -48,7 +48,10 @@ struct BranchArgs {
 // for all 4 pixels, so registers stay low and occupancy high.
 constexpr int DW_CH = 64;                  // channels per block (8 vectors of 8)
 constexpr int DW_LANES = 32;               // pixel lanes per block
-constexpr int DW_PPT = 4;                  // pixels per thread
+#ifndef DEFCON_DW_PPT
+#define DEFCON_DW_PPT 4
+#endif
+constexpr int DW_PPT = DEFCON_DW_PPT;      // pixels per thread
 constexpr int DW_THREADS = DW_LANES * DW_CH / 8;
 constexpr int DW_PIX = DW_LANES * DW_PPT;  // pixels per block
 
