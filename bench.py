@@ -282,9 +282,25 @@ def gpu_arm(args, rank, world, local_rank, dist):
     torch.cuda.synchronize()
     ms_e2e = a.elapsed_time(bq) / e2e_steps
 
+    # ---------------- collectives outside the timed region: per-image fp64
+    # checksums of y all-gathered (invariance: an image's y does not depend on its rank), and
+    # every rank's y gathered into rank 0, timed on its own
+    with torch.cuda.stream(stream):
+        y0 = sets[0].y
+        cks = sharding.gather_checksums(dist, sharding.image_checksums(y0))
+        barrier()
+        ga, gb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ga.record(stream)
+        yall = sharding.gather_outputs(dist, y0)
+        gb.record(stream)
+    torch.cuda.synchronize()
+    ms_gather = ga.elapsed_time(gb)
+    gather_bytes = int(yall.numel() * yall.element_size())
+    del yall
+
     # ---------------- max over ranks
-    ms_total, ms_e2e, ms_dcn, ms_branch = sharding.max_over_ranks(
-        dist, [ms_total, ms_e2e, ms_dcn, ms_branch], dev)
+    ms_total, ms_e2e, ms_dcn, ms_branch, ms_gather = sharding.max_over_ranks(
+        dist, [ms_total, ms_e2e, ms_dcn, ms_branch, ms_gather], dev)
 
     flops = configs.contraction_flops(c)
     ms_step = ms_total / args.steps
@@ -339,7 +355,13 @@ def gpu_arm(args, rank, world, local_rank, dist):
             "ms_per_step": round(ms_e2e, 4),
             "api": "defcon_layer_forward_host (C ABI, pinned host x -> y)",
         },
-        "gpu_launches": 3 * args.steps,   # dw_bn_relu + pw_sigmoid (step 1) + dcn_fwd (step 2)
+        "gpu_launches": 3 * args.steps,   # dw_bn_relu + 1x1 (step 1) + dcn_fwd (step 2)
+        "collectives": {                  # outside the timed region
+            "checksum_images": int(cks.shape[0]),
+            "y_checksum_image0": [round(float(v), 6) for v in cks[0].tolist()],
+            "y_gather_ms": round(ms_gather, 4),
+            "y_gather_bytes": gather_bytes,
+        },
     }
     return line
 

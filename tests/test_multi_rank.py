@@ -42,9 +42,13 @@ def _worker(rank, world, port, out_dir):
     gathered = [torch.empty_like(t) for _ in range(world)]
     dist.all_gather(gathered, t)
     mx = sharding.max_over_ranks(dist, [float(rank + 1), 10.0 - rank], "cpu")
+    cks = sharding.gather_checksums(dist, sharding.image_checksums(t))
+    yall = sharding.gather_outputs(dist, t)
     if rank == 0:
         np.save(os.path.join(out_dir, "sharded.npy"), torch.cat(gathered).numpy())
         np.save(os.path.join(out_dir, "max.npy"), np.array(mx))
+        np.save(os.path.join(out_dir, "cks.npy"), cks.numpy())
+        np.save(os.path.join(out_dir, "yall.npy"), yall.numpy())
     dist.barrier()
     dist.destroy_process_group()
 
@@ -58,6 +62,11 @@ def test_gloo_sharding_matches_single_process(tmp_path, oracle_mod):
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
     assert np.array_equal(sharded, ref)          # bitwise: same images, same order
     assert list(np.load(tmp_path / "max.npy")) == [2.0, 10.0]
+    # the gathered per-image checksums equal those of the single-process result (invariance),
+    # and the output gather reproduces it
+    single = sharding.image_checksums(torch.from_numpy(np.ascontiguousarray(ref))).numpy()
+    assert np.array_equal(np.load(tmp_path / "cks.npy"), single)
+    assert np.array_equal(np.load(tmp_path / "yall.npy"), ref)
 
 
 def test_shard_images():
