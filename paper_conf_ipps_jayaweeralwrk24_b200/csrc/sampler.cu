@@ -11,6 +11,8 @@
 // neighbouring threads are contiguous runs of the same NHWC pixel.  Needs (Cin/G) * ES a
 // multiple of 32 bytes (bf16 Cin/G % 16, fp32 % 8).  fp32 weights and lerp (FFMA2); bf16
 // output RNE.
+#include <cstdlib>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -140,6 +142,97 @@ __global__ void __launch_bounds__(256) deform_columns_kernel(const ColArgs a) {
     }
 }
 
+// Row-mapped variant: a (pixel, tap) row is PIECES consecutive lanes (32 / PIECES rows per warp),
+// all index math 32-bit and done once per row (each lane of the row recomputes it from the same
+// broadcast offset / mask loads -- no 64-bit divisions), two rows in flight per thread.
+// The row's (dy, dx, mask) -- loaded one iteration ahead of its use (software pipelining), so
+// a row costs one dependent memory round trip (the corner gathers), not two.
+struct RowMeta {
+    float2 d;
+    float mv;
+};
+
+template <bool BF16>
+__device__ __forceinline__ RowMeta row_meta(const ColArgs& a, int r, int piece) {
+    RowMeta q;
+    q.d = make_float2(0.f, 0.f);
+    q.mv = 0.f;
+    if (r >= a.M * a.KK) return q;
+    const int m = r / a.KK, k = r - (r / a.KK) * a.KK;
+    const int g = piece * Piece<BF16>::CPP / a.Cg;
+    const int pix = m * a.G + g;
+    q.d = __ldg(reinterpret_cast<const float2*>(a.offset) + pix * a.KK + k);
+    q.mv = a.mask ? __ldg(a.mask + pix * a.KK + k) : 1.f;
+    return q;
+}
+
+template <bool BF16, int PIECES>
+__device__ __forceinline__ void row_issue(const ColArgs& a, int r, int piece, const RowMeta& rm, Piece<BF16>& P,
+                                          long& dst_off) {
+    constexpr int CPP = Piece<BF16>::CPP, ES = Piece<BF16>::ES;
+    const int m = r / a.KK, k = r - (r / a.KK) * a.KK;
+    const int c0 = piece * CPP;
+    const int hw = a.Ho * a.Wo;
+    const int n = m / hw;
+    const int rem = m - n * hw;
+    const int ho = rem / a.Wo;
+    const int wo = rem - ho * a.Wo;
+    const int i = k / a.Kw, j = k - (k / a.Kw) * a.Kw;
+    const float2 d = rm.d;
+    const float mv = rm.mv;
+    float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
+    float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
+    py = fminf(fmaxf(py, -2.f), (float)a.H + 1.f);     // beyond one pixel out: zeros only
+    px = fminf(fmaxf(px, -2.f), (float)a.W + 1.f);
+    const uint8_t* img = reinterpret_cast<const uint8_t*>(a.x) + ((size_t)n * a.H * a.W * a.Cin + c0) * ES;
+    int off[4] = {0, 0, 0, 0};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) P.w[q] = 0.f;
+    if (py == py && px == px) {
+        const float fy = floorf(py), fx = floorf(px);
+        const float ly = py - fy, lx = px - fx;
+        const int y0 = (int)fy, x0 = (int)fx;
+        const float wq[4] = {(1.f - ly) * (1.f - lx) * mv, (1.f - ly) * lx * mv, ly * (1.f - lx) * mv, ly * lx * mv};
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int yy = y0 + (q >> 1), xx = x0 + (q & 1);
+            if (yy >= 0 && yy < a.H && xx >= 0 && xx < a.W) {   // else: weight 0, harmless in-image load
+                P.w[q] = wq[q];
+                off[q] = (yy * a.W + xx) * a.Cin;
+            }
+        }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) P.v[q] = ldg_nc_v8(img + (size_t)off[q] * ES);
+    dst_off = ((long)r * a.Cin + c0) * ES;
+}
+
+template <bool BF16, int PIECES>
+__global__ void __launch_bounds__(256) deform_columns_rows_kernel(const ColArgs a) {
+    griddep_wait();
+    griddep_launch_dependents();
+    constexpr int RPW = 32 / PIECES;                       // rows per warp per step
+    const int lane = threadIdx.x & 31;
+    const int piece = lane % PIECES, sub = lane / PIECES;
+    const int warps = gridDim.x * (blockDim.x >> 5);
+    const int gw = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int rows = a.M * a.KK;
+    const int stride = warps * RPW;
+    int r = gw * RPW + sub;
+    RowMeta q0 = row_meta<BF16>(a, r, piece), q1 = row_meta<BF16>(a, r + stride, piece);
+    for (; r < rows; r += 2 * stride) {
+        Piece<BF16> P0, P1;
+        long d0, d1 = 0;
+        row_issue<BF16, PIECES>(a, r, piece, q0, P0, d0);
+        const bool two = r + stride < rows;
+        if (two) row_issue<BF16, PIECES>(a, r + stride, piece, q1, P1, d1);
+        q0 = row_meta<BF16>(a, r + 2 * stride, piece);      // next iteration's rows
+        q1 = row_meta<BF16>(a, r + 3 * stride, piece);
+        piece_store<BF16>(a, P0, d0);
+        if (two) piece_store<BF16>(a, P1, d1);
+    }
+}
+
 }  // namespace
 
 cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* offset, const float* mask,
@@ -156,6 +249,17 @@ cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* 
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     const long long blocks = (a.total + 255) / 256;
     const int grid = (int)(blocks < (long long)nsm * 8 ? blocks : (long long)nsm * 8);
+    // row-mapped kernel when a row is 8 / 16 / 32 pieces and every index fits 32 bits
+    const bool rows32 = (long long)g.M * g.KK * g.Cin < (1ll << 31) &&
+                        (long long)g.N * g.H * g.W * g.Cin < (1ll << 31) && !getenv("DEFCON_COLUMNS_PIECEWISE");
+    if (rows32 && (a.pieces == 8 || a.pieces == 16 || a.pieces == 32)) {
+        auto pick = [&](auto kb, auto kf) { return bf16 ? kb : kf; };
+        void (*kern)(ColArgs) =
+            a.pieces == 8 ? pick(deform_columns_rows_kernel<true, 8>, deform_columns_rows_kernel<false, 8>)
+            : a.pieces == 16 ? pick(deform_columns_rows_kernel<true, 16>, deform_columns_rows_kernel<false, 16>)
+                             : pick(deform_columns_rows_kernel<true, 32>, deform_columns_rows_kernel<false, 32>);
+        return launch_pdl(kern, dim3(nsm * 2), dim3(256), 0, stream, a);   // 2 blocks per SM resident
+    }
     return bf16 ? launch_pdl(deform_columns_kernel<true>, dim3(grid), dim3(256), 0, stream, a)
                 : launch_pdl(deform_columns_kernel<false>, dim3(grid), dim3(256), 0, stream, a);
 }
