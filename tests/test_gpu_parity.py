@@ -91,6 +91,20 @@ def test_dcn_small_parity(oracle_mod, d, dev, c):
         assert err < 1e-5
 
 
+@pytest.mark.parametrize("c", [small("bf16_k1", K=1, pad=0), small("f32_k1", K=1, pad=0, dtype="f32", Cin=32),
+                               small("bf16_k5", K=5, pad=2, Cin=64, Cout=32, H=11, W=9),
+                               small("f32_k5_s2", K=5, pad=2, stride=2, dtype="f32", Cin=32, Cout=24, H=13, W=11)],
+                         ids=lambda c: c.name)
+def test_dcn_kernel_sizes(oracle_mod, d, dev, c):
+    """K = 1 (a deformable 1x1: grid_sample + 1x1, pin P7) and K = 5 (25 taps: the bf16 shapes
+    the tensor-core kernel's metadata table does not hold go to the CUDA-core path)."""
+    L = inputs.gen_layer(c)
+    y = run_dcn(d, dev, c, L)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
+                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    assert normwise(y, ref) < TOL[c.dtype] / (2 if c.dtype == "bf16" else 100)
+
+
 def test_dcn_f32_anchor_matches_tiled(oracle_mod, d, dev, monkeypatch):
     """The simple fp32 anchor kernel (DEFCON_F32_ANCHOR=1) and the register-tiled fp32 kernel
     both reach fp32 accuracy against the oracle on the same inputs."""
