@@ -402,8 +402,22 @@ def oracle_sample(c, target_s, images=4):
 def cpu_baseline(c):
     import oracle
     v, dt, sample, _ = oracle_sample(c, target_s=10.0)
-    return {"value": v, "unit": "TFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": sample, "seconds": round(dt, 2)}
+    out = {"value": v, "unit": "TFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
+           "sample": sample, "seconds": round(dt, 2)}
+    # the oracle also single-core on config 1 (the tiny DCNv1 fp32 layer)
+    t = configs.TINY
+    L = inputs.gen_layer(t)
+    ncores = oracle.num_threads()
+    oracle.set_num_threads(1)
+    try:
+        t0 = time.perf_counter()
+        oracle.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
+        t1 = time.perf_counter() - t0
+    finally:
+        oracle.set_num_threads(ncores)
+    out["tiny_1core"] = {"config": t.name, "seconds": round(t1, 4),
+                         "tflops": round(configs.contraction_flops(t) / t1 / 1e12, 6)}
+    return out
 
 
 def reference_arm(args, world):
