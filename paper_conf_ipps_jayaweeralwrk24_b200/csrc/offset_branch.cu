@@ -8,10 +8,13 @@
 //   dw_bn_relu_kernel  thread = (8 channels, 4 pixels), taps outer so each tap's weights
 //                      are read once from shared memory for 4 pixels; 16-byte loads of x
 //                      (lanes along channels, coalesced), fp32 FMA, BN + ReLU, t ->
-//                      workspace (fp32, [M][C], L2-resident between the two launches).
-//   pw_sigmoid_kernel  the 1x1 projection [M x C] x [C x OC] on the tensor cores
-//                      (mma.sync m16n8k8 TF32 with the 3xTF32 split for fp32-level
-//                      accuracy), then offsets and sigmoid(mask logits) written out.
+//                      workspace ([M][C], L2-resident between the two launches): one fp32
+//                      plane, or tf32 hi / lo planes (and W2 split likewise) for pw_tc_kernel.
+//   pw_tc_kernel       the 1x1 projection [M x C] x [C x OC] on tcgen05 (3xTF32 from the
+//                      TMA-loaded planes, TMEM accumulators) -- chosen when its tiles fill
+//                      whole rounds of CTAs;
+//   pw_sigmoid_kernel  otherwise the same projection with mma.sync m16n8k8 TF32 (3xTF32);
+//                      both then write the offsets and sigmoid(mask logits).
 // bf16 x is widened exactly; all sums are fp32.
 #include <algorithm>
 #include <cstdlib>
