@@ -345,6 +345,10 @@ def gpu_arm(args, rank, world, local_rank, dist):
             "unit": "TFLOP/s",
             "frac": round(achieved / peaks["bf16_tflops"], 4),
             "traffic": traffic,
+            # context: the measured sustained bf16 figure (cuBLAS back to back for 4 s)
+            "peak_sustained": peaks.get("bf16_tflops_sustained"),
+            "frac_sustained": (round(achieved / peaks["bf16_tflops_sustained"], 4)
+                               if peaks.get("bf16_tflops_sustained") else None),
         },
         "clocks": clocks,
         "e2e": {
