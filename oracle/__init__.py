@@ -57,6 +57,9 @@ def _load():
         lib.oracle_dcn_pixels_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, i,
                                               i, i, i, i, i, i, i, i, i,
                                               ctypes.POINTER(ctypes.c_int64), i, dp]
+        lib.oracle_dcn_pixels_texq_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, i,
+                                                   i, i, i, i, i, i, i, i, i, i,
+                                                   ctypes.POINTER(ctypes.c_int64), i, dp]
         lib.oracle_deform_columns_f64.argtypes = [dp, i, i, i, i, dp, dp, i, i, i, i, i, i, i, i, i,
                                                   ctypes.POINTER(ctypes.c_int64), ctypes.c_long, dp]
         lib.oracle_offset_branch_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, dp,
@@ -143,8 +146,10 @@ def dcn_forward(x, offset, weight, bias=None, mask=None, stride=1, pad=1, dil=1,
 
 def dcn_forward_texq(x, offset, weight, bias=None, mask=None, stride=1, pad=1, dil=1, G=1,
                      quant="round"):
-    """Texture-filter model of the layer (R14): fractions quantised to 1/256."""
-    qm = {"round": 1, "trunc": 2}[quant]
+    """Texture-filter model of the layer (R14): fractions quantised to 1/256 ("round" /
+    "trunc"), or "hw": the half4-texel filter as measured on B200 -- fractions and the four
+    bilinear weights rounded to 1/256 (ties to even), result rounded to binary16."""
+    qm = {"round": 1, "trunc": 2, "hw": 3}[quant]
     x, offset, weight, bias, mask = map(_f64, (x, offset, weight, bias, mask))
     (N, H, W, Cin, Cout, Kh, Kw, sh, sw, ph, pw, dh, dw, Ho, Wo) = _dcn_shapes(
         x, offset, weight, _pair(stride), _pair(pad), _pair(dil), G)
@@ -157,18 +162,25 @@ def dcn_forward_texq(x, offset, weight, bias=None, mask=None, stride=1, pad=1, d
     return y
 
 
-def dcn_pixels(x, offset, weight, pix_idx, bias=None, mask=None, stride=1, pad=1, dil=1, G=1):
+def dcn_pixels(x, offset, weight, pix_idx, bias=None, mask=None, stride=1, pad=1, dil=1, G=1,
+               quant=None):
     """Same definition as dcn_forward, evaluated at flattened output pixels
-    pix_idx[t] = (n*Ho + ho)*Wo + wo.  Returns [len(pix_idx), Cout] fp64."""
+    pix_idx[t] = (n*Ho + ho)*Wo + wo.  Returns [len(pix_idx), Cout] fp64.
+    quant="round"/"trunc": the texture-filter model (R14) of dcn_forward_texq instead."""
     x, offset, weight, bias, mask = map(_f64, (x, offset, weight, bias, mask))
     (N, H, W, Cin, Cout, Kh, Kw, sh, sw, ph, pw, dh, dw, Ho, Wo) = _dcn_shapes(
         x, offset, weight, _pair(stride), _pair(pad), _pair(dil), G)
     idx = np.ascontiguousarray(np.asarray(pix_idx, dtype=np.int64))
     out = np.empty((idx.size, Cout), np.float64)
-    rc = _load().oracle_dcn_pixels_f64(
-        _p(x), N, H, W, Cin, _p(offset), _p(mask), _p(weight), _p(bias), Cout, Kh, Kw,
-        sh, sw, ph, pw, dh, dw, G, idx.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
-        int(idx.size), _p(out))
+    ip = idx.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+    if quant is None:
+        rc = _load().oracle_dcn_pixels_f64(
+            _p(x), N, H, W, Cin, _p(offset), _p(mask), _p(weight), _p(bias), Cout, Kh, Kw,
+            sh, sw, ph, pw, dh, dw, G, ip, int(idx.size), _p(out))
+    else:
+        rc = _load().oracle_dcn_pixels_texq_f64(
+            _p(x), N, H, W, Cin, _p(offset), _p(mask), _p(weight), _p(bias), Cout, Kh, Kw,
+            sh, sw, ph, pw, dh, dw, G, {"round": 1, "trunc": 2, "hw": 3}[quant], ip, int(idx.size), _p(out))
     if rc:
         raise ValueError(f"oracle_dcn_pixels_f64 rc={rc}")
     return out

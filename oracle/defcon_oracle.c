@@ -96,18 +96,32 @@ double oracle_bilinear_f64(const double *plane, int H, int W, long pix_stride,
 
 /* Texture-unit model (R14, CUDA programming guide "linear filtering"):
  * the fractional part is held in 9-bit fixed point with 8 fractional bits.
- * quant_mode: 1 = round to nearest 1/256, 2 = truncate to 1/256. */
+ * quant_mode: 1 = round to nearest 1/256, 2 = truncate to 1/256, 3 = the measured half4 filter
+ * (bilinear_texq below). */
 static double quant_frac(double f, int quant_mode) {
     if (quant_mode == 1) return floor(f * 256.0 + 0.5) / 256.0;
     if (quant_mode == 2) return floor(f * 256.0) / 256.0;
     return f;
 }
 
+/* Round to the nearest binary16 value, ties to even (normal and subnormal range; the
+ * texels of the half4 texture are binary16, and so is the filter's result, R14). */
+static double round_to_f16(double v) {
+    if (v == 0.0 || v != v) return v;
+    int e;
+    frexp(v, &e);                          /* |v| = m * 2^e, 0.5 <= m < 1 */
+    double q = ldexp(1.0, (e - 1 >= -14 ? e - 1 : -14) - 10);   /* 11 significant bits */
+    return rint(v / q) * q;                /* default rounding mode: to nearest, ties to even */
+}
+
+/* quant_mode 3 ("hw", the half4-texel filter as measured on B200, R14): both fractions and
+ * each of the four products (1-a)(1-b), a(1-b), (1-a)b, ab rounded to the nearest 1/256
+ * (ties to even), the weighted sum of the four binary16 texels rounded to binary16. */
 static double bilinear_texq(const double *plane, int H, int W, long pix_stride,
                             double py, double px, int quant_mode) {
     double y0 = floor(py), x0 = floor(px);
-    double ay = quant_frac(py - y0, quant_mode);
-    double ax = quant_frac(px - x0, quant_mode);
+    double ay = quant_mode == 3 ? rint((py - y0) * 256.0) / 256.0 : quant_frac(py - y0, quant_mode);
+    double ax = quant_mode == 3 ? rint((px - x0) * 256.0) / 256.0 : quant_frac(px - x0, quant_mode);
     double wy[2] = {1.0 - ay, ay}, wx[2] = {1.0 - ax, ax};
     double acc = 0.0;
     for (int a = 0; a < 2; ++a) {
@@ -117,10 +131,12 @@ static double bilinear_texq(const double *plane, int H, int W, long pix_stride,
             double qx = x0 + b;
             if (qx < 0.0 || qx > (double)(W - 1)) continue;
             long idx = ((long)qy * W + (long)qx) * pix_stride;
-            acc += wy[a] * wx[b] * plane[idx];
+            double w = wy[a] * wx[b];
+            if (quant_mode == 3) w = rint(w * 256.0) / 256.0;
+            acc += w * plane[idx];
         }
     }
-    return acc;
+    return quant_mode == 3 ? round_to_f16(acc) : acc;
 }
 
 /* Output size "computed similarly to a regular convolution" (R3). */
@@ -245,7 +261,7 @@ int oracle_dcn_forward_texq_f64(const double *x, int N, int H, int W, int Cin,
                                 const double *weight, const double *bias, int Cout,
                                 int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
                                 int G, int quant_mode, double *y) {
-    if (quant_mode != 1 && quant_mode != 2) return 1;
+    if (quant_mode < 1 || quant_mode > 3) return 1;
     return dcn_grid(x, N, H, W, Cin, offset, mask, weight, bias, Cout, Kh, Kw,
                     sh, sw, ph, pw, dh, dw, G, quant_mode, y);
 }
@@ -253,11 +269,11 @@ int oracle_dcn_forward_texq_f64(const double *x, int N, int H, int W, int Cin,
 /* The same definition evaluated only at `n_pix` flattened output pixels
  * pix_idx[t] = (n*Ho + ho)*Wo + wo; y_out is [n_pix][Cout].  Lets the tests
  * check full-size GPU launches on sampled outputs. */
-int oracle_dcn_pixels_f64(const double *x, int N, int H, int W, int Cin,
-                          const double *offset, const double *mask,
-                          const double *weight, const double *bias, int Cout,
-                          int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
-                          int G, const int64_t *pix_idx, int n_pix, double *y_out) {
+static int dcn_pixels(const double *x, int N, int H, int W, int Cin,
+                      const double *offset, const double *mask,
+                      const double *weight, const double *bias, int Cout,
+                      int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
+                      int G, const int64_t *pix_idx, int n_pix, int quant_mode, double *y_out) {
     int Ho = oracle_out_size(H, Kh, sh, ph, dh);
     int Wo = oracle_out_size(W, Kw, sw, pw, dw);
     if (dcn_check(N, H, W, Cin, Cout, Kh, Kw, sh, sw, dh, dw, G, Ho, Wo)) return 1;
@@ -281,12 +297,34 @@ int oracle_dcn_pixels_f64(const double *x, int N, int H, int W, int Cin,
             int n = (int)(pix / ((long)Wo * Ho));
             dcn_one_pixel(x, H, W, Cin, offset + pix * G * KK * 2,
                           mask ? mask + pix * G * KK : NULL, weight, bias, Cout,
-                          Kh, Kw, sh, sw, ph, pw, dh, dw, G, n, ho, wo, 0,
+                          Kh, Kw, sh, sw, ph, pw, dh, dw, G, n, ho, wo, quant_mode,
                           col, y_out + (long)t * Cout);
         }
         free(col);
     }
     return fail ? 2 : 0;
+}
+
+int oracle_dcn_pixels_f64(const double *x, int N, int H, int W, int Cin,
+                          const double *offset, const double *mask,
+                          const double *weight, const double *bias, int Cout,
+                          int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
+                          int G, const int64_t *pix_idx, int n_pix, double *y_out) {
+    return dcn_pixels(x, N, H, W, Cin, offset, mask, weight, bias, Cout, Kh, Kw, sh, sw, ph, pw,
+                      dh, dw, G, pix_idx, n_pix, 0, y_out);
+}
+
+/* The texture-filter model (R14, as oracle_dcn_forward_texq_f64) at sampled output pixels,
+ * so full-size texture-sampler launches can be checked against it. */
+int oracle_dcn_pixels_texq_f64(const double *x, int N, int H, int W, int Cin,
+                               const double *offset, const double *mask,
+                               const double *weight, const double *bias, int Cout,
+                               int Kh, int Kw, int sh, int sw, int ph, int pw, int dh, int dw,
+                               int G, int quant_mode, const int64_t *pix_idx, int n_pix,
+                               double *y_out) {
+    if (quant_mode < 1 || quant_mode > 3) return 1;
+    return dcn_pixels(x, N, H, W, Cin, offset, mask, weight, bias, Cout, Kh, Kw, sh, sw, ph, pw,
+                      dh, dw, G, pix_idx, n_pix, quant_mode, y_out);
 }
 
 /*

@@ -14,6 +14,16 @@ from defcon_workloads import configs, inputs
 pytestmark = pytest.mark.gpu
 
 TOL = {"f32": 1e-4, "bf16": 2e-2}
+# Regression gates beside the contract gates: ~2x the normwise error measured on B200 (bf16
+# A-tile rounding + fp32 accumulation: 2.3-3.0e-3 over the configs here, SURVEY P12 sim 2.3e-3),
+# so a kernel change that loses precision fails long before the 2e-2 contract does.
+REG = {"f32": 1e-5, "bf16": 6e-3}
+
+
+def ulp_close(y, y_ref, scale):
+    """y and y_ref differ only in fp32 summation order before the final RNE to bf16: at most
+    one bf16 ulp (2^-7 relative) apart, plus fp32-level slack near zero."""
+    return bool(np.all(np.abs(y - y_ref) <= 2.0 ** -7 * np.abs(y_ref) + 1e-5 * scale))
 TDT = {"f32": torch.float32, "bf16": torch.bfloat16}
 
 
@@ -87,8 +97,7 @@ def test_dcn_small_parity(oracle_mod, d, dev, c):
                                  stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
     err = normwise(y, ref)
     assert err < TOL[c.dtype], err
-    if c.dtype == "f32":
-        assert err < 1e-5
+    assert err < REG[c.dtype], err
 
 
 @pytest.mark.parametrize("c", [small("bf16_k1", K=1, pad=0), small("f32_k1", K=1, pad=0, dtype="f32", Cin=32),
@@ -102,7 +111,7 @@ def test_dcn_kernel_sizes(oracle_mod, d, dev, c):
     y = run_dcn(d, dev, c, L)
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
                                  stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
-    assert normwise(y, ref) < TOL[c.dtype] / (2 if c.dtype == "bf16" else 100)
+    assert normwise(y, ref) < REG[c.dtype]
 
 
 def test_dcn_f32_anchor_matches_tiled(oracle_mod, d, dev, monkeypatch):
@@ -130,7 +139,7 @@ def test_dcn_special_offsets(oracle_mod, d, dev, dist, dtype):
         b = inputs.round_to(np.broadcast_to(L["bias"], y.shape), dtype)
         assert np.array_equal(y, b)
     else:
-        assert normwise(y, ref) < TOL[dtype] / (2 if dtype == "bf16" else 1)
+        assert normwise(y, ref) < REG[dtype]
 
 
 @pytest.mark.parametrize("pair", ["0", "1"])
@@ -146,10 +155,10 @@ def test_dcn_stream_k_partitions(oracle_mod, d, dev, monkeypatch, ctas, pair):
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
     monkeypatch.setenv("DEFCON_MAX_CTAS", ctas)
     y = run_dcn(d, dev, c, L)
-    assert normwise(y, ref) < TOL["bf16"]
+    assert normwise(y, ref) < REG["bf16"]
     monkeypatch.delenv("DEFCON_MAX_CTAS")
     y_default = run_dcn(d, dev, c, L)
-    assert np.max(np.abs(y - y_default)) <= 2e-2 * np.max(np.abs(ref))
+    assert ulp_close(y, y_default, np.max(np.abs(ref)))
 
 
 @pytest.mark.parametrize("pair", ["0", "1"])
@@ -202,8 +211,8 @@ def test_dcn_pair_full_size_sampled(oracle_mod, d, dev, monkeypatch, c):
     r = np.random.default_rng(5)
     idx = np.unique(np.concatenate([np.arange(0, 300), np.arange(c.M - 300, c.M), r.integers(0, c.M, 400)]))
     ref = oracle_mod.dcn_pixels(L["x"], L["offset"], L["weight"], idx, L["bias"], mask=L["mask"], G=c.G)
-    assert normwise(y2.reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
-    assert np.max(np.abs(y2 - y1)) <= 2e-2 * np.max(np.abs(ref))
+    assert normwise(y2.reshape(c.M, c.Cout)[idx], ref) < REG["bf16"]
+    assert ulp_close(y2, y1, np.max(np.abs(ref)))
 
 
 def test_dcn_deterministic(d, dev):
@@ -229,7 +238,10 @@ def test_dcn_full_size_sampled(oracle_mod, d, dev, c):
                                     r.integers(0, c.M, 300)]))
     ref = oracle_mod.dcn_pixels(L["x"], L["offset"], L["weight"], idx, L["bias"], mask=L["mask"],
                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
-    assert normwise(y[idx], ref) < TOL[c.dtype]
+    err = normwise(y[idx], ref)
+    print(f"{c.name}: normwise error {err:.3e}")
+    assert err < TOL[c.dtype]
+    assert err < REG[c.dtype]
 
 
 STACK = [l.replace(N=2) for l in configs.stack_layers(64) if l.name in ("stack_c3b0", "stack_c4b0", "stack_c4b3",
@@ -255,7 +267,7 @@ def test_stack_layers_with_branch_sampled(oracle_mod, d, dev, c):
     r = np.random.default_rng(11)
     idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(c.M - 64, c.M), r.integers(0, c.M, 200)]))
     ref = oracle_mod.dcn_pixels(x, ro, w, idx, b, mask=rm, stride=c.stride, pad=c.pad, dil=c.dil)
-    assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
+    assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < REG["bf16"]
 
 
 def gen_branch_dev(c, dev):
@@ -323,7 +335,7 @@ def test_layer_chain_and_host_entry(oracle_mod, d, dev, monkeypatch, chunks):
     r = np.random.default_rng(3)
     idx = np.unique(np.concatenate([np.arange(200), r.integers(0, c.M, 300)]))
     ref = oracle_mod.dcn_pixels(x, ro, w, idx, b, mask=rm)
-    assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < TOL["bf16"]
+    assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < REG["bf16"]
 
 
 # ---------------------------------------------------------------- texture sampler
@@ -349,28 +361,80 @@ def test_tex_filter_fixed_point(d, dev):
     print("texture filter fraction mode:", mode)
 
 
+def rms_rel(g, r):
+    """Frobenius-normwise error ||g - r|| / ||r||: averages the per-element roundings, so it
+    separates a systematic model error from the bf16 A-tile rounding noise."""
+    g = np.asarray(g, np.float64)
+    r = np.asarray(r, np.float64)
+    return float(np.linalg.norm(g - r) / max(np.linalg.norm(r), 1e-30))
+
+
+def hybrid_rows(M):
+    """Rows the hybrid producer samples through the texture unit: warps 0..3 of 8 produce
+    rows r with (r mod 64) < 32 of every 128-row tile (tiles start at multiples of 128)."""
+    return (np.arange(M) % 64) < 32
+
+
 @pytest.mark.parametrize("c", [small("tex_c128", Cout=128), small("tex_v1", modulated=False),
                                small("tex_g2", G=2), small("tex_g2_v1", G=2, modulated=False),
                                configs.C5.replace(N=2), small("tex_s2", stride=2, H=23, W=21)],
                          ids=lambda c: c.name)
 @pytest.mark.parametrize("sampler", ["tex", "hybrid"])
 def test_tex_sampler_parity(oracle_mod, d, dev, c, sampler):
-    """TEX sampler: equals the texture-model oracle (fp16 texels, 1/256 fractions,
-    measured rounding) to bf16 precision, and the exact oracle within the 5e-3 gate."""
+    """TEX sampler against the texture-model oracle (R14 as measured on B200:
+    fp16 texels, fractions and bilinear weights rounded to 1/256, fp16 filter result; for the
+    hybrid producer on its texture rows only): as accurate as the LDG path is against the exact
+    oracle (the bf16 A-tile rounding), closer to the model than to the exact oracle, and within
+    the 5e-3 contract gate of the exact oracle."""
     mode = tex_mode(d, dev)
+    assert mode == "round"     # the "hw" model below assumes the measured fraction rounding
     L = inputs.gen_layer(c)
     plan = d.TexPlan(c.N, c.H, c.W, c.Cin, torch.bfloat16)
-    y = run_dcn(d, dev, c, dict(L), sampler=sampler, tex_plan=plan)
+    y = run_dcn(d, dev, c, dict(L), sampler=sampler, tex_plan=plan).reshape(c.M, c.Cout)
+    y_ldg = run_dcn(d, dev, c, dict(L), sampler="ldg").reshape(c.M, c.Cout)
+    plan.close()
     x16 = inputs.round_to(L["x"], "f16")
     refq = oracle_mod.dcn_forward_texq(x16, L["offset"], L["weight"], L["bias"], mask=L["mask"],
-                                       stride=c.stride, pad=c.pad, dil=c.dil, G=c.G, quant=mode)
+                                       stride=c.stride, pad=c.pad, dil=c.dil, G=c.G, quant="hw").reshape(c.M, c.Cout)
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
-                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G).reshape(c.M, c.Cout)
+    if sampler == "hybrid":
+        refq = np.where(hybrid_rows(c.M)[:, None], refq, ref)
     e_q, e_x = normwise(y, refq), normwise(y, ref)
-    print(f"{c.name} {sampler}: vs texture model {e_q:.2e}, vs exact oracle {e_x:.2e}")
-    assert e_q < 1e-2
+    r_q, r_x, r_ldg = rms_rel(y, refq), rms_rel(y, ref), rms_rel(y_ldg, ref)
+    print(f"{c.name} {sampler}: max-normwise vs model {e_q:.2e}, vs exact {e_x:.2e}; "
+          f"rms vs model {r_q:.2e}, vs exact {r_x:.2e}, ldg vs exact {r_ldg:.2e}")
+    assert r_q < 1.15 * r_ldg     # the model leaves only the A-tile rounding (measured 1.03-1.07x)
+    assert r_q < r_x              # and explains the texture unit's quantisation
+    assert e_q < 5e-3
     assert e_x < 5e-3
+
+
+def test_tex_sampler_full_size_c5(oracle_mod, d, dev):
+    """BASELINE config 4 on the texture sampler at its full size (C5, N = 32: 32 stacked images,
+    128 layers), the launch the sampler probe times; sampled pixels vs the texture model and the
+    exact oracle, with the LDG sampler on the same inputs as the yardstick."""
+    mode = tex_mode(d, dev)
+    assert mode == "round"
+    c = configs.C5
+    L = inputs.gen_layer(c)
+    plan = d.TexPlan(c.N, c.H, c.W, c.Cin, torch.bfloat16)
+    y = run_dcn(d, dev, c, dict(L), sampler="tex", tex_plan=plan).reshape(c.M, c.Cout)
+    y_ldg = run_dcn(d, dev, c, dict(L), sampler="ldg").reshape(c.M, c.Cout)
     plan.close()
+    r = np.random.default_rng(8)
+    idx = np.unique(np.concatenate([np.arange(0, 130), np.arange(c.M - 130, c.M), r.integers(0, c.M, 200)]))
+    x16 = inputs.round_to(L["x"], "f16")
+    refq = oracle_mod.dcn_pixels(x16, L["offset"], L["weight"], idx, L["bias"], mask=L["mask"], quant="hw")
+    ref = oracle_mod.dcn_pixels(L["x"], L["offset"], L["weight"], idx, L["bias"], mask=L["mask"])
+    e_q, e_x = normwise(y[idx], refq), normwise(y[idx], ref)
+    r_q, r_x, r_ldg = rms_rel(y[idx], refq), rms_rel(y[idx], ref), rms_rel(y_ldg[idx], ref)
+    print(f"C5 N=32 tex: max-normwise vs model {e_q:.2e}, vs exact {e_x:.2e}; "
+          f"rms vs model {r_q:.2e}, vs exact {r_x:.2e}, ldg vs exact {r_ldg:.2e}")
+    assert r_q < 1.15 * r_ldg
+    assert r_q < r_x
+    assert e_q < 5e-3
+    assert e_x < 5e-3
 
 
 # ------------------------------------------------------------------ sampling step alone
@@ -412,5 +476,5 @@ def test_unfused_columns_gemm_matches_fused(oracle_mod, d, dev):
     y1 = d.defcon_dcn_forward(xd, off, msk, w, to_dev(L["bias"], torch.float32, dev))
     torch.cuda.synchronize()
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"]).reshape(-1, c.Cout)
-    assert normwise(y2.cpu().numpy(), ref) < TOL["bf16"]
-    assert normwise(y1.float().cpu().numpy().reshape(-1, c.Cout), ref) < TOL["bf16"]
+    assert normwise(y2.cpu().numpy(), ref) < REG["bf16"]
+    assert normwise(y1.float().cpu().numpy().reshape(-1, c.Cout), ref) < REG["bf16"]

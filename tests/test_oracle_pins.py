@@ -224,9 +224,12 @@ def test_pixels_equals_grid(oracle_mod):
 
 
 # ---------------------------------------------------------------- P10: offset branch
-@pytest.mark.parametrize("G,with_mask,stride", [(1, True, 1), (4, True, 2), (2, False, 1)])
-def test_p10_offset_branch_matches_torch(oracle_mod, G, with_mask, stride):
-    r = np.random.default_rng(30 + G)
+@pytest.mark.parametrize("G,with_mask,stride,pad,dil", [
+    (1, True, 1, 1, 1), (4, True, 2, 1, 1), (2, False, 1, 1, 1),
+    # geometry other than pad = dil = 1 (R10: the branch uses the DCN's stride/pad/dil)
+    (1, True, 1, 2, 2), (1, True, 2, 0, 1), (2, True, 2, 3, 3), (1, False, 1, 0, 2)])
+def test_p10_offset_branch_matches_torch(oracle_mod, G, with_mask, stride, pad, dil):
+    r = np.random.default_rng(30 + G + 7 * pad + 13 * dil)
     N, H, W, C, K = 2, 9, 8, 6, 3
     x = r.standard_normal((N, H, W, C))
     dw = r.standard_normal((C, 3, 3))
@@ -234,8 +237,9 @@ def test_p10_offset_branch_matches_torch(oracle_mod, G, with_mask, stride):
     OC = G * K * K * (3 if with_mask else 2)
     w2, b2 = r.standard_normal((OC, C)), r.standard_normal(OC)
     off, msk = oracle_mod.offset_branch(x, dw, sc, sh, w2, b2, K=K, G=G, with_mask=with_mask,
-                                        stride=stride)
-    t = F.conv2d(nchw(x), torch.from_numpy(dw)[:, None], stride=stride, padding=1, groups=C)
+                                        stride=stride, pad=pad, dil=dil)
+    t = F.conv2d(nchw(x), torch.from_numpy(dw)[:, None], stride=stride, padding=pad, dilation=dil,
+                 groups=C)
     t = torch.relu(t * torch.from_numpy(sc)[None, :, None, None]
                    + torch.from_numpy(sh)[None, :, None, None])
     u = F.conv2d(t, torch.from_numpy(w2)[:, :, None, None], torch.from_numpy(b2))
@@ -295,6 +299,74 @@ def test_p13_texq_error_bound(oracle_mod):
         bound = 2 * da * 2 * np.max(np.abs(x)) + 1e-12
         assert np.max(np.abs(yq - ye)) <= bound
         assert np.max(np.abs(yq - ye)) > 0
+
+
+def test_p13_texq_closed_form(oracle_mod):
+    """Texture model on the 2x2 image [[1,2],[3,4]] (f = 1 + x + 2y inside, K=1, w=1): the
+    sample at (y, x) = (dy, dx) equals 1 + q(dx) + 2 q(dy), q the fraction quantised to 1/256
+    (round: nearest 1/256; trunc: floor) -- the R14 model written out by hand."""
+    x = np.array([1.0, 2.0, 3.0, 4.0]).reshape(1, 2, 2, 1)
+    w = np.ones((1, 1, 1, 1))
+    r = np.random.default_rng(62)
+    f = r.uniform(0, 1, (1, 2, 2, 1, 1, 2))
+    # every sample stays inside [0,1]^2: position (ho + dy, wo + dx) with the integer part removed
+    pos = np.stack(np.meshgrid(np.arange(2), np.arange(2), indexing="ij"), -1).reshape(1, 2, 2, 1, 1, 2)
+    off = f - pos
+    for q, fn in (("round", lambda v: np.floor(v * 256 + 0.5) / 256), ("trunc", lambda v: np.floor(v * 256) / 256)):
+        yq = oracle_mod.dcn_forward_texq(x, off, w, None, pad=0, quant=q)[..., 0]
+        expect = 1 + fn(f[..., 1]) + 2 * fn(f[..., 0])
+        np.testing.assert_allclose(yq, expect.reshape(1, 2, 2), rtol=0, atol=1e-14)
+
+
+def test_p13_texq_hw_hand_value(oracle_mod):
+    """The measured half4 filter model ("hw", R14), worked by hand with K = 1, w = 1.
+    (a) [[1,2],[3,4]] at (dy, dx) = (0.7, 0.3): a = rne(76.8)/256 = 77/256, b = rne(179.2)/256
+        = 179/256; weights*256 = rne(179*77/256 = 53.84) = 54, rne(77*77/256 = 23.16) = 23,
+        rne(179*179/256 = 125.16) = 125, rne(77*179/256) = 54;
+        value = (54*1 + 23*2 + 125*3 + 54*4)/256 = 691/256 (binary16-exact).
+    (b) [[0,0],[0,1]] at (0.21, 0.37): value = w11 = ab; a = rne(94.72) = 95, b = rne(53.76)
+        = 54 (in 1/256), w11 = rne(95*54/256 = 20.04)/256 = 20/256, while the fraction-only
+        model ("round") keeps the unrounded product 95*54/65536."""
+    w = np.ones((1, 1, 1, 1))
+    pad_ = ((0, 0), (0, 1), (0, 1), (0, 0), (0, 0), (0, 0))   # 2x2 output grid, sample (0, 0)
+    x = np.array([1.0, 2.0, 3.0, 4.0]).reshape(1, 2, 2, 1)
+    off = np.pad(np.array([0.7, 0.3]).reshape(1, 1, 1, 1, 1, 2), pad_)
+    assert oracle_mod.dcn_forward_texq(x, off, w, None, pad=0, quant="hw")[0, 0, 0, 0] == 691 / 256
+    xs = np.array([0.0, 0.0, 0.0, 1.0]).reshape(1, 2, 2, 1)
+    off = np.pad(np.array([0.21, 0.37]).reshape(1, 1, 1, 1, 1, 2), pad_)
+    assert oracle_mod.dcn_forward_texq(xs, off, w, None, pad=0, quant="hw")[0, 0, 0, 0] == 20 / 256
+    yr = oracle_mod.dcn_forward_texq(xs, off, w, None, pad=0, quant="round")[0, 0, 0, 0]
+    assert abs(yr - 95 * 54 / 65536) < 1e-15
+
+
+def test_p13_texq_hw_exact_cases_and_bound(oracle_mod):
+    """"hw" model: with fractions on the 1/16 grid every weight product is a multiple of 1/256
+    and small-integer texels keep the sum binary16-exact, so it equals the exact oracle; in
+    general it stays within fraction rounding (2 x 1/512 x 2 max|x|) + weight rounding
+    (4 x 1/512 max|x|) + binary16 rounding (2^-11 max|x|) of it (K = 1, w = 1)."""
+    r = np.random.default_rng(64)
+    x = r.integers(-8, 9, (1, 8, 8, 1)).astype(np.float64)
+    off = np.round(3 * r.standard_normal((1, 8, 8, 1, 1, 2)) * 16) / 16
+    w = np.ones((1, 1, 1, 1))
+    ye = oracle_mod.dcn_forward(x, off, w, None, pad=0)
+    yh = oracle_mod.dcn_forward_texq(x, off, w, None, pad=0, quant="hw")
+    assert np.array_equal(ye, yh)
+    x = r.standard_normal((1, 8, 8, 1))
+    off = 3 * r.standard_normal((1, 8, 8, 1, 1, 2))
+    ye = oracle_mod.dcn_forward(x, off, w, None, pad=0)
+    yh = oracle_mod.dcn_forward_texq(x, off, w, None, pad=0, quant="hw")
+    mx = np.max(np.abs(x))
+    assert np.max(np.abs(yh - ye)) <= (4 / 512 + 4 / 512 + 2.0 ** -11) * mx
+    assert np.max(np.abs(yh - ye)) > 0
+
+
+def test_p13_texq_pixels_equals_grid(oracle_mod):
+    x, w, b, off, m, Ho, Wo = rand_layer(seed=63, G=2)
+    idx = np.array([0, 3, 11, x.shape[0] * Ho * Wo - 1])
+    for q in ("round", "trunc", "hw"):
+        y = oracle_mod.dcn_forward_texq(x, off, w, b, mask=m, G=2, quant=q)
+        yp = oracle_mod.dcn_pixels(x, off, w, idx, b, mask=m, G=2, quant=q)
+        assert np.array_equal(yp, y.reshape(-1, y.shape[-1])[idx])
 
 
 # ---------------------------------------------------------------- P14: FLOP model
