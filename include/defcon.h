@@ -17,7 +17,10 @@
  *    texture plans (defcon_tex_plan_create / _destroy) and the two streams the host
  *    entry point pipelines on (created once, see defcon_layer_forward_host).
  *  - Tensors are dense, row-major, channel-last (NHWC), with the layouts given per
- *    argument.  Every tensor pointer must be 16-byte aligned (DEFCON_ERR_MISALIGNED).
+ *    argument.  Every tensor pointer must be 16-byte aligned; x on the bf16 tensor-core
+ *    path (Cin/G % 64 == 0) and x / columns of defcon_deform_columns must be 32-byte
+ *    aligned (they are read / written with 32-byte vectors).  Violations return
+ *    DEFCON_ERR_MISALIGNED before any launch.
  *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
  *    Calls are asynchronous on that stream; no host synchronisation happens,
  *    except in defcon_layer_forward_host (see there).
@@ -46,7 +49,7 @@ typedef enum {
     DEFCON_OK = 0,
     DEFCON_ERR_INVALID_ARG = 1,  /* shape / enum / pointer argument invalid        */
     DEFCON_ERR_UNSUPPORTED = 2,  /* valid, but this build has no kernel for it     */
-    DEFCON_ERR_MISALIGNED = 3,   /* a tensor pointer is not 16-byte aligned        */
+    DEFCON_ERR_MISALIGNED = 3,   /* a tensor pointer is not 16- (or 32-) byte aligned */
     DEFCON_ERR_CUDA = 4,         /* a CUDA runtime call or kernel launch failed    */
     DEFCON_ERR_LIMIT = 5         /* exceeds an index / texture / workspace limit   */
 } defcon_status_t;
@@ -59,7 +62,11 @@ typedef enum {
 typedef enum {
     DEFCON_SAMPLER_LDG = 0,  /* software bilinear: vectorised NHWC gathers, fp32 weights */
     DEFCON_SAMPLER_TEX = 1,  /* hardware bilinear: tex2DLayered, border (zero) addressing,
-                                the paper's texel-based optimisation         */
+                                the paper's texel-based optimisation.  bf16 x
+                                is staged as binary16 texels (CUDA has no bf16 texel
+                                format): |x| > 65504 becomes inf and |x| < 2^-24 flushes
+                                to 0, so x must lie in the binary16 range; the filter
+                                rounds fractions and weights to 1/256 (reading R14)    */
     DEFCON_SAMPLER_HYBRID = 2 /* half of the A-producer warps use TEX, half LDG, so the
                                 texture units and the FMA pipes work in parallel (SURVEY
                                 section 8(f) NEXT 1); needs a tex_plan like TEX         */
@@ -139,14 +146,19 @@ int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_
  *            bytes (may be NULL when that size is 0).  The tensor-core path uses it for
  *            stream-K tile counters and fp32 partial tiles.  The workspace must be
  *            ZERO-FILLED before its first use (e.g. one cudaMemset after allocation); every
- *            completed call leaves it zero-filled again, so no per-call reset is launched
- *            (graph-capture friendly).  Calls that may run concurrently need distinct
- *            workspaces.  The kernels are launched with programmatic dependent launch: their
+ *            completed call leaves its tile counters zero again, so no per-call reset is
+ *            launched (graph-capture friendly).  The counters sit at the same offset for
+ *            every shape (behind a partial-tile region of one device-wide size), so one
+ *            zero-filled workspace serves any sequence of shapes whose
+ *            defcon_dcn_workspace_size() it covers.  A call that faults or is aborted
+ *            mid-kernel can leave counters non-zero: zero-fill again after an error.  Calls
+ *            that may run concurrently need distinct workspaces.  The kernels are launched with programmatic dependent launch: their
  *            prologue may overlap the previous kernel on `stream`, never its data.
  * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G not dividing Cin, bad enums,
  *   NULL required pointers; UNSUPPORTED for (Cin/G) % 8 != 0 (bf16) or % 4 != 0 (fp32),
  *   or a Cout not multiple of 16 on the tensor-core paths; LIMIT when N*H*W*Cin >= 2^31
- *   or the workspace is too small; MISALIGNED for unaligned pointers.
+ *   or the workspace is too small; MISALIGNED for pointers not 16-byte aligned, or x not
+ *   32-byte aligned on the bf16 tensor-core path.
  */
 int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin,
                        const float* offset, const float* mask,
@@ -190,7 +202,11 @@ int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, in
  * (DEFCON_HOST_CHUNKS overrides) that flow H2D -> step 1 -> step 2 -> D2H on two
  * internal streams ordered after the caller's prior work on `stream`: the copies of
  * one range overlap the kernels of the other.  The internal streams / events are
- * created once per process on first use; concurrent calls are serialised.
+ * created once per process on first use; concurrent calls are serialised.  Only
+ * DEFCON_SAMPLER_LDG is accepted (UNSUPPORTED otherwise: the entry owns no texture plan).
+ * Every per-chunk device region is 256-byte aligned whatever the per-image sizes.  If an
+ * error occurs after the first copy was enqueued, the internal streams are synchronised
+ * before returning, so no copy touches x_host / y_host after the call returns.
  * dev_workspace must hold defcon_layer_workspace_size() bytes (x, offsets, mask, y and
  * two step-1 / step-2 workspaces are carved out of it).  modulated != 0 selects DCNv2.
  * Per-image results equal defcon_dcn_forward on the same images up to the fp32
@@ -209,11 +225,12 @@ int defcon_layer_workspace_size(int N, int H, int W, int Cin, int dtype, int Cou
                                 size_t* bytes);
 
 /*
- * Texture plan for DEFCON_SAMPLER_TEX: one 2-D layered cudaArray per image
- * (one layer per 4 channels, half4 texels for bf16 input and float4 texels for fp32;
- * H x W texels per layer) with a texture object using border (zero) addressing,
- * linear filtering and unnormalised coordinates.  One object per image keeps the
- * layer count at Cin/4 per object, inside the 2048-layer limit the paper notes.
+ * Texture plan for DEFCON_SAMPLER_TEX / HYBRID: ONE 2-D layered cudaArray
+ * (layer l = channels 4l..4l+3; half4 texels for bf16 input, float4 for fp32) holding
+ * the N images stacked along y with one zero row after each image (W x N*(H+1) texels
+ * per layer), and a texture object with border (zero) addressing, linear filtering and
+ * unnormalised coordinates.  Stacking images keeps the layer count at Cin/4, inside the
+ * 2048-layer limit the paper notes, and the texture handle warp-uniform.
  * Errors: INVALID_ARG for bad sizes, UNSUPPORTED for Cin % 4 != 0, LIMIT for
  * Cin/4 > device max layers or H, W above the layered-texture limits, CUDA on
  * allocation failure.  destroy(NULL) is a no-op returning DEFCON_OK.

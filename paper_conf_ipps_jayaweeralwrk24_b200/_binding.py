@@ -136,6 +136,22 @@ def _stream_handle(stream):
     return ctypes.c_void_p(s.cuda_stream)
 
 
+def _on(stream):
+    """Context that makes `stream` current while this module allocates outputs and scratch:
+    the workspace zero-fill is then ordered before the kernel on the same stream, and the
+    caching allocator ties the temporaries to that stream (their blocks are not reused by
+    another stream while the kernel may still run)."""
+    return torch.cuda.stream(stream) if stream is not None else _NullCtx()
+
+
+class _NullCtx:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        return False
+
+
 def defcon_offset_workspace_size(N, H, W, C, K=3, stride=1, pad=1, dil=1, offset_groups=1) -> int:
     lib = load_library()
     out = ctypes.c_size_t(0)
@@ -163,19 +179,20 @@ def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, str
     _dev_tensor(dw_shift, "dw_shift", torch.float32, (C,))
     _dev_tensor(pw_w, "pw_w", torch.float32, (OC, C))
     _dev_tensor(pw_b, "pw_b", torch.float32, (OC,), allow_none=True)
-    if offset is None:
-        offset = torch.empty((N, Ho, Wo, G, KK, 2), device=x.device, dtype=torch.float32)
+    with _on(stream):
+        if offset is None:
+            offset = torch.empty((N, Ho, Wo, G, KK, 2), device=x.device, dtype=torch.float32)
+        if with_mask and mask is None:
+            mask = torch.empty((N, Ho, Wo, G, KK), device=x.device, dtype=torch.float32)
+        if workspace is None:
+            workspace = torch.empty(defcon_offset_workspace_size(N, H, W, C, K, stride, pad, dil,
+                                                                 offset_groups),
+                                    dtype=torch.uint8, device=x.device)
     _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, KK, 2))
     if with_mask:
-        if mask is None:
-            mask = torch.empty((N, Ho, Wo, G, KK), device=x.device, dtype=torch.float32)
         _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, KK))
     else:
         mask = None
-    if workspace is None:
-        workspace = torch.empty(defcon_offset_workspace_size(N, H, W, C, K, stride, pad, dil,
-                                                             offset_groups),
-                                dtype=torch.uint8, device=x.device)
     rc = lib.defcon_offset_dw_conv(_ptr(x), N, H, W, C, _DTYPES[x.dtype], _ptr(dw_w), _ptr(dw_scale),
                                    _ptr(dw_shift), _ptr(pw_w), _ptr(pw_b), K, cv, _ptr(offset),
                                    _ptr(mask), _ptr(workspace),
@@ -215,14 +232,15 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
     _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
     _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
     _dev_tensor(bias, "bias", torch.float32, (Cout,), allow_none=True)
-    if y is None:
-        y = torch.empty((N, Ho, Wo, Cout), device=x.device, dtype=x.dtype)
+    with _on(stream):
+        if y is None:
+            y = torch.empty((N, Ho, Wo, Cout), device=x.device, dtype=x.dtype)
+        if workspace is None:
+            need = defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw, stride, pad, dil,
+                                             offset_groups, x.dtype, sampler, fp32_mode)
+            if need:   # zero before first use, on the stream the kernel runs on
+                workspace = torch.zeros(need, dtype=torch.uint8, device=x.device)
     _dev_tensor(y, "y", x.dtype, (N, Ho, Wo, Cout))
-    if workspace is None:
-        need = defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw, stride, pad, dil,
-                                         offset_groups, x.dtype, sampler, fp32_mode)
-        if need:
-            workspace = torch.zeros(need, dtype=torch.uint8, device=x.device)   # zero before first use
     ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
     plan = None if tex_plan is None else tex_plan.handle
     rc = lib.defcon_dcn_forward(_ptr(x), N, H, W, Cin, _ptr(offset), _ptr(mask), _ptr(weight),
@@ -249,7 +267,8 @@ def defcon_deform_columns(x, offset, mask, K=3, stride=1, pad=1, dil=1, offset_g
     _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
     _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
     if columns is None:
-        columns = torch.empty((N * Ho * Wo, Kh * Kw * Cin), device=x.device, dtype=x.dtype)
+        with _on(stream):
+            columns = torch.empty((N * Ho * Wo, Kh * Kw * Cin), device=x.device, dtype=x.dtype)
     _dev_tensor(columns, "columns", x.dtype, (N * Ho * Wo, Kh * Kw * Cin))
     rc = lib.defcon_deform_columns(_ptr(x), N, H, W, Cin, _ptr(offset), _ptr(mask), Kh, Kw, cv,
                                    _DTYPES[x.dtype], _ptr(columns), _stream_handle(stream))
@@ -320,7 +339,8 @@ def defcon_tex_filter_probe(px, py, out=None, stream=None):
     _dev_tensor(px, "px", torch.float32)
     _dev_tensor(py, "py", torch.float32, tuple(px.shape))
     if out is None:
-        out = torch.empty_like(px)
+        with _on(stream):
+            out = torch.empty_like(px)
     rc = lib.defcon_tex_filter_probe(_ptr(px), _ptr(py), _ptr(out), px.numel(), _stream_handle(stream))
     _check(rc, "defcon_tex_filter_probe")
     return out

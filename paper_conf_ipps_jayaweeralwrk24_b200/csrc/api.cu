@@ -30,6 +30,7 @@ static int cuda_fail(cudaError_t e, const char* what) {
 }
 
 static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+static bool aligned32(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 31u) == 0; }
 
 static int out_size(int in, int k, int stride, int pad, int dil) {
     const long span = (long)in + 2L * pad - (long)dil * (k - 1) - 1;
@@ -118,8 +119,11 @@ static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, 
 static size_t path_workspace(const DcnGeom& g, Path path) {
     return path == Path::TC_BF16 ? dcn_tc_bf16_workspace(g) : 0;
 }
-static size_t path_workspace_zeroed(const DcnGeom& g, Path path) {
-    return path == Path::TC_BF16 ? dcn_tc_bf16_workspace_zeroed(g) : 0;
+// The workspace byte range [*off, *off + *bytes) that must be zero before a launch.
+static void path_workspace_counters(const DcnGeom& g, Path path, size_t* off, size_t* bytes) {
+    *off = 0;
+    *bytes = 0;
+    if (path == Path::TC_BF16) dcn_tc_bf16_workspace_counters(g, off, bytes);
 }
 
 }  // namespace defcon
@@ -232,6 +236,9 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     Path path;
     rc = select_path(g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
+    // the tensor-core producers gather x with 32-byte vector loads (ld.global.nc.v8)
+    if (path == Path::TC_BF16 && !aligned32(x))
+        return fail(DEFCON_ERR_MISALIGNED, "x must be 32-byte aligned for the tensor-core path");
     TexPlan* tp = nullptr;
     if (sampler == DEFCON_SAMPLER_TEX || sampler == DEFCON_SAMPLER_HYBRID) {
         tp = reinterpret_cast<TexPlan*>(tex_plan);
@@ -270,6 +277,8 @@ int defcon_deform_columns(const void* x, int N, int H, int W, int Cin, const flo
     const void* ptrs[] = {x, offset, mask, columns};
     for (const void* p : ptrs)
         if (p && !aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "tensor pointer not 16-byte aligned");
+    if (!aligned32(x) || !aligned32(columns))   // 32-byte vector gathers and stores
+        return fail(DEFCON_ERR_MISALIGNED, "x and columns must be 32-byte aligned");
     if ((long)g.M * g.KK * Cin >= (1L << 31))
         return fail(DEFCON_ERR_LIMIT, "column matrix too large for 32-bit element indexing");
     const int vec = dtype == DEFCON_BF16 ? 16 : 8;     // 32-byte pieces within one offset group
@@ -303,9 +312,27 @@ static int host_chunks(int N) {
 
 struct LayerCarve {
     int nchunk, per;                    // chunks, images per chunk (last may be short)
-    size_t x, y, offm, ws, tws, total;  // offm = all per-chunk offset + mask regions
-    size_t ws_zero;                     // leading step-2 workspace bytes that must start at zero
+    size_t xy, ws, tws, total;          // xy = per-chunk x, y, offset and mask regions
+    size_t ctr_off, ctr_bytes;          // step-2 workspace bytes that must start at zero
 };
+
+// Per-chunk device regions of the host entry, each 256-byte aligned (so every chunk's x and y
+// meet the kernels' alignment rules whatever the per-image sizes are).
+struct ChunkCarve {
+    size_t x, y, off, msk;   // region sizes
+    size_t total() const { return x + y + off + msk; }
+};
+
+static ChunkCarve chunk_carve(const DcnGeom& g, int dtype, int Cout, int modulated, int nc) {
+    const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
+    const size_t hw = (size_t)g.Ho * g.Wo;
+    ChunkCarve c;
+    c.x = align_up((size_t)nc * g.H * g.W * g.Cin * es);
+    c.y = align_up((size_t)nc * hw * Cout * es);
+    c.off = align_up((size_t)nc * hw * g.G * g.KK * 2 * sizeof(float));
+    c.msk = modulated ? align_up((size_t)nc * hw * g.G * g.KK * sizeof(float)) : 0;
+    return c;
+}
 
 static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
                        const defcon_conv_t& cv, int modulated, int sampler, int fp32_mode,
@@ -315,24 +342,20 @@ static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
     Path path;
     rc = select_path(*g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
-    const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
+    // the host entry owns no texture plan: texture samplers are device-entry only
+    if (sampler != DEFCON_SAMPLER_LDG)
+        return fail(DEFCON_ERR_UNSUPPORTED, "the host entry point supports DEFCON_SAMPLER_LDG only");
     c->nchunk = host_chunks(N);
     c->per = (N + c->nchunk - 1) / c->nchunk;
     c->nchunk = (N + c->per - 1) / c->per;
-    const size_t hw = (size_t)g->Ho * g->Wo;
-    c->x = align_up((size_t)N * H * W * Cin * es);
-    c->y = align_up((size_t)g->M * Cout * es);
-    c->offm = 0;
-    for (int k = 0; k < c->nchunk; ++k) {
-        const size_t nc = (size_t)std::min(c->per, N - k * c->per);
-        c->offm += align_up(nc * hw * g->G * g->KK * 2 * sizeof(float));
-        if (modulated) c->offm += align_up(nc * hw * g->G * g->KK * sizeof(float));
-    }
+    c->xy = 0;
+    for (int k = 0; k < c->nchunk; ++k)
+        c->xy += chunk_carve(*g, dtype, Cout, modulated, std::min(c->per, N - k * c->per)).total();
     // step-2 / branch workspaces sized for the full batch cover every chunk
     c->ws = align_up(path_workspace(*g, path));
-    c->ws_zero = path_workspace_zeroed(*g, path);
+    path_workspace_counters(*g, path, &c->ctr_off, &c->ctr_bytes);
     c->tws = align_up(offset_branch_workspace(g->M, Cin));
-    c->total = c->x + c->y + c->offm + HOST_PIPE_STREAMS * (c->ws + c->tws);
+    c->total = c->xy + HOST_PIPE_STREAMS * (c->ws + c->tws);
     return DEFCON_OK;
 }
 
@@ -395,11 +418,8 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
     std::lock_guard<std::mutex> lock(g_pipe_mu);
     cudaError_t e = host_pipe_ready();
     if (e != cudaSuccess) return cuda_fail(e, "host pipeline streams");
-    uint8_t* base = static_cast<uint8_t*>(dev_workspace);
-    uint8_t* xd = base;
-    uint8_t* yd = base + c.x;
-    uint8_t* offm = yd + c.y;
-    uint8_t* wsbase = offm + c.offm;
+    uint8_t* cur = static_cast<uint8_t*>(dev_workspace);
+    uint8_t* wsbase = cur + c.xy;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const size_t es = dtype == DEFCON_BF16 ? 2 : 4;
     const size_t hw = (size_t)g.Ho * g.Wo;
@@ -408,46 +428,49 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
     if ((e = cudaEventRecord(g_pipe.start, st)) != cudaSuccess) return cuda_fail(e, "event record");
     for (int i = 0; i < HOST_PIPE_STREAMS; ++i)
         if ((e = cudaStreamWaitEvent(g_pipe.s[i], g_pipe.start, 0)) != cudaSuccess) return cuda_fail(e, "event wait");
+    // Any failure after the first enqueue: drain the internal streams before returning, so no
+    // copy still reads x_host / writes y_host once the caller sees the error.
+    auto bail = [&](int status) {
+        for (int i = 0; i < HOST_PIPE_STREAMS; ++i) cudaStreamSynchronize(g_pipe.s[i]);
+        return status;
+    };
     bool cleared[HOST_PIPE_STREAMS] = {};
     for (int k = 0; k < c.nchunk; ++k) {
         const int si = k % HOST_PIPE_STREAMS;
         cudaStream_t s = g_pipe.s[si];
         const int n0 = k * c.per, nc = std::min(c.per, N - n0);
-        float* offd = reinterpret_cast<float*>(offm);
-        offm += align_up((size_t)nc * hw * g.G * g.KK * 2 * sizeof(float));
-        float* mskd = nullptr;
-        if (modulated) {
-            mskd = reinterpret_cast<float*>(offm);
-            offm += align_up((size_t)nc * hw * g.G * g.KK * sizeof(float));
-        }
-        void* wsd = c.ws ? wsbase + si * (c.ws + c.tws) : nullptr;
+        const ChunkCarve cc = chunk_carve(g, dtype, Cout, modulated, nc);
+        uint8_t* xk = cur;
+        uint8_t* yk = xk + cc.x;
+        float* offd = reinterpret_cast<float*>(yk + cc.y);
+        float* mskd = modulated ? reinterpret_cast<float*>(yk + cc.y + cc.off) : nullptr;
+        cur += cc.total();
+        uint8_t* wsd = c.ws ? wsbase + si * (c.ws + c.tws) : nullptr;
         void* twsd = wsbase + si * (c.ws + c.tws) + c.ws;
-        uint8_t* xk = xd + n0 * x_img;
-        uint8_t* yk = yd + n0 * y_img;
         e = cudaMemcpyAsync(xk, static_cast<const uint8_t*>(x_host) + n0 * x_img, nc * x_img,
                             cudaMemcpyHostToDevice, s);
-        if (e != cudaSuccess) return cuda_fail(e, "H2D copy of x");
+        if (e != cudaSuccess) return bail(cuda_fail(e, "H2D copy of x"));
         rc = defcon_offset_dw_conv(xk, nc, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
                                    offd, mskd, twsd, c.tws, s);
-        if (rc) return rc;
-        if (wsd && c.ws_zero && !cleared[si]) {   // the caller's workspace carries no zero-fill
+        if (rc) return bail(rc);
+        if (wsd && c.ctr_bytes && !cleared[si]) {   // the caller's workspace carries no zero-fill
             cleared[si] = true;      // guarantee: clear step 2's tile counters once (self-cleaning after)
-            e = cudaMemsetAsync(wsd, 0, c.ws_zero, s);
-            if (e != cudaSuccess) return cuda_fail(e, "workspace clear");
+            e = cudaMemsetAsync(wsd + c.ctr_off, 0, c.ctr_bytes, s);
+            if (e != cudaSuccess) return bail(cuda_fail(e, "workspace clear"));
         }
         rc = defcon_dcn_forward(xk, nc, H, W, Cin, offd, mskd, weight, bias, Cout, K, K, cv, dtype,
                                 sampler, fp32_mode, yk, wsd, c.ws, nullptr, s);
-        if (rc) return rc;
+        if (rc) return bail(rc);
         e = cudaMemcpyAsync(static_cast<uint8_t*>(y_host) + n0 * y_img, yk, nc * y_img,
                             cudaMemcpyDeviceToHost, s);
-        if (e != cudaSuccess) return cuda_fail(e, "D2H copy of y");
+        if (e != cudaSuccess) return bail(cuda_fail(e, "D2H copy of y"));
     }
     for (int i = 0; i < HOST_PIPE_STREAMS; ++i) {
-        if ((e = cudaEventRecord(g_pipe.done[i], g_pipe.s[i])) != cudaSuccess) return cuda_fail(e, "event record");
-        if ((e = cudaStreamWaitEvent(st, g_pipe.done[i], 0)) != cudaSuccess) return cuda_fail(e, "event wait");
+        if ((e = cudaEventRecord(g_pipe.done[i], g_pipe.s[i])) != cudaSuccess) return bail(cuda_fail(e, "event record"));
+        if ((e = cudaStreamWaitEvent(st, g_pipe.done[i], 0)) != cudaSuccess) return bail(cuda_fail(e, "event wait"));
     }
     e = cudaStreamSynchronize(st);
-    if (e != cudaSuccess) return cuda_fail(e, "stream synchronize");
+    if (e != cudaSuccess) return bail(cuda_fail(e, "stream synchronize"));
     return DEFCON_OK;
 }
 

@@ -962,11 +962,19 @@ Plan<BLOCK_N> make_plan(const DcnGeom& g, bool pair = false) {
     return p;
 }
 
+// Workspace layout: [0, partials_region) fp32 partial tiles, then the stream-K tile counters.
+// The partial region has ONE size for every shape on this device (2 slots per CTA of a full
+// persistent grid at the widest tile, BLOCK_N = 512), so the counters of every shape start at
+// the same offset and no shape's partials ever land on another shape's counters: a workspace
+// zero-filled once stays valid for any sequence of shapes it is large enough for (every launch
+// leaves its counters at zero again).
+size_t partials_region() {
+    return ((size_t)2 * num_sms() * 512 * BM * sizeof(float) + 255) & ~size_t(255);
+}
+
 template <int BLOCK_N>
 size_t workspace_impl(const DcnGeom& g) {
-    auto p = make_plan<BLOCK_N>(g, false);
-    auto q = make_plan<BLOCK_N>(g, true);
-    return p.counters_bytes + std::max(p.partial_bytes, q.partial_bytes);
+    return partials_region() + make_plan<BLOCK_N>(g, false).counters_bytes;
 }
 
 #ifndef DEFCON_PAIR_DEFAULT
@@ -1008,8 +1016,9 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
         if (getenv("DEFCON_DEBUG")) fprintf(stderr, "defcon: %d co-resident 2-CTA clusters\n", nclusters);
     }
     auto plan = make_plan<BLOCK_N>(g, PAIR);
-    if (ws_bytes < plan.counters_bytes + plan.partial_bytes || ws == nullptr) {
-        *detail = "workspace too small for the stream-K partials";
+    if (ws_bytes < partials_region() + plan.counters_bytes || ws == nullptr ||
+        plan.partial_bytes > partials_region()) {
+        *detail = "workspace too small for the stream-K partials and counters";
         return cudaErrorInvalidValue;
     }
     PFN_encodeTiled encode = get_encode_tiled();
@@ -1049,8 +1058,8 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.mask = p.mask;
     a.bias = p.bias;
     a.y = static_cast<__nv_bfloat16*>(p.y);
-    a.counters = static_cast<int*>(ws);
-    a.partials = reinterpret_cast<float*>(static_cast<uint8_t*>(ws) + plan.counters_bytes);
+    a.partials = static_cast<float*>(ws);
+    a.counters = reinterpret_cast<int*>(static_cast<uint8_t*>(ws) + partials_region());
     a.H = g.H; a.W = g.W; a.Cin = g.Cin; a.Cout = g.Cout; a.Kw = g.Kw; a.Ho = g.Ho; a.Wo = g.Wo;
     a.sh = g.sh; a.sw = g.sw; a.ph = g.ph; a.pw = g.pw; a.dh = g.dh; a.dw = g.dw;
     a.G = g.G; a.Cg = g.Cg; a.M = g.M; a.KK = g.KK;
@@ -1115,13 +1124,15 @@ bool dcn_tc_bf16_supported(const DcnGeom& g) {
     return true;
 }
 
-// Leading bytes of the workspace that must be zero before the first launch (the stream-K tile
-// counters; every launch leaves them zero again).  The fp32 partials need no initialisation.
-size_t dcn_tc_bf16_workspace_zeroed(const DcnGeom& g) {
-    if (g.Cout <= 64) return make_plan<64>(g).counters_bytes;
-    if (g.Cout <= 128) return make_plan<128>(g).counters_bytes;
-    if (g.Cout <= 256) return make_plan<256>(g).counters_bytes;
-    return make_plan<512>(g).counters_bytes;
+// The workspace bytes that must be zero before the first launch: the stream-K tile counters
+// at [offset, offset + bytes) (every launch leaves them zero again).  The fp32 partials need
+// no initialisation.
+void dcn_tc_bf16_workspace_counters(const DcnGeom& g, size_t* offset, size_t* bytes) {
+    *offset = partials_region();
+    if (g.Cout <= 64) *bytes = make_plan<64>(g).counters_bytes;
+    else if (g.Cout <= 128) *bytes = make_plan<128>(g).counters_bytes;
+    else if (g.Cout <= 256) *bytes = make_plan<256>(g).counters_bytes;
+    else *bytes = make_plan<512>(g).counters_bytes;
 }
 
 size_t dcn_tc_bf16_workspace(const DcnGeom& g) {

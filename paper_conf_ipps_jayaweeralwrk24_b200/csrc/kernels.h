@@ -61,7 +61,7 @@ cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaS
 // ---- step 2, fused gather + tcgen05 implicit GEMM, bf16 (dcn_tc_bf16.cu)
 bool dcn_tc_bf16_supported(const DcnGeom& g);
 size_t dcn_tc_bf16_workspace(const DcnGeom& g);   // stream-K counters + fp32 partials
-size_t dcn_tc_bf16_workspace_zeroed(const DcnGeom& g);   // leading bytes that start at zero (counters)
+void dcn_tc_bf16_workspace_counters(const DcnGeom& g, size_t* offset, size_t* bytes);   // must start at zero
 struct TexPlan;
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
                                const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail);

@@ -67,6 +67,7 @@ def _fwd(lib, x=FAKE, N=2, H=8, W=8, Cin=64, off=FAKE, mask=FAKE, w=FAKE, b=FAKE
     (dict(dtype=7), 1), (dict(sampler=9), 1), (dict(fp32_mode=4), 1),
     (dict(x=0), 1), (dict(off=0), 1), (dict(y=0), 1),
     (dict(x=FAKE + 8), 3), (dict(mask=FAKE + 4), 3), (dict(w=FAKE + 2), 3),
+    (dict(x=FAKE + 16), 3),               # tensor-core path: x is gathered in 32-byte vectors
     (dict(cv="g16_bf16"), 2),             # Cin/G = 4, not a multiple of 8 for bf16
 ])
 def test_dcn_forward_validation(lib, kw, status):
@@ -117,6 +118,22 @@ def test_workspace_size_and_layer_size(lib):
     assert out.value >= 2 * 8 * 8 * 64 * 2 * 2 + 2 * 64 * 9 * 3 * 4
     assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(offset_groups=3), 1, 0, 1,
                                          ctypes.byref(out)) == 1
+    # the host entry owns no texture plan: TEX / HYBRID are refused before anything is enqueued
+    for sampler in (1, 2):
+        assert lib.defcon_layer_workspace_size(2, 8, 8, 64, 1, 64, 3, _conv(), 1, sampler, 1,
+                                               ctypes.byref(out)) == 2
+
+
+def test_workspace_counters_at_a_shape_independent_offset(lib):
+    """The stream-K counters follow a partial-tile region of one device-wide size, so the
+    workspace sizes of two shapes differ only by their counter bytes (one zero-filled
+    workspace serves both; include/defcon.h, defcon_dcn_forward)."""
+    a, b = ctypes.c_size_t(0), ctypes.c_size_t(0)
+    assert lib.defcon_dcn_workspace_size(1, 8, 8, 64, 256, 3, 3, _conv(), 1, 0, 1, ctypes.byref(a)) == 0
+    assert lib.defcon_dcn_workspace_size(64, 35, 35, 64, 256, 3, 3, _conv(), 1, 0, 1, ctypes.byref(b)) == 0
+    tiles_a = -(-1 * 8 * 8 // 128)
+    tiles_b = -(-64 * 35 * 35 // 128)
+    assert b.value - a.value == ((2 * (-(-tiles_b // 2)) * 4 + 255) // 256 - (2 * (-(-tiles_a // 2)) * 4 + 255) // 256) * 256
 
 
 def test_binding_rejects_host_tensors():
@@ -150,5 +167,6 @@ def test_deform_columns_validation(lib):
     assert call(x=0) == 1 and call(cols=0) == 1
     assert call(cv=_conv(offset_groups=3)) == 1          # G does not divide Cin
     assert call(cols=FAKE + 8) == 3                      # misaligned
+    assert call(cols=FAKE + 16) == 3 and call(x=FAKE + 16) == 3   # 32-byte vectors: 32-byte alignment
     assert call(cv=_conv(offset_groups=8)) == 2          # Cin/G = 8: 32-byte bf16 pieces need 16
     assert call(dtype=5) == 1

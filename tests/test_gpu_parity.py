@@ -184,8 +184,11 @@ def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas, pair):
     fn()
     torch.cuda.synchronize()
     y0 = y.clone()
-    n_tiles = ((c.M + 127) // 128 + 1) * ((c.Cout + 255) // 256)
-    assert int(ws[: n_tiles * 4].count_nonzero()) == 0
+    # the tile counters: the last bytes of the workspace, behind the partial-tile region
+    ntn = (c.Cout + 255) // 256
+    ctr_bytes = -(-max(-(-c.M // 128), 2 * -(-c.M // 256)) * ntn * 4 // 256) * 256
+    ctrs = ws[need - ctr_bytes:]
+    assert int(ctrs.count_nonzero()) == 0
     for _ in range(3):
         fn()
     s = torch.cuda.Stream()
@@ -197,7 +200,34 @@ def test_dcn_workspace_self_cleaning(d, dev, monkeypatch, ctas, pair):
     g.replay()
     torch.cuda.synchronize()
     assert torch.equal(y, y0)
-    assert int(ws[: n_tiles * 4].count_nonzero()) == 0
+    assert int(ctrs.count_nonzero()) == 0
+
+
+def test_dcn_workspace_reused_across_shapes(d, dev, monkeypatch):
+    """One workspace, zero-filled once, serves a small-M shape, then a large-M shape (more
+    tiles: a longer counter region), then the small one again: every result is bit-identical
+    to a run on a fresh workspace (the counters sit at a shape-independent offset behind the
+    partial tiles, include/defcon.h)."""
+    monkeypatch.setenv("DEFCON_MAX_CTAS", "37")    # force split tiles (partials + counters in use)
+    small_c = small("ws_small", Cout=256, Cin=64, N=1, H=9, W=11)
+    big_c = small("ws_big", Cout=256, Cin=64, N=4, H=31, W=29)
+    dt = torch.bfloat16
+    need = max(d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K, c.stride, c.pad,
+                                           c.dil, c.G, dt) for c in (small_c, big_c))
+    ws = torch.zeros(need, dtype=torch.uint8, device=dev)
+
+    def run(c, workspace):
+        L = inputs.gen_layer(c)
+        args = [to_dev(L["x"], dt, dev), to_dev(L["offset"], torch.float32, dev),
+                to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], dt, dev),
+                to_dev(L["bias"], torch.float32, dev)]
+        y = d.defcon_dcn_forward(*args, workspace=workspace)
+        torch.cuda.synchronize()
+        return y.cpu()
+
+    ref_small, ref_big = run(small_c, None), run(big_c, None)
+    for c, ref in ((small_c, ref_small), (big_c, ref_big), (small_c, ref_small), (big_c, ref_big)):
+        assert torch.equal(run(c, ws), ref), c.name
 
 
 @pytest.mark.parametrize("c", [configs.C4, configs.C4_G4], ids=lambda c: c.name)
@@ -336,6 +366,33 @@ def test_layer_chain_and_host_entry(oracle_mod, d, dev, monkeypatch, chunks):
     idx = np.unique(np.concatenate([np.arange(200), r.integers(0, c.M, 300)]))
     ref = oracle_mod.dcn_pixels(x, ro, w, idx, b, mask=rm)
     assert normwise(y.float().cpu().numpy().reshape(c.M, c.Cout)[idx], ref) < REG["bf16"]
+
+
+def test_host_entry_odd_chunk_sizes(oracle_mod, d, dev, monkeypatch):
+    """Host entry with per-image sizes that are not 16-byte multiples (fp32 CUDA-core path,
+    Cout = 20, Ho*Wo odd) over 3 chunks: each chunk's device regions are carved 256-byte
+    aligned, so every chunk runs (no MISALIGNED after chunk 0) and y equals the device path."""
+    monkeypatch.setenv("DEFCON_HOST_CHUNKS", "3")
+    c = small("host_odd", dtype="f32", Cin=16, Cout=20, N=3, H=9, W=7)
+    x = inputs.gen_x(c)
+    w, b = inputs.gen_weight(c)
+    P, Pd = gen_branch_dev(c, dev)
+    xd, wd, bd = to_dev(x, torch.float32, dev), to_dev(w, torch.float32, dev), to_dev(b, torch.float32, dev)
+    off, msk = d.defcon_offset_dw_conv(xd, Pd["dw_w"], Pd["dw_scale"], Pd["dw_shift"], Pd["pw_w"], Pd["pw_b"])
+    y = d.defcon_dcn_forward(xd, off, msk, wd, bd)
+    ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, dtype=torch.float32),
+                     dtype=torch.uint8, device=dev)
+    xh = torch.from_numpy(x).float().pin_memory()
+    yh = torch.empty(tuple(y.shape), dtype=torch.float32).pin_memory()
+    d.defcon_layer_forward_host(xh, Pd, wd, bd, yh, ws)
+    torch.cuda.synchronize()
+    assert torch.equal(yh, y.cpu())
+
+
+def test_host_entry_rejects_texture_sampler(d, dev):
+    c = small("host_tex", N=2)
+    with pytest.raises(d.DefconError):
+        d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, sampler="tex")
 
 
 # ---------------------------------------------------------------- texture sampler
