@@ -168,7 +168,11 @@ int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_
     int Ho, Wo;
     int rc = branch_geom(N, H, W, C, K, cv, &Ho, &Wo);
     if (rc) return rc;
-    *bytes = offset_branch_workspace(N * Ho * Wo, C);
+    size_t b[2];
+    for (int bf = 0; bf < 2; ++bf)   // x's dtype is not an argument here: cover both
+        b[bf] = offset_branch_workspace(N, H, W, C, Ho, Wo, K, cv.offset_groups, cv.stride_h, cv.stride_w,
+                                        cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, bf == 1);
+    *bytes = std::max(b[0], b[1]);
     return DEFCON_OK;
 }
 
@@ -192,7 +196,8 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
     if (OC > 256) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 256", OC);
     if ((long)N * Ho * Wo * OC >= (1L << 31))
         return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
-    const size_t need = offset_branch_workspace(N * Ho * Wo, C);
+    const size_t need = offset_branch_workspace(N, H, W, C, Ho, Wo, K, cv.offset_groups, cv.stride_h, cv.stride_w,
+                                                cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, x_dtype == DEFCON_BF16);
     if (!workspace || workspace_bytes < need)
         return fail(DEFCON_ERR_LIMIT, "workspace of %zu bytes < required %zu", workspace_bytes, need);
     cudaError_t e = launch_offset_branch(x, x_dtype == DEFCON_BF16, N, H, W, C, dw_w, dw_scale,
@@ -354,7 +359,8 @@ static int layer_carve(int N, int H, int W, int Cin, int dtype, int Cout, int K,
     // step-2 / branch workspaces sized for the full batch cover every chunk
     c->ws = align_up(path_workspace(*g, path));
     path_workspace_counters(*g, path, &c->ctr_off, &c->ctr_bytes);
-    c->tws = align_up(offset_branch_workspace(g->M, Cin));
+    c->tws = align_up(offset_branch_workspace(N, H, W, Cin, g->Ho, g->Wo, K, g->G, cv.stride_h, cv.stride_w, cv.pad_h,
+                                              cv.pad_w, cv.dil_h, cv.dil_w, dtype == DEFCON_BF16));
     c->total = c->xy + HOST_PIPE_STREAMS * (c->ws + c->tws);
     return DEFCON_OK;
 }

@@ -130,6 +130,26 @@ DEFCON_DEVICE void tma_load_2d(void* smem_dst, const CUtensorMap* map, uint64_t*
         : "memory");
 }
 
+// 3-D tiled TMA load global -> shared (coordinates innermost first; out-of-bounds elements of the
+// box are zero-filled), completion signalled on `bar` (tx bytes = the full box).
+DEFCON_DEVICE void tma_load_3d(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                               int c2) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(smem_dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
+        : "memory");
+}
+
+// 1-D bulk copy global -> shared (bytes a multiple of 16, both addresses 16-byte aligned),
+// completion signalled on `bar` (tx bytes).
+DEFCON_DEVICE void bulk_load(void* smem_dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(smem_dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
 // 4-D tiled TMA load global -> shared (coordinates innermost first; out-of-bounds elements of the
 // box are zero-filled), completion signalled on `bar` (tx bytes = the full box).
 DEFCON_DEVICE void tma_load_4d(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
@@ -203,6 +223,36 @@ DEFCON_DEVICE void mma_tf32_ss(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc
         "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
         : "memory");
 }
+
+// D[tmem] (+)= A[tmem] * B[smem desc]^T, kind::tf32 (the A operand read from tensor memory:
+// M = 128 lanes, K = 8 consecutive 32-bit columns starting at a_tmem).
+DEFCON_DEVICE void mma_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                               uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+        : "memory");
+}
+
+// registers -> tensor memory, 16 lanes x 256 bits, 4 repetitions along the columns: thread t
+// writes lanes (t/4) and (t/4)+8 of the 16-lane block at `taddr`, columns 8c + 2(t%4) and
+// 8c + 2(t%4) + 1 of repetition c: r[4c..4c+1] to the first lane, r[4c+2..4c+3] to the second.
+DEFCON_DEVICE void tmem_st_16x256b_x4(uint32_t taddr, const uint32_t (&r)[16]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.16x256b.x4.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
+        "%12, %13, %14, %15, %16};" ::"r"(taddr),
+        "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]),
+        "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+        : "memory");
+}
+DEFCON_DEVICE void tmem_st_16x256b_x2(uint32_t taddr, const uint32_t (&r)[8]) {
+    asm volatile("tcgen05.st.sync.aligned.16x256b.x2.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(taddr),
+                 "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7])
+                 : "memory");
+}
+DEFCON_DEVICE void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // Arrive on `bar` when all previously issued tcgen05.mma of this thread complete.
 DEFCON_DEVICE void mma_commit(uint64_t* bar) {

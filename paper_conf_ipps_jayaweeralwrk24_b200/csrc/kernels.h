@@ -33,7 +33,20 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                  float* offset, float* mask, float* t_ws, cudaStream_t stream);
-size_t offset_branch_workspace(int M, int C);   // bytes of the fp32 t buffer (two-pass path)
+// workspace of defcon_offset_dw_conv: the one-pass kernel's packed parameters when it can run
+// this shape (decided for the widest branch, OC = 3*G*K*K), else the two-pass t buffers
+size_t offset_branch_workspace(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph,
+                               int pw, int dh, int dw, bool x_bf16);
+// one pass per tile (offset_branch_onepass.cu): TMA-staged dw on CUDA cores -> t as tf32 hi/lo
+// operand planes in smem -> 1x1 on tcgen05 3xTF32; t never leaves the SM
+bool offset_branch_onepass_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, int ph, int pw,
+                                int dh, int dw, int OC, bool x_bf16);
+size_t offset_branch_onepass_workspace(int C, int OC);   // packed per-chunk parameter blocks
+cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int H, int W, int C,
+                                         const float* dw_w, const float* dw_scale, const float* dw_shift,
+                                         const float* pw_w, const float* pw_b, int n_off, int n_msk,
+                                         int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
+                                         float* offset, float* mask, void* ws, cudaStream_t stream);
 // single-launch branch: dw on CUDA cores -> t in smem -> 1x1 on tcgen05 (3xTF32)
 bool offset_branch_tc_supported(int C, int OC);
 cudaError_t launch_offset_branch_tc(const void* x, bool x_bf16, int N, int H, int W, int C,

@@ -503,7 +503,21 @@ cudaError_t launch_pw_tc_any(const BranchArgs& a, cudaStream_t stream) {
 
 // t as two fp32 planes (tf32 hi / lo) for the tcgen05 1x1 (or plain t in the first plane), then
 // the W2 hi / lo planes padded to 256 rows
-size_t offset_branch_workspace(int M, int C) { return (2 * (size_t)M * C + 2 * (size_t)256 * C) * sizeof(float); }
+static size_t two_pass_workspace(int M, int C) { return (2 * (size_t)M * C + 2 * (size_t)256 * C) * sizeof(float); }
+
+static bool use_onepass(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph, int pw,
+                        int dh, int dw, bool x_bf16) {
+    const char* impl = getenv("DEFCON_OFFSET_IMPL");
+    if (impl && !strcmp(impl, "two_pass")) return false;
+    return offset_branch_onepass_plan(N, H, W, C, Ho, Wo, sh, sw, ph, pw, dh, dw, 3 * G * K * K, x_bf16);
+}
+
+size_t offset_branch_workspace(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph,
+                               int pw, int dh, int dw, bool x_bf16) {
+    if (use_onepass(N, H, W, C, Ho, Wo, K, G, sh, sw, ph, pw, dh, dw, x_bf16))
+        return offset_branch_onepass_workspace(C, 3 * G * K * K);
+    return two_pass_workspace(N * Ho * Wo, C);
+}
 
 cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W, int C,
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
@@ -524,6 +538,10 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     // DEFCON_OFFSET_IMPL=tc (or DEFCON_OFFSET_TC=1) selects the single-launch tcgen05 branch
     // (offset_branch_tc.cu: t stays on chip), =row_tc the row-tile kernel with TMA-staged input
     // (offset_branch_fused.cu).  All three are parity-tested.
+    if (use_onepass(N, H, W, C, Ho, Wo, K, G, s_h, s_w, p_h, p_w, d_h, d_w, x_bf16))
+        return launch_offset_branch_onepass(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
+                                            a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
+                                            mask, t_ws, stream);
     const char* impl = getenv("DEFCON_OFFSET_IMPL");
     if (((impl && !strcmp(impl, "tc")) || getenv("DEFCON_OFFSET_TC")) && offset_branch_tc_supported(C, a.OC))
         return launch_offset_branch_tc(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b, a.n_off,

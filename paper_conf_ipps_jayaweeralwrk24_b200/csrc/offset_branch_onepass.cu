@@ -1,0 +1,582 @@
+// offset_branch_onepass.cu -- the paper's lightweight offset branch
+// as ONE pass over each tile of output pixels, the intermediate t never leaving the SM:
+//   t[c] = ReLU(scale[c] * sum_{3x3} W1[c] * x + shift[c])    depthwise 3x3 + folded BN (R10)
+//   u[o] = b2[o] + sum_c W2[o][c] * t[c]                      1x1 to OC = G*K*K*(2|3) (R11)
+//   offset = u[0 : 2GK^2] ([G][K*K][2] = (dy, dx), R4),  mask = sigmoid(u[2GK^2 :]) (R6)
+//
+// Tile = R output rows x Wseg columns of one image (R * Wseg <= 128 pixels = the UMMA M rows).
+// Per 32-channel chunk:
+//   * TMA brings the tile's input window (IR rows x IC columns x 32 channels of NHWC x, box
+//     coordinates starting at -pad: the unit zero-fills everything outside the image, which
+//     IS the depthwise conv's zero padding) into a swizzled shared-memory stage (SWIZZLE_64B
+//     for bf16's 64-byte rows, SWIZZLE_128B for fp32's 128-byte rows), XS chunks ahead;
+//   * the 8 warps compute t on the CUDA cores: task = (8 channels, output row, run of RUN
+//     adjacent pixels); for stride 1 / dilation 1 each input column of a tap row is loaded and
+//     widened once and used by every output of the run that covers it (packed FFMA2, fp32);
+//   * t goes straight into the 1x1's A operand: two tf32 planes in the canonical K-major
+//     SWIZZLE_128B layout, hi = t with the low 13 mantissa bits cleared, lo = t - hi (both exact),
+//     and W2's chunk likewise into B (rows >= OC and channels >= C are zero);
+//   * one thread issues tcgen05.mma kind::tf32 (M = 128, N = OC rounded up to 16, K = 8) three
+//     times per k-step -- lo*hi + hi*lo + hi*hi, the 3xTF32 scheme, fp32-level accuracy --
+//     accumulating in TMEM while the warps compute the next chunk (double-buffered A / B).
+// Epilogue: TMEM -> + b2 -> offsets, sigmoid -> mask.  Fixed summation order: deterministic.
+// Only x is read and only offsets / mask are written: the branch's HBM traffic is the
+// algorithmic minimum (x once + halo re-reads from L2, offsets + mask once).
+#include <algorithm>
+#include <climits>
+#include <cstdio>
+#include <cstdlib>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace defcon {
+namespace {
+
+constexpr int OP_KC = 32;              // channels per chunk = one 128-byte tf32 operand row
+constexpr uint32_t TF32_HI = 0xFFFFE000u;
+constexpr int OP_MAXT = 256;           // threads = 2 * TP (TP <= 128 pixels per tile)
+
+#ifdef DEFCON_PROBE_OP_TIMELINE   // dev probe: per-CTA phase timestamps (globaltimer, ns)
+__device__ unsigned long long g_op_tl[1024][32];
+__device__ __forceinline__ void op_stamp(int i) {
+    if (threadIdx.x == 0 && blockIdx.x < 1024 && i < 32) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_op_tl[blockIdx.x][i] = t;
+    }
+}
+#define OPTL(i) op_stamp(i)
+#else
+#define OPTL(i) ((void)0)
+#endif
+
+struct OpArgs {
+    const float* dw_w;      // [C][3][3]
+    const float* dw_scale;  // [C]
+    const float* dw_shift;  // [C]
+    const float* pw_w;      // [OC][C]
+    const float* pw_b;      // [OC] or null
+    const uint8_t* packed;  // per-chunk parameter blocks (op_pack_kernel)
+    float* offset;          // [M][n_off]
+    float* mask;            // [M][n_msk] or null
+    int H, W, C, Ho, Wo, Wv;   // Wv = Wo rounded up to even: virtual row length of the tiling
+    int MV;                 // N * Ho * Wv virtual pixels
+    int sh, sw, ph, pw, dh, dw;
+    int n_off, n_msk, OC, OCN;
+    int TP;                 // virtual pixels per tile (even; = A rows / TMEM lanes used)
+    int IR, IC;             // input window (box) rows over the stacked N*H rows / columns
+    int nch;                // 32-channel chunks
+    int XS;                 // x stages in flight
+    int x_stage;            // bytes per x stage (1024-aligned)
+    int tmem_cols, a_col;   // TMEM allocation and first A column
+};
+
+// SWIZZLE_128B: 16-byte unit (bits 4-6) XOR the 128-byte row index (bits 7-9) within 1024 B.
+__device__ __forceinline__ uint32_t sw128(uint32_t byte) { return byte ^ (((byte >> 7) & 7u) << 4); }
+// SWIZZLE_64B: 16-byte unit (bits 4-5) XOR bits 7-8 within 512 B (the x stage of bf16 input,
+// whose 32-channel box rows are 64 bytes: the swizzle span must match the box row).
+__device__ __forceinline__ uint32_t sw64(uint32_t byte) { return byte ^ (((byte >> 7) & 3u) << 4); }
+
+// 8 channels at stage byte offset `byte` of stage base `b` -> 4 fp32 pairs.
+template <int ES>
+__device__ __forceinline__ void lds_x8(const uint8_t* b, uint32_t byte, uint64_t (&v)[4]) {
+    if (ES == 2) {
+        const uint4 u = *reinterpret_cast<const uint4*>(b + sw64(byte));
+        v[0] = bf16x2_to_f32x2(u.x); v[1] = bf16x2_to_f32x2(u.y);
+        v[2] = bf16x2_to_f32x2(u.z); v[3] = bf16x2_to_f32x2(u.w);
+    } else {
+        const uint4 u0 = *reinterpret_cast<const uint4*>(b + sw128(byte));
+        const uint4 u1 = *reinterpret_cast<const uint4*>(b + sw128(byte + 16u));
+        v[0] = ((uint64_t)u0.y << 32) | u0.x; v[1] = ((uint64_t)u0.w << 32) | u0.z;
+        v[2] = ((uint64_t)u1.y << 32) | u1.x; v[3] = ((uint64_t)u1.w << 32) | u1.z;
+    }
+}
+
+// ---- packed per-chunk parameters (written once per call by op_pack_kernel into the caller's
+// workspace, then bulk-copied into shared memory with each chunk's x stage): chunk k's block is
+//   [W2 hi plane | W2 lo plane]  OCN rows x 32 K positions fp32 each, the exact shared-memory
+//        image of the UMMA B operand (K-major SWIZZLE_128B, the permuted K order below, tf32
+//        hi = w with the low 13 mantissa bits cleared, lo = w - hi; rows >= OC and channels >= C 0)
+//   [dw]  9 taps x 32 channels (transposed), then BN scale[32], shift[32]   (352 fp32)
+// K permutation: K position 8c + 2g + e holds channel 8g + 2c + e (the tcgen05.st.16x256b pattern).
+__host__ __device__ constexpr int op_block_bytes(int OCN) { return ((2 * OCN * 128 + 11 * OP_KC * 4) + 1023) & ~1023; }
+
+__global__ void __launch_bounds__(256) op_pack_kernel(const float* __restrict__ dw_w, const float* __restrict__ dw_scale,
+                                                      const float* __restrict__ dw_shift,
+                                                      const float* __restrict__ pw_w, int C, int OC, int OCN,
+                                                      uint8_t* __restrict__ packed) {
+    griddep_launch_dependents();
+    const int k = blockIdx.x;
+    uint8_t* blk = packed + (size_t)k * op_block_bytes(OCN);
+    const int B_PLANE = OCN * 128;
+    for (int e = threadIdx.x; e < OCN * OP_KC; e += blockDim.x) {      // B: (row o, K position kp)
+        const int o = e / OP_KC, kp = e % OP_KC;
+        const int cq = kp >> 3, g = (kp >> 1) & 3, ee = kp & 1;
+        const int ch = k * OP_KC + 8 * g + 2 * cq + ee;
+        const float w = (o < OC && ch < C) ? pw_w[(long)o * C + ch] : 0.f;
+        const uint32_t h = __float_as_uint(w) & TF32_HI;
+        const uint32_t byte = (uint32_t)(o * 128 + kp * 4) ^ ((uint32_t)(o & 7) << 4);
+        *reinterpret_cast<uint32_t*>(blk + byte) = h;
+        *reinterpret_cast<uint32_t*>(blk + B_PLANE + byte) = __float_as_uint(w - __uint_as_float(h));
+    }
+    float* dwp = reinterpret_cast<float*>(blk + 2 * B_PLANE);
+    for (int e = threadIdx.x; e < 11 * OP_KC; e += blockDim.x) {
+        float v = 0.f;
+        if (e < 9 * OP_KC) {                              // [tap][ch]
+            const int tap = e / OP_KC, c = k * OP_KC + e % OP_KC;
+            if (c < C) v = dw_w[(long)c * 9 + tap];
+        } else {
+            const int c = k * OP_KC + (e - 9 * OP_KC) % OP_KC;
+            if (c < C) v = (e < 10 * OP_KC ? dw_scale : dw_shift)[c];
+        }
+        dwp[e] = v;
+    }
+    griddep_wait();   // complete only after the previous kernel: the branch kernel's PDL wait covers both
+}
+
+// Warp roles.  Tile pixels are taken in pairs (virtual columns 2q, 2q+1 of a row: rows have
+// even virtual length Wv and tiles start at even pixels, so a pair never straddles a row); the
+// tile's nblk = TP/16 blocks of 8 pairs live in TMEM lane quarters: block b in lanes 32b .. 32b+15,
+// the left pixel of pair 8b+l in lane 32b+l and the right one in lane 32b+l+8 (the lane pattern
+// of tcgen05.st.16x256b).  Compute warp w (w % 4 = block, w / 4 = channel half) and lane t of it
+// work on pair l = t/4, channels 8g + 4*half .. +3 of the chunk's 32 (g = t%4): two warps per
+// block, so the warps per SM are not bounded by 16 pixels per warp.  The 4 input columns of a tap
+// row serve both pixels, the tap weights are read once for both.  t goes to the A operand in
+// TENSOR memory (tf32 hi / lo planes, 32 columns each), so the MMAs read only W2 from shared
+// memory.  The issuer warp (the first unused id) loads each chunk's x window (TMA) and packed
+// parameters (bulk copy) into a stage and issues the chunk's MMAs once the compute warps have
+// published its A operand.
+template <int ES, bool S1>
+__global__ void __maxnreg__(80)
+    offset_branch_onepass_kernel(const __grid_constant__ CUtensorMap xmap, const OpArgs a) {
+    extern __shared__ __align__(1024) uint8_t op_raw[];
+    // 1024-aligned base by pointer arithmetic on the __shared__ array (keeps every derived
+    // pointer in the shared window, so plain loads / stores compile to LDS / STS)
+    uint8_t* smem = op_raw + ((1024u - (smem_u32(op_raw) & 1023u)) & 1023u);
+    const int B_PLANE = a.OCN * 128;
+    const int PBLK = op_block_bytes(a.OCN);
+    const int STG = a.x_stage + PBLK;                          // stage = [x window | packed params]
+    uint8_t* st_base = smem;                                   // [XS] stages
+    uint8_t* zero = st_base + a.XS * STG;                      // 1 KB of zeros
+    float* bias_s = reinterpret_cast<float*>(zero + 1024);     // [256] 1x1 bias (0 when absent)
+    uint64_t* xfull = reinterpret_cast<uint64_t*>(bias_s + 256);   // [XS] stage landed
+    uint64_t* afull = xfull + a.XS;                            // [2] chunk's A published
+    uint64_t* mma_done = afull + 2;                            // [2] chunk's MMAs complete
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(mma_done + 2);
+    float* out_s = reinterpret_cast<float*>(smem);             // epilogue staging (stages)
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int TP = a.TP;
+    const int nblk = TP >> 4;                                  // 16-lane blocks (<= 4)
+    const int issuer_warp = nblk < 4 ? nblk : 8;
+    const int v0 = blockIdx.x * TP;                            // first virtual pixel of the tile
+    const uint32_t tcols = a.tmem_cols;
+    const uint32_t ACOL = a.a_col;                             // first A column (after the accumulator)
+
+    OPTL(0);
+    for (int e = tid; e < 256; e += blockDim.x) {
+        reinterpret_cast<float*>(zero)[e] = 0.f;
+        bias_s[e] = (a.pw_b && e < a.OC) ? __ldg(a.pw_b + e) : 0.f;
+    }
+    if (tid == 0) {
+        for (int s = 0; s < a.XS; ++s) mbar_init(&xfull[s], 1);
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(&afull[b], 1);
+            mbar_init(&mma_done[b], 1);
+        }
+        fence_barrier_init();
+        tma_prefetch_desc(&xmap);
+    }
+    if (warp == 0) {   // TMEM: accumulator (OCN columns) + A (hi / lo x 32 columns)
+        if (tcols == 128) tmem_alloc<128>(tmem_slot);
+        else if (tcols == 256) tmem_alloc<256>(tmem_slot);
+        else tmem_alloc<512>(tmem_slot);
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    OPTL(1);
+    griddep_wait();                     // PDL: x and the packed parameters are complete
+    griddep_launch_dependents();
+    OPTL(2);
+
+    const int HoWv = a.Ho * a.Wv;
+    const int n0 = v0 / HoWv, ho0 = (v0 - n0 * HoWv) / a.Wv;
+    const int Y0 = n0 * a.H + ho0 * a.sh - a.ph;              // window origin (stacked rows)
+
+    if (warp == issuer_warp) {
+        // ===================== TMA + MMA issuer =====================
+        if (lane == 0) {
+            const uint32_t tx = (uint32_t)(a.IR * a.IC * OP_KC * ES + PBLK);
+            auto load_stage = [&](int k, int s) {
+                uint8_t* st = st_base + s * STG;
+                mbar_arrive_expect_tx(&xfull[s], tx);
+                tma_load_3d(st, &xmap, &xfull[s], k * OP_KC, -a.pw, Y0);
+                bulk_load(st + a.x_stage, a.packed + (size_t)k * PBLK, (uint32_t)PBLK, &xfull[s]);
+            };
+            for (int k = 0; k < a.XS && k < a.nch; ++k) load_stage(k, k);
+            const uint32_t idesc = make_idesc(2u /*TF32*/, 128, (uint32_t)a.OCN);
+            int s = 0;
+            for (int k = 0; k < a.nch; ++k) {
+                const int ab = k & 1;
+                mbar_wait(&afull[ab], (uint32_t)(k >> 1) & 1u);   // A of chunk k published
+                tc_fence_after();
+                const uint32_t ah = tmem + ACOL, al = ah + 32u;
+                const uint32_t bh = smem_u32(st_base + s * STG + a.x_stage), bl = bh + B_PLANE;
+#pragma unroll
+                for (int kk = 0; kk < OP_KC / 8; ++kk) {
+                    const uint64_t dbh = make_sw128_desc(bh + kk * 32), dbl = make_sw128_desc(bl + kk * 32);
+                    mma_tf32_ts(tmem, al + kk * 8, dbh, idesc, (k | kk) != 0 ? 1u : 0u);
+                    mma_tf32_ts(tmem, ah + kk * 8, dbl, idesc, 1u);
+                    mma_tf32_ts(tmem, ah + kk * 8, dbh, idesc, 1u);
+                }
+                mma_commit(&mma_done[ab]);
+                if (k + a.XS < a.nch) {
+                    // stage s: x consumed (afull) and its W2 read by MMA(k): refill with chunk k+XS
+                    mbar_wait(&mma_done[ab], (uint32_t)(k >> 1) & 1u);
+                    load_stage(k + a.XS, s);
+                }
+                if (++s == a.XS) s = 0;
+            }
+        }
+        return;
+    }
+    if (warp >= 8 || (warp & 3) >= nblk) return;   // unused ids (small tiles)
+
+    // ===================== compute warps =====================
+    const int NC = 64 * nblk;                                  // compute threads
+    const int ctid = ((warp >> 2) * nblk + (warp & 3)) * 32 + lane;   // 0 .. NC-1
+    const int blk = warp & 3, half = warp >> 2;
+    const int l = lane >> 2, g = lane & 3;
+    const int q = 8 * blk + l;                                 // pixel pair within the tile
+    const int vp = v0 + 2 * q;                                 // virtual pixel of the left one
+    const bool pix_ok = vp < a.MV;
+    const int vpc = pix_ok ? vp : v0;
+    const int n = vpc / HoWv;
+    const int rem = vpc - n * HoWv;
+    const int ho = rem / a.Wv, wo = rem - ho * a.Wv;           // wo even
+    constexpr uint32_t PB = OP_KC * ES;                        // bytes per input position of a stage
+    const uint32_t chb = (uint32_t)(8 * g + 4 * half) * ES;    // byte offset of this thread's 4 channels
+    uint32_t row_byte[3];   // stage byte offset of tap (i, 0) of the left pixel + channels
+    uint32_t row_ok = 0;    // tap rows in the zero padding (incl. a neighbouring image's rows)
+#pragma unroll
+    for (int i = 0; i < 3; ++i) {
+        const int yy = ho * a.sh - a.ph + i * a.dh;
+        const bool ok = pix_ok && yy >= 0 && yy < a.H;
+        row_ok |= ok ? 1u << i : 0u;
+        row_byte[i] = (ok ? (uint32_t)((n * a.H + yy - Y0) * a.IC + wo * a.sw) * PB : 0u) + chb;
+    }
+    const uint32_t col_step = (uint32_t)a.dw * PB;   // next tap column
+    const uint32_t px_step = (uint32_t)a.sw * PB;    // the right pixel of the pair
+    const uint32_t a_addr = tmem + ((uint32_t)(32 * blk) << 16) + ACOL + 16u * half;
+    const int wofs = 2 * B_PLANE / 4 + 8 * g + 4 * half;       // this thread's dw weights in a stage (floats)
+
+    int s = 0;                          // stage of chunk k (k mod XS)
+    uint32_t xphase = 0;
+    for (int k = 0; k < a.nch; ++k) {
+        const uint8_t* xst = st_base + s * STG;
+        const float* wk = reinterpret_cast<const float*>(xst + a.x_stage) + wofs;
+        mbar_wait(&xfull[s], xphase);
+        if (k < 8) OPTL(4 + 2 * k);
+        // ---- depthwise 3x3 of 4 channels at two pixels, fp32 pairs (FFMA2)
+        uint64_t acc0[2] = {0ull, 0ull}, acc1[2] = {0ull, 0ull};
+#ifdef OP_PROBE_NO_DW   // dev probe: skip the depthwise work (garbage t)
+        if (row_ok == 0xFFu)
+#endif
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+            const bool ok = (row_ok >> i) & 1u;
+            const uint8_t* rb = ok ? xst : zero;
+            uint64_t w[3][2];
+#pragma unroll
+            for (int jj = 0; jj < 3; ++jj) {
+                const float4 w0 = *reinterpret_cast<const float4*>(wk + (i * 3 + jj) * OP_KC);
+                w[jj][0] = f32x2_pack(w0.x, w0.y);
+                w[jj][1] = f32x2_pack(w0.z, w0.w);
+            }
+            auto ld4 = [&](uint32_t byte, uint64_t (&v)[2]) {   // 4 channels -> 2 fp32 pairs
+                if (ES == 2) {
+                    const uint2 u = *reinterpret_cast<const uint2*>(rb + sw64(byte));
+                    v[0] = bf16x2_to_f32x2(u.x);
+                    v[1] = bf16x2_to_f32x2(u.y);
+                } else {
+                    const uint4 u = *reinterpret_cast<const uint4*>(rb + sw128(byte));
+                    v[0] = ((uint64_t)u.y << 32) | u.x;
+                    v[1] = ((uint64_t)u.w << 32) | u.z;
+                }
+            };
+            if (S1) {
+                // stride-1 / dilation-1 columns: c = 0..3 feed the left pixel through tap c and
+                // the right one through tap c - 1
+#pragma unroll
+                for (int c = 0; c < 4; ++c) {
+                    uint64_t v[2];
+                    ld4(ok ? row_byte[i] + c * PB : chb, v);
+#pragma unroll
+                    for (int p = 0; p < 2; ++p) {
+                        if (c < 3) acc0[p] = f32x2_fma(w[c][p], v[p], acc0[p]);
+                        if (c > 0) acc1[p] = f32x2_fma(w[c - 1][p], v[p], acc1[p]);
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int jj = 0; jj < 3; ++jj) {
+                    uint64_t v[2], u[2];
+                    ld4(ok ? row_byte[i] + jj * col_step : chb, v);
+                    ld4(ok ? row_byte[i] + jj * col_step + px_step : chb, u);
+#pragma unroll
+                    for (int p = 0; p < 2; ++p) {
+                        acc0[p] = f32x2_fma(w[jj][p], v[p], acc0[p]);
+                        acc1[p] = f32x2_fma(w[jj][p], u[p], acc1[p]);
+                    }
+                }
+            }
+        }
+        // ---- folded BN + ReLU, tf32 hi / lo split; register 4c' + 2x + e = channel
+        // 8g + 4*half + 2c' + e of pixel x (the 16x256b.x2 store pattern)
+        uint32_t hv[8], lv[8];
+        {
+            const float4 sc = *reinterpret_cast<const float4*>(wk + 9 * OP_KC);
+            const float4 sf = *reinterpret_cast<const float4*>(wk + 10 * OP_KC);
+            const float scv[4] = {sc.x, sc.y, sc.z, sc.w};
+            const float sfv[4] = {sf.x, sf.y, sf.z, sf.w};
+#pragma unroll
+            for (int x = 0; x < 2; ++x) {
+                const uint64_t* acc = x ? acc1 : acc0;
+#pragma unroll
+                for (int c = 0; c < 2; ++c) {
+#pragma unroll
+                    for (int e = 0; e < 2; ++e) {
+                        const float v = __uint_as_float(e ? (uint32_t)(acc[c] >> 32) : (uint32_t)(acc[c] & 0xFFFFFFFFull));
+                        const float t = fmaxf(fmaf(scv[2 * c + e], v, sfv[2 * c + e]), 0.f);
+                        const uint32_t h = __float_as_uint(t) & TF32_HI;
+                        hv[4 * c + 2 * x + e] = h;
+                        lv[4 * c + 2 * x + e] = __float_as_uint(t - __uint_as_float(h));
+                    }
+                }
+            }
+        }
+        // the single A buffer was last read by MMA(k-1)
+        if (k >= 1) mbar_wait(&mma_done[(k - 1) & 1], (uint32_t)((k - 1) >> 1) & 1u);
+        tc_fence_after();
+        tmem_st_16x256b_x2(a_addr, hv);
+        tmem_st_16x256b_x2(a_addr + 32u, lv);
+        tmem_st_wait();
+        tc_fence_before();
+        named_bar_sync(1, NC);      // A of chunk k complete; stage s read
+        if (k < 8) OPTL(5 + 2 * k);
+        if (ctid == 0) mbar_arrive(&afull[k & 1]);
+        if (++s == a.XS) {
+            s = 0;
+            xphase ^= 1u;
+        }
+    }
+    // ---- epilogue: accumulator lane = tile pixel (pair layout above), column = output channel;
+    // + b2, sigmoid on the mask channels, staged in shared memory in the global layout (the tile's
+    // real pixels are one contiguous range of m), then copied out coalesced.  Warp w reads lanes
+    // 32*(w%4) .. +15 and the column half w/4.
+    OPTL(20);
+    mbar_wait(&mma_done[(a.nch - 1) & 1], (uint32_t)((a.nch - 1) >> 1) & 1u);
+    tc_fence_after();
+    OPTL(21);
+    const int vl = min(v0 + TP, a.MV) - 1;
+    auto real_m = [&](int v, bool up) {   // m of virtual pixel v (dead column: next / previous real)
+        const int r = v / a.Wv, c = v - r * a.Wv;
+        if (c >= a.Wo) return up ? (r + 1) * a.Wo : r * a.Wo + a.Wo - 1;
+        return r * a.Wo + c;
+    };
+    const int mf = real_m(v0, true), ml = real_m(vl, false);
+    const int nreal = ml - mf + 1;
+    float* off_s = out_s;
+    float* msk_s = out_s + nreal * a.n_off;
+    {
+        const int li = lane & 15;
+        const int v = v0 + 2 * (8 * blk + (li & 7)) + (li >> 3);   // virtual pixel of lane 32*blk + li
+        const int rr = v / a.Wv, cc = v - rr * a.Wv;
+        const bool ok = lane < 16 && v < a.MV && cc < a.Wo;
+        const int dm = rr * a.Wo + cc - mf;                   // real-pixel index within the tile
+        const int ngrp = a.OCN >> 4;                           // 16-column groups
+        for (int cg = half; cg < ngrp; cg += 2) {
+            uint32_t vv[16];
+            tmem_ld_32x32b_x16(tmem + ((uint32_t)(32 * blk) << 16) + (uint32_t)(16 * cg), vv);
+            tmem_ld_wait();
+            if (!ok) continue;
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+                const int o = 16 * cg + u;
+                const float val = __uint_as_float(vv[u]) + bias_s[o];
+                if (o < a.n_off) off_s[dm * a.n_off + o] = val;
+                else if (o < a.OC) msk_s[dm * a.n_msk + (o - a.n_off)] = __fdividef(1.f, 1.f + __expf(-val));
+            }
+        }
+    }
+    tc_fence_before();
+    named_bar_sync(1, NC);   // staged; TMEM no longer read
+    if (warp == 0) {
+        tc_fence_after();
+        if (tcols == 128) tmem_dealloc<128>(tmem);
+        else if (tcols == 256) tmem_dealloc<256>(tmem);
+        else tmem_dealloc<512>(tmem);
+    }
+    {
+        float* go = a.offset + (long)mf * a.n_off;
+        for (int e = ctid; e < nreal * a.n_off; e += NC) go[e] = off_s[e];
+        if (a.n_msk) {
+            float* gm = a.mask + (long)mf * a.n_msk;
+            for (int e = ctid; e < nreal * a.n_msk; e += NC) gm[e] = msk_s[e];
+        }
+    }
+    OPTL(22);
+}
+
+struct OpPlan {
+    OpArgs a;
+    int tiles, cps;
+    size_t smem;
+};
+
+constexpr size_t OP_SMEM_CAP = 228 * 1024 - 1024;   // per SM, less the per-CTA reserve
+#ifdef OP_PROBE_ONE_CTA   // dev probe: one CTA per SM
+constexpr size_t OP_SMEM_TWO = 0;
+#else
+constexpr size_t OP_SMEM_TWO = 113 * 1024;   // two CTAs per SM
+#endif
+
+size_t op_smem(const OpArgs& a) {
+    return 1024 + (size_t)a.XS * (a.x_stage + op_block_bytes(a.OCN)) + 2048 + (a.XS + 4) * 8 + 16;
+}
+
+// Tile = TP consecutive pixels of the virtual [N][Ho][Wv] grid (a tile may run across an image
+// boundary: its input window covers the stacked N*H rows, and taps in another image's rows are
+// masked as zero padding).  TP (a multiple of 16, <= 128 = the UMMA M) spreads the pixels evenly
+// over the CTA slots: minimise rounds x CTAs-per-SM x TP, the pixels one SM processes.
+bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, int ph, int pw, int dh, int dw,
+                  int OC, int es, OpPlan* p) {
+    OpArgs& a = p->a;
+    a.H = H; a.W = W; a.C = C; a.Ho = Ho; a.Wo = Wo;
+    a.Wv = Wo + (Wo & 1);
+    a.sh = sh; a.sw = sw; a.ph = ph; a.pw = pw; a.dh = dh; a.dw = dw;
+    a.OC = OC;
+    a.OCN = (OC + 15) & ~15;
+    const long MV = (long)N * Ho * a.Wv;
+    if (a.OCN > 256 || C % 8 != 0 || MV >= (1L << 31)) return false;
+    a.MV = (int)MV;
+    a.nch = (C + OP_KC - 1) / OP_KC;
+    a.IC = (a.Wv - 1) * sw + 2 * dw + 1;
+    if (a.IC > 256) return false;                 // TMA box limit: wide images keep the two-pass path
+    // TMEM: accumulator columns (OCN rounded to 32), then the A operand (hi, lo) x 32 columns
+    a.a_col = (a.OCN + 31) & ~31;
+    a.tmem_cols = a.a_col + 64 <= 128 ? 128 : a.a_col + 64 <= 256 ? 256 : 512;
+    int sms = 148;
+    {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    long best = LONG_MAX;
+    bool found = false;
+    for (int TP = 16; TP <= 64; TP += 16) {
+        if (TP > Ho * a.Wv && TP > 16) break;     // a tile spans at most two images
+        OpArgs t = a;
+        t.TP = TP;
+        const int orows = (a.Wv - 2 + TP + a.Wv - 1) / a.Wv;          // output rows a tile can touch
+        t.IR = (orows - 1) * sh + std::max(0, H - Ho * sh) + 2 * dh + 1;
+        if (t.IR > 256) continue;
+        t.x_stage = (int)(((size_t)t.IR * t.IC * OP_KC * es + 1023) & ~size_t(1023));
+        // epilogue staging ([TP][OC] fp32) reuses the x stages
+        t.XS = 3;
+        while (op_smem(t) > OP_SMEM_CAP / 3 && t.XS > 2) --t.XS;
+        if ((size_t)TP * OC * 4 > (size_t)t.XS * t.x_stage) continue;
+        const size_t sm = op_smem(t);
+        if (sm > OP_SMEM_CAP) continue;
+        // CTAs per SM: shared memory, TMEM columns (512 per SM), registers
+        const int nwarps = TP == 64 ? 9 : (TP / 16 < 4 ? 4 + TP / 16 : 9);
+        int cps = (int)std::min<size_t>(OP_SMEM_CAP / sm, 512 / t.tmem_cols);
+        // 80 registers per thread (__maxnreg__): 6 warps per SM sub-partition (16K registers each)
+        cps = std::min(cps, 24 / nwarps);
+        if (cps < 1) continue;
+        const long tiles = (MV + TP - 1) / TP;
+        const long rounds = (tiles + (long)sms * cps - 1) / ((long)sms * cps);
+        const long cost = rounds * cps * (TP + 16);   // + a per-tile overhead: ties go to larger tiles
+        if (cost < best) {
+            best = cost;
+            a = t;
+            p->tiles = (int)tiles;
+            p->cps = cps;
+            p->smem = sm;
+            found = true;
+        }
+    }
+    return found;
+}
+
+template <int ES>
+cudaError_t launch_op(const OpPlan& p, const CUtensorMap& xmap, cudaStream_t stream) {
+    if (getenv("DEFCON_DEBUG"))
+        fprintf(stderr, "defcon onepass: TP=%d tiles=%d cps=%d XS=%d IR=%d IC=%d smem=%zu tmem=%d\n", p.a.TP,
+                p.tiles, p.cps, p.a.XS, p.a.IR, p.a.IC, p.smem, p.a.tmem_cols);
+    const bool s1 = p.a.sw == 1 && p.a.dw == 1;
+    auto kern = s1 ? offset_branch_onepass_kernel<ES, true> : offset_branch_onepass_kernel<ES, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
+    if (e != cudaSuccess) return e;
+    const int nblk = p.a.TP / 16;
+    const int threads = 32 * (nblk < 4 ? 4 + nblk : 9);   // compute warps 0..nblk-1, 4..3+nblk + issuer
+    return launch_pdl(kern, dim3(p.tiles), dim3(threads), p.smem, stream, xmap, p.a);
+}
+
+}  // namespace
+
+#ifdef DEFCON_PROBE_OP_TIMELINE
+extern "C" int defcon_debug_op_timeline(unsigned long long* host) {
+    return (int)cudaMemcpyFromSymbol(host, g_op_tl, sizeof(g_op_tl));
+}
+#endif
+
+bool offset_branch_onepass_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, int ph, int pw,
+                                int dh, int dw, int OC, bool x_bf16) {
+    OpPlan p;
+    return get_encode_tiled() != nullptr &&
+           make_op_plan(N, H, W, C, Ho, Wo, sh, sw, ph, pw, dh, dw, OC, x_bf16 ? 2 : 4, &p);
+}
+
+size_t offset_branch_onepass_workspace(int C, int OC) {
+    const int OCN = (OC + 15) & ~15;
+    return (size_t)((C + OP_KC - 1) / OP_KC) * op_block_bytes(OCN);
+}
+
+cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int H, int W, int C,
+                                         const float* dw_w, const float* dw_scale, const float* dw_shift,
+                                         const float* pw_w, const float* pw_b, int n_off, int n_msk,
+                                         int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
+                                         float* offset, float* mask, void* ws, cudaStream_t stream) {
+    const int es = x_bf16 ? 2 : 4;
+    OpPlan p;
+    if (!make_op_plan(N, H, W, C, Ho, Wo, s_h, s_w, p_h, p_w, d_h, d_w, n_off + n_msk, es, &p))
+        return cudaErrorInvalidValue;
+    OpArgs& a = p.a;
+    a.dw_w = dw_w; a.dw_scale = dw_scale; a.dw_shift = dw_shift;
+    a.pw_w = pw_w; a.pw_b = pw_b; a.offset = offset; a.mask = mask;
+    a.n_off = n_off; a.n_msk = n_msk;
+    a.packed = static_cast<const uint8_t*>(ws);
+    cudaError_t e = launch_pdl(op_pack_kernel, dim3(a.nch), dim3(256), 0, stream, dw_w, dw_scale, dw_shift, pw_w, C,
+                               a.OC, a.OCN, static_cast<uint8_t*>(ws));
+    if (e != cudaSuccess) return e;
+    PFN_encodeTiled encode = get_encode_tiled();
+    if (!encode) return cudaErrorNotSupported;
+    // x as a 3-D tensor [N*H][W][C] (C innermost); box = 32 channels x IC columns x IR rows
+    CUtensorMap xmap;
+    cuuint64_t dims[3] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)N * H};
+    cuuint64_t strides[2] = {(cuuint64_t)C * es, (cuuint64_t)W * C * es};
+    cuuint32_t box[3] = {(cuuint32_t)OP_KC, (cuuint32_t)a.IC, (cuuint32_t)a.IR};
+    cuuint32_t estr[3] = {1, 1, 1};
+    CUresult cr = encode(&xmap, x_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
+                         const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         x_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (cr != CUDA_SUCCESS) return cudaErrorInvalidValue;
+    return x_bf16 ? launch_op<2>(p, xmap, stream) : launch_op<4>(p, xmap, stream);
+}
+
+}  // namespace defcon

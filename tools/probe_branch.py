@@ -1,9 +1,8 @@
 """Time the lightweight offset branch (defcon_offset_dw_conv) alone, graph-replayed, per config.
 
   python tools/probe_branch.py [config,...]
-Prints one JSON line per (config, path): the default two-launch path ("two_pass"), the
-single-launch tcgen05 kernel ("tc") and the TMA-staged row-tile kernel ("row_tc"), selected
-through DEFCON_OFFSET_IMPL.
+Prints one JSON line per (config, path): the default one-pass kernel ("onepass") and the
+two-launch path ("two_pass", dw kernel + 1x1 kernel through an HBM intermediate).
 """
 import json
 import os
@@ -50,8 +49,8 @@ if __name__ == "__main__":
                                                              "yolact_r101_c4_v2_g4", "yolact_r101_c5_v2"]
     d.load_library()
     for n in names:
-        c = configs.SINGLE_LAYER[n]
-        for path in ("row_tc", "tc", "two_pass"):
+        c = configs.SINGLE_LAYER[n] if n in configs.SINGLE_LAYER else {l.name: l for l in configs.stack_layers(64)}[n]
+        for path in ("onepass", "two_pass"):
             os.environ["DEFCON_OFFSET_IMPL"] = path
             us = time_branch(c)
             byt = configs.offset_branch_compulsory_bytes(c)
