@@ -110,7 +110,8 @@ __global__ void __launch_bounds__(256) op_pack_kernel(const float* __restrict__ 
     const int k = blockIdx.x;
     uint8_t* blk = packed + (size_t)k * op_block_bytes(OCN);
     const int B_PLANE = OCN * 128;
-    for (int e = threadIdx.x; e < OCN * OP_KC; e += blockDim.x) {      // B: (row o, K position kp)
+    const int nthr = blockDim.x * gridDim.y, t0 = blockIdx.y * blockDim.x + threadIdx.x;
+    for (int e = t0; e < OCN * OP_KC; e += nthr) {      // B: (row o, K position kp)
         const int o = e / OP_KC, kp = e % OP_KC;
         const int cq = kp >> 3, g = (kp >> 1) & 3, ee = kp & 1;
         const int ch = k * OP_KC + 8 * g + 2 * cq + ee;
@@ -121,7 +122,7 @@ __global__ void __launch_bounds__(256) op_pack_kernel(const float* __restrict__ 
         *reinterpret_cast<uint32_t*>(blk + B_PLANE + byte) = __float_as_uint(w - __uint_as_float(h));
     }
     float* dwp = reinterpret_cast<float*>(blk + 2 * B_PLANE);
-    for (int e = threadIdx.x; e < 11 * OP_KC; e += blockDim.x) {
+    for (int e = t0; e < 11 * OP_KC; e += nthr) {
         float v = 0.f;
         if (e < 9 * OP_KC) {                              // [tap][ch]
             const int tap = e / OP_KC, c = k * OP_KC + e % OP_KC;
@@ -132,7 +133,6 @@ __global__ void __launch_bounds__(256) op_pack_kernel(const float* __restrict__ 
         }
         dwp[e] = v;
     }
-    griddep_wait();   // complete only after the previous kernel: the branch kernel's PDL wait covers both
 }
 
 // Warp roles.  Tile pixels are taken in pairs (virtual columns 2q, 2q+1 of a row: rows have
@@ -560,8 +560,10 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
     a.pw_w = pw_w; a.pw_b = pw_b; a.offset = offset; a.mask = mask;
     a.n_off = n_off; a.n_msk = n_msk;
     a.packed = static_cast<const uint8_t*>(ws);
-    cudaError_t e = launch_pdl(op_pack_kernel, dim3(a.nch), dim3(256), 0, stream, dw_w, dw_scale, dw_shift, pw_w, C,
-                               a.OC, a.OCN, static_cast<uint8_t*>(ws));
+    // plain stream order (not PDL): measured faster behind a host-to-device copy in the host entry
+    op_pack_kernel<<<dim3(a.nch, (a.OCN * OP_KC + 255) / 256), 256, 0, stream>>>(dw_w, dw_scale, dw_shift, pw_w, C,
+                                                                               a.OC, a.OCN, static_cast<uint8_t*>(ws));
+    cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     PFN_encodeTiled encode = get_encode_tiled();
     if (!encode) return cudaErrorNotSupported;
