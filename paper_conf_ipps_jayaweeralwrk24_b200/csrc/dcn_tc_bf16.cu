@@ -47,6 +47,19 @@ constexpr int TPR = 4;               // producer threads per 128-byte A row (32 
 constexpr int ROWS = BM * TPR / NPT; // A rows per producer thread
 constexpr int RPW = 32 / TPR;        // rows per warp per pass
 
+#ifdef DEFCON_PROBE_KTRACE   // dev probe: per-k-iteration event clock64 stamps of CTA `KTRACE_CTA`
+__device__ long long g_kt[8][64];
+#ifndef KTRACE_CTA
+#define KTRACE_CTA 5
+#endif
+__device__ __forceinline__ void kt_stamp(int ev, int q) {
+    if (blockIdx.x == KTRACE_CTA && q < 64) g_kt[ev][q] = clock64();
+}
+#define KT(ev, q) kt_stamp(ev, q)
+#else
+#define KT(ev, q) ((void)0)
+#endif
+
 #ifdef DEFCON_PROBE_TIMELINE   // dev probe: per-CTA phase timestamps (globaltimer, ns)
 __device__ unsigned long long g_tl[256][16];
 __device__ __forceinline__ void tl_stamp(int i) {
@@ -648,7 +661,9 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         const int nlayer = nchunk != chunk ? layer + BK / 4 : layer;
 
         const int s = q % STAGES;
+        if (t == 0) KT(0, q);
         mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
+        if (t == 0) KT(1, q);
         const uint32_t stage = a_s + s * A_STAGE_BYTES;
 #pragma unroll
         for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
@@ -661,6 +676,8 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
             if (PAIR) mbar_arrive_cluster(&full_a[s], 0);   // the pair's MMA issuer is rank 0
             else mbar_arrive(&full_a[s]);
         }
+        if (t == 0) KT(2, q);
+        if (t == 224) KT(7, q);   // the last producer warp
 
         if (has_next && !prefetch) {          // offset group changes: new table
             named_bar_sync(1, NPT);
@@ -865,8 +882,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         mbar_wait_cluster(&full_a[s], ph);
                         mbar_wait_cluster(&full_b[s], ph);
                     } else {
+                        KT(3, q);
                         mbar_wait(&full_a[s], ph);
+                        KT(4, q);
                         mbar_wait(&full_b[s], ph);
+                        KT(5, q);
                     }
                     tc_fence_after();
                     const uint32_t a_addr = smem_u32(sA + s * A_STAGE_BYTES);
@@ -888,6 +908,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     }
                     if (PAIR) mma_commit_pair(&empty[s], 0x3);
                     else mma_commit(&empty[s]);
+                    KT(6, q);
                 }
                 if (PAIR) mma_commit_pair(&tmem_full[buf], 0x3);
                 else mma_commit(&tmem_full[buf]);
@@ -1109,6 +1130,12 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
 }
 
 }  // namespace
+
+#ifdef DEFCON_PROBE_KTRACE
+extern "C" int defcon_debug_ktrace(long long* host) {
+    return (int)cudaMemcpyFromSymbol(host, g_kt, sizeof(g_kt));
+}
+#endif
 
 #ifdef DEFCON_PROBE_TIMELINE
 extern "C" int defcon_debug_timeline(unsigned long long* host) {
