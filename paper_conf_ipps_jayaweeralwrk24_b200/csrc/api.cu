@@ -92,7 +92,7 @@ static int make_geom(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
     return DEFCON_OK;
 }
 
-enum class Path { SIMT_F32, SIMT_BF16, TC_BF16 };
+enum class Path { SIMT_F32, SIMT_BF16, TC_BF16, TC_F32 };
 
 static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, Path* path) {
     if (sampler != DEFCON_SAMPLER_LDG && sampler != DEFCON_SAMPLER_TEX && sampler != DEFCON_SAMPLER_HYBRID)
@@ -109,21 +109,27 @@ static int select_path(const DcnGeom& g, int dtype, int sampler, int fp32_mode, 
     if (dtype == DEFCON_BF16) {
         *path = dcn_tc_bf16_supported(g) ? Path::TC_BF16 : Path::SIMT_BF16;
     } else {
-        if (fp32_mode == DEFCON_FP32_3XTF32)
-            return fail(DEFCON_ERR_UNSUPPORTED, "3xTF32 fp32 path not built in this version");
-        *path = Path::SIMT_F32;
+        if (fp32_mode == DEFCON_FP32_3XTF32) {
+            if (!dcn_tc_f32_supported(g))
+                return fail(DEFCON_ERR_UNSUPPORTED,
+                            "3xTF32 tensor-core path needs Cin/G %% 32 == 0 and Cout %% 16 == 0");
+            *path = Path::TC_F32;
+        } else {
+            *path = Path::SIMT_F32;
+        }
     }
     return DEFCON_OK;
 }
 
 static size_t path_workspace(const DcnGeom& g, Path path) {
-    return path == Path::TC_BF16 ? dcn_tc_bf16_workspace(g) : 0;
+    return path == Path::TC_BF16 ? dcn_tc_bf16_workspace(g) : path == Path::TC_F32 ? dcn_tc_f32_workspace(g) : 0;
 }
 // The workspace byte range [*off, *off + *bytes) that must be zero before a launch.
 static void path_workspace_counters(const DcnGeom& g, Path path, size_t* off, size_t* bytes) {
     *off = 0;
     *bytes = 0;
     if (path == Path::TC_BF16) dcn_tc_bf16_workspace_counters(g, off, bytes);
+    if (path == Path::TC_F32) dcn_tc_f32_workspace_counters(g, off, bytes);
 }
 
 }  // namespace defcon
@@ -242,7 +248,7 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     rc = select_path(g, dtype, sampler, fp32_mode, &path);
     if (rc) return rc;
     // the tensor-core producers gather x with 32-byte vector loads (ld.global.nc.v8)
-    if (path == Path::TC_BF16 && !aligned32(x))
+    if ((path == Path::TC_BF16 || path == Path::TC_F32) && !aligned32(x))
         return fail(DEFCON_ERR_MISALIGNED, "x must be 32-byte aligned for the tensor-core path");
     TexPlan* tp = nullptr;
     if (sampler == DEFCON_SAMPLER_TEX || sampler == DEFCON_SAMPLER_HYBRID) {
@@ -264,6 +270,7 @@ int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin, const float*
     switch (path) {
         case Path::TC_BF16: e = launch_dcn_tc_bf16(g, p, workspace, workspace_bytes, tp,
                                                    sampler == DEFCON_SAMPLER_HYBRID, st, &detail); break;
+        case Path::TC_F32: e = launch_dcn_tc_f32(g, p, workspace, workspace_bytes, st, &detail); break;
         case Path::SIMT_BF16: e = launch_dcn_simt(g, p, true, st); break;
         default: e = launch_dcn_simt(g, p, false, st); break;
     }

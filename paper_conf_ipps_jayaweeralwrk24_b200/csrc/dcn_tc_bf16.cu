@@ -24,6 +24,7 @@
 // sampling metadata (4 corner offsets, 4 mask-scaled weights) is built once per
 // (tile, offset group) into shared memory and reused by every chunk of that group.
 #include <algorithm>
+#include <type_traits>
 #include <cstdio>
 #include <cstdlib>
 
@@ -35,7 +36,17 @@ namespace {
 
 constexpr int BM = 128;          // rows per tile (UMMA M)
 constexpr int BK = 64;           // bf16 elements per K chunk (= one 128-byte swizzle row)
-constexpr int A_STAGE_BYTES = BM * BK * 2;
+constexpr int A_PLANE = BM * 128;   // one A operand plane: BM rows x 128 bytes
+// Element type of x / W / y: bf16 (kind::f16, one plane, 64 channels per k-iteration) or fp32
+// (kind::tf32 3xTF32: hi / lo planes, 32 channels per k-iteration).  A k-iteration covers one
+// 128-byte row of channels either way.
+template <bool F32>
+struct Elem {
+    static constexpr int ES = F32 ? 4 : 2;           // bytes per element
+    static constexpr int CPI = 128 / ES;             // channels per k-iteration
+    static constexpr int PLANES = F32 ? 2 : 1;       // operand planes (tf32 hi / lo)
+    static constexpr int A_STAGE = A_PLANE * PLANES;
+};
 constexpr int META_ENTRY = 32;   // int4 corner offsets + float4 weights
 constexpr int NPW = 8;           // producer warps
 constexpr int EPI_WARP0 = 8;     // 4 epilogue warps: TMEM lane quarters 0..3
@@ -73,17 +84,18 @@ __device__ __forceinline__ void tl_stamp(int i) {
 #endif
 
 struct TcArgs {
-    const __nv_bfloat16* x;
+    const void* x;
     const float* offset;
     const float* mask;
     const float* bias;
-    __nv_bfloat16* y;
+    void* y;
     float* partials;       // [2 * gridDim.x][BLOCK_N / 4][BM][4] fp32
     int* counters;         // [num_tiles], zeroed before launch
     int H, W, Cin, Cout, Kw, Ho, Wo;
     int sh, sw, ph, pw, dh, dw;
     int G, Cg, M, KK;
-    int ipt;               // k-iterations per tile = (Cin / BK) * KK
+    int ipt;               // k-iterations per tile = (Cin / CPI) * KK
+    int es, cpi;           // element bytes, channels per k-iteration
     int n_tiles_n;         // tiles along Cout
     long long total_iters; // num_tiles * ipt
     unsigned long long tex;          // DEFCON_SAMPLER_TEX: stacked-image texture object, else 0
@@ -98,12 +110,14 @@ __host__ __device__ constexpr int bias_smem_offset(int stages, int nbuf) {
     return (((3 * stages + 2 * nbuf) * 8 + 12) + 15) & ~15;
 }
 
-template <int BLOCK_N, bool PAIR = false>
+template <int BLOCK_N, bool PAIR = false, bool F32 = false>
 struct TcCfg {
     static constexpr int UMMA_N = BLOCK_N > 256 ? 256 : BLOCK_N;
     static constexpr int N_MMA = BLOCK_N / UMMA_N;
     static constexpr int B_ROWS = PAIR ? BLOCK_N / 2 : BLOCK_N;   // B rows staged by this CTA
-    static constexpr int B_STAGE_BYTES = B_ROWS * BK * 2;
+    static constexpr int B_PLANE = B_ROWS * 128;
+    static constexpr int B_STAGE_BYTES = B_PLANE * Elem<F32>::PLANES;
+    static constexpr int A_STAGE_BYTES = Elem<F32>::A_STAGE;
     static constexpr int STAGE_BYTES = A_STAGE_BYTES + B_STAGE_BYTES;
     static constexpr int NBUF = BLOCK_N <= 256 ? 2 : 1;      // TMEM accumulator buffers
     static constexpr int TMEM_COLS = (BLOCK_N * NBUF) < 32 ? 32 : BLOCK_N * NBUF;
@@ -203,7 +217,7 @@ __device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& 
             const bool vy0 = (y0 >= 0) && (y0 < a.H), vy1 = (y0 + 1 >= 0) && (y0 + 1 < a.H);
             const bool vx0 = (x0 >= 0) && (x0 < a.W), vx1 = (x0 + 1 >= 0) && (x0 + 1 < a.W);
             const uint32_t base = (uint32_t)(rp.n * a.H);
-            const uint32_t rowb = (uint32_t)a.Cin * 2u;   // bytes per pixel
+            const uint32_t rowb = (uint32_t)(a.Cin * a.es);   // bytes per pixel
             if (vy0 && vx0) { off.x = ((base + y0) * a.W + x0) * rowb;         wt.x = (1.f - ly) * (1.f - lx) * mk; }
             if (vy0 && vx1) { off.y = ((base + y0) * a.W + x0 + 1) * rowb;     wt.y = (1.f - ly) * lx * mk; }
             if (vy1 && vx0) { off.z = ((base + y0 + 1) * a.W + x0) * rowb;     wt.z = ly * (1.f - lx) * mk; }
@@ -375,6 +389,48 @@ struct Sampler<true> {
     }
 };
 
+// fp32 x (3xTF32 path): the 4 corner vectors of 8 channels, fp32 bilinear sum (packed FFMA2,
+// no widening), then the tf32 split written to the two A planes: hi = v with the low 13
+// mantissa bits cleared, lo = v - hi (both exact; the MMAs take lo*hi + hi*lo + hi*hi).
+__device__ __forceinline__ void lerp_store_row_f32(const RowLoad& L, uint32_t d0, uint32_t d1) {
+    uint64_t acc[4];
+    const float wq[4] = {L.w.x, L.w.y, L.w.z, L.w.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const uint64_t w2 = f32x2_pack(wq[q], wq[q]);
+#pragma unroll
+        for (int h = 0; h < 4; ++h) {
+            const uint64_t c = ((uint64_t)L.v[q].w[2 * h + 1] << 32) | L.v[q].w[2 * h];
+            acc[h] = q == 0 ? f32x2_mul(c, w2) : f32x2_fma(c, w2, acc[h]);
+        }
+    }
+    uint32_t hi[8], lo[8];
+#pragma unroll
+    for (int h = 0; h < 4; ++h) {
+        const float v0 = __uint_as_float((uint32_t)(acc[h] & 0xFFFFFFFFull));
+        const float v1 = __uint_as_float((uint32_t)(acc[h] >> 32));
+        hi[2 * h] = __float_as_uint(v0) & 0xFFFFE000u;
+        hi[2 * h + 1] = __float_as_uint(v1) & 0xFFFFE000u;
+        lo[2 * h] = __float_as_uint(v0 - __uint_as_float(hi[2 * h]));
+        lo[2 * h + 1] = __float_as_uint(v1 - __uint_as_float(hi[2 * h + 1]));
+    }
+    st_shared_v4(d0, hi[0], hi[1], hi[2], hi[3]);
+    st_shared_v4(d1, hi[4], hi[5], hi[6], hi[7]);
+    st_shared_v4(d0 + A_PLANE, lo[0], lo[1], lo[2], lo[3]);
+    st_shared_v4(d1 + A_PLANE, lo[4], lo[5], lo[6], lo[7]);
+}
+
+struct SamplerF32 {
+    using Load = RowLoad;
+    static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
+                                                 uint32_t meta) {
+        issue_row(L, xb, meta);
+    }
+    static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
+        lerp_store_row_f32(L, lo, hi);
+    }
+};
+
 // CTA range -> segments helper (every role walks the same sequence).
 __device__ __forceinline__ int count_segments(const TcArgs& a, long long it_begin, long long it_end) {
     if (it_end <= it_begin) return 0;
@@ -418,7 +474,10 @@ __device__ __forceinline__ int ld_acquire_gpu(const int* p) {
 // swizzled layout (conflict-free) and stored by one TMA bulk-tensor store (rows >= M and
 // columns >= Cout are clipped by the TMA unit).  Two buffers alternate per warp.
 constexpr int CS = 32;
-constexpr int EPI_SCRATCH_PER_WARP = 2 * 2048;
+constexpr int EPI_SCRATCH_PER_WARP = 2 * 2048;   // bf16: two 2 KB buffers (32 rows x 64 B)
+// fp32 y: two 4 KB buffers per warp (32 rows x 128 B, 128-byte swizzle)
+template <bool F32>
+__host__ __device__ constexpr int epi_scratch_per_warp() { return F32 ? 2 * 4096 : EPI_SCRATCH_PER_WARP; }
 
 __device__ __forceinline__ void store_group_tma(const CUtensorMap* ymap, uint8_t* scratch, int gi,
                                                 const uint32_t (&pk)[CS / 2], int col, int row0,
@@ -441,7 +500,29 @@ __device__ __forceinline__ void store_group_tma(const CUtensorMap* ymap, uint8_t
     }
 }
 
-template <int BLOCK_N, int NCOLS, bool PAIR>
+// fp32 y: 32 columns of this lane's row (128 B) into a 4 KB buffer in the 128-byte swizzled
+// layout (16-byte unit c of row r at c ^ (r % 8)), stored by one 32 x 32 TMA box.
+__device__ __forceinline__ void store_group_tma_f32(const CUtensorMap* ymap, uint8_t* scratch, int gi,
+                                                    const float (&v)[CS], int col, int row0, int lane) {
+    uint8_t* buf = scratch + (gi & 1) * 4096;
+    if (gi >= 2) {
+        if (lane == 0) bulk_wait_read<1>();
+        __syncwarp();
+    }
+    const uint32_t base = smem_u32(buf) + lane * 128;
+#pragma unroll
+    for (int cc = 0; cc < 8; ++cc)
+        st_shared_v4(base + ((cc ^ (lane & 7)) << 4), __float_as_uint(v[4 * cc]), __float_as_uint(v[4 * cc + 1]),
+                     __float_as_uint(v[4 * cc + 2]), __float_as_uint(v[4 * cc + 3]));
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {
+        tma_store_2d(ymap, buf, col, row0);
+        bulk_commit();
+    }
+}
+
+template <int BLOCK_N, int NCOLS, bool PAIR, bool F32>
 __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensorMap* ymap, const Segment& sg,
                                                  uint32_t tacc, int r, int col0, int bar_id, int nthr,
                                                  bool leader, int* fix_flag, long long T, int nct,
@@ -519,17 +600,22 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
 #pragma unroll
             for (int u = 0; u < CS; ++u) acc[u] += __uint_as_float(v[u]);
         }
-        uint32_t pk[CS / 2];
 #pragma unroll
         for (int u = 0; u < CS / 4; ++u) {
             const int co = n0 + c + 4 * u;
             float4 bb = make_float4(0.f, 0.f, 0.f, 0.f);
             if (bias_s) bb = *reinterpret_cast<const float4*>(bias_s + co);     // broadcast
             else if (a.bias && co < a.Cout) bb = __ldg(reinterpret_cast<const float4*>(a.bias + co));
-            pk[2 * u] = pack_bf16x2(acc[4 * u] + bb.x, acc[4 * u + 1] + bb.y);
-            pk[2 * u + 1] = pack_bf16x2(acc[4 * u + 2] + bb.z, acc[4 * u + 3] + bb.w);
+            acc[4 * u] += bb.x; acc[4 * u + 1] += bb.y; acc[4 * u + 2] += bb.z; acc[4 * u + 3] += bb.w;
         }
-        store_group_tma(ymap, scratch, gi, pk, n0 + c, row0, lane);
+        if (F32) {
+            store_group_tma_f32(ymap, scratch, gi, acc, n0 + c, row0, lane);
+        } else {
+            uint32_t pk[CS / 2];
+#pragma unroll
+            for (int u = 0; u < CS / 2; ++u) pk[u] = pack_bf16x2(acc[2 * u], acc[2 * u + 1]);
+            store_group_tma(ymap, scratch, gi, pk, n0 + c, row0, lane);
+        }
     };
     auto drain = [&]() {
         if (lane == 0) bulk_wait_all();
@@ -626,16 +712,17 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
 // soon as the row's registers are free (rolling prefetch).  Warps with TEXW use the texture
 // sampler, the others LDG gathers + software lerp; the metadata table holds each row in the
 // format its warp consumes (warp of row r = (r mod 64) / 8).
-template <bool TEXW, int STAGES, int NTEX, bool PAIR>
+template <bool TEXW, int STAGES, int NTEX, bool PAIR, bool F32>
 __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
                                                 const uint32_t (&dst_lo)[ROWS], const uint32_t (&dst_hi)[ROWS],
                                                 const uint32_t (&mrow)[ROWS], uint32_t a_s, uint64_t* empty,
                                                 uint64_t* full_a, int t, int sub, int lane, int next_m0) {
-    using Smp = Sampler<TEXW>;
+    using Smp = typename std::conditional<F32, SamplerF32, Sampler<TEXW>>::type;
+    using E = Elem<F32>;
     const int m0 = tile_m0<PAIR>(a, sg.tile);
     int chunk = sg.kb / a.KK;
     int tap = sg.kb - chunk * a.KK;
-    int g = (chunk * BK) / a.Cg;
+    int g = (chunk * E::CPI) / a.Cg;
     named_bar_sync(1, NPT);          // previous table no longer read
 #ifdef DEFCON_PROBE_TL_META
     if (t == 0) TL(9);
@@ -645,7 +732,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     prefetch_meta_l2(a, next_m0, t);
     if (t == 0) TL(10 + (q ? 1 : 0));     // metadata table ready (first / later segment)
     // position of this thread's 16 channels: byte pointer (LDG) / texture layer (TEX)
-    const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + (chunk * BK + sub * 16) * 2;
+    const uint8_t* xb = reinterpret_cast<const uint8_t*>(a.x) + 128 * chunk + 32 * sub;
     int layer = chunk * (BK / 4) + sub * 4;
     typename Smp::Load L[ROWS];
 #pragma unroll
@@ -655,16 +742,16 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         if (ntap == a.KK) { ntap = 0; ++nchunk; }
         const bool has_next = kt + 1 < sg.ke;
         int ng = g;
-        if (has_next && nchunk != chunk) ng = (nchunk * BK) / a.Cg;
+        if (has_next && nchunk != chunk) ng = (nchunk * E::CPI) / a.Cg;
         const bool prefetch = has_next && ng == g;
-        const uint8_t* nxb = nchunk != chunk ? xb + BK * 2 : xb;
+        const uint8_t* nxb = nchunk != chunk ? xb + 128 : xb;
         const int nlayer = nchunk != chunk ? layer + BK / 4 : layer;
 
         const int s = q % STAGES;
         if (t == 0) KT(0, q);
         mbar_wait(&empty[s], ((uint32_t)(q / STAGES) & 1u) ^ 1u);
         if (t == 0) KT(1, q);
-        const uint32_t stage = a_s + s * A_STAGE_BYTES;
+        const uint32_t stage = a_s + s * E::A_STAGE;
 #pragma unroll
         for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
             Smp::store(L[p], stage + dst_lo[p], stage + dst_hi[p]);
@@ -694,19 +781,22 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     }
 }
 
-template <int BLOCK_N, int STAGES, int NTEX, bool PAIR>
+// F32: fp32 x / W / y on kind::tf32 with the 3xTF32 split (wmap = W hi plane, wmap_lo = W lo
+// plane, both prepared by dcn_w_split_kernel); otherwise bf16 on kind::f16 (wmap_lo unused).
+template <int BLOCK_N, int STAGES, int NTEX, bool PAIR, bool F32>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
-    dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const __grid_constant__ CUtensorMap ymap,
-                           const TcArgs a) {
-    using Cfg = TcCfg<BLOCK_N, PAIR>;
+    dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const __grid_constant__ CUtensorMap wmap_lo,
+                           const __grid_constant__ CUtensorMap ymap, const TcArgs a) {
+    using Cfg = TcCfg<BLOCK_N, PAIR, F32>;
+    constexpr int EPI_W = epi_scratch_per_warp<F32>();
 
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                ~uintptr_t(1023));
     uint8_t* sA = smem;
-    uint8_t* sB = smem + STAGES * A_STAGE_BYTES;
-    uint8_t* epi_scratch = sB + STAGES * Cfg::B_STAGE_BYTES;   // 4 epilogue warps x 4 KB
-    uint8_t* meta = epi_scratch + 4 * EPI_SCRATCH_PER_WARP;
+    uint8_t* sB = smem + STAGES * Cfg::A_STAGE_BYTES;
+    uint8_t* epi_scratch = sB + STAGES * Cfg::B_STAGE_BYTES;   // 4 epilogue warps x EPI_W
+    uint8_t* meta = epi_scratch + 4 * EPI_W;
     uint64_t* bars = reinterpret_cast<uint64_t*>(meta + BM * a.KK * META_ENTRY);
     uint64_t* full_a = bars;
     uint64_t* full_b = bars + STAGES;
@@ -742,6 +832,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         fence_barrier_init();
         tma_prefetch_desc(&wmap);
+        if (F32) tma_prefetch_desc(&wmap_lo);
         tma_prefetch_desc(&ymap);
     }
     if (warp == MMA_WARP) {
@@ -782,11 +873,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 ? tile_m0<PAIR>(a, segment_j(a, it_begin, it_end, seg_order(o + 1, nseg)).tile) : -1;
             if (t == 0 && o < 4) TL(2 + 2 * o);
             if (warp < NTEX)
-                produce_segment<true, STAGES, NTEX, PAIR>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
-                                                    t, sub, lane, next_m0);
+                produce_segment<true, STAGES, NTEX, PAIR, F32>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty,
+                                                               full_a, t, sub, lane, next_m0);
             else
-                produce_segment<false, STAGES, NTEX, PAIR>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty, full_a,
-                                                     t, sub, lane, next_m0);
+                produce_segment<false, STAGES, NTEX, PAIR, F32>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty,
+                                                                full_a, t, sub, lane, next_m0);
             if (t == 0 && o < 4) TL(3 + 2 * o);
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
@@ -804,9 +895,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (t == 0) TL(12);
             // idle pipeline buffers: A stages hold the per-warp store scratch, B stages the
             // staged stream-K partials
-            epilogue_segment<BLOCK_N, SLICE, PAIR>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT, t == 0,
-                                             fix_flag + 1, T, nct, a.bias_in_smem ? bias_s : nullptr,
-                                             sA + warp * EPI_SCRATCH_PER_WARP, sB,
+            epilogue_segment<BLOCK_N, SLICE, PAIR, F32>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT,
+                                                  t == 0, fix_flag + 1, T, nct, a.bias_in_smem ? bias_s : nullptr,
+                                                  sA + warp * EPI_W, sB,
                                              (size_t)STAGES * Cfg::B_STAGE_BYTES, t);
             if (t == 0) TL(13);
         }
@@ -820,9 +911,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             mbar_wait(&tmem_full[buf], (uint32_t)(o / Cfg::NBUF) & 1u);
             tc_fence_after();
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
-            epilogue_segment<BLOCK_N, BLOCK_N, PAIR>(a, &ymap, sg, tacc, r, 0, 2, 128, threadIdx.x == EPI_WARP0 * 32,
-                                               fix_flag, T, nct, a.bias_in_smem ? bias_s : nullptr,
-                                               epi_scratch + (warp - EPI_WARP0) * EPI_SCRATCH_PER_WARP);
+            epilogue_segment<BLOCK_N, BLOCK_N, PAIR, F32>(a, &ymap, sg, tacc, r, 0, 2, 128,
+                                                    threadIdx.x == EPI_WARP0 * 32, fix_flag, T, nct,
+                                                    a.bias_in_smem ? bias_s : nullptr,
+                                                    epi_scratch + (warp - EPI_WARP0) * EPI_W);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) {
@@ -846,7 +938,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     mbar_arrive(&full_b[s]);
                     (void)n0;
 #else
-                    const int kd = tap * a.Cin + chunk * BK;
+                    const int kd = tap * a.Cin + chunk * Elem<F32>::CPI;
                     if (PAIR) {   // this CTA's half of B; both halves complete on rank 0's barrier
                         if (rank == 0) mbar_arrive_expect_tx(&full_b[s], 2 * Cfg::B_STAGE_BYTES);
                         tma_load_2d_pair(sB + s * Cfg::B_STAGE_BYTES, &wmap, &full_b[s], kd,
@@ -854,9 +946,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     } else {
                         mbar_arrive_expect_tx(&full_b[s], Cfg::B_STAGE_BYTES);
 #pragma unroll
-                        for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h)
+                        for (int h = 0; h < BLOCK_N / Cfg::TMA_BOX_N; ++h) {
                             tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + h * Cfg::TMA_BOX_N * 128, &wmap,
                                         &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+                            if (F32)   // the W lo plane behind the hi plane
+                                tma_load_2d(sB + s * Cfg::B_STAGE_BYTES + Cfg::B_PLANE + h * Cfg::TMA_BOX_N * 128,
+                                            &wmap_lo, &full_b[s], kd, n0 + h * Cfg::TMA_BOX_N);
+                        }
                     }
 #endif
                     if (++tap == a.KK) { tap = 0; ++chunk; }
@@ -866,7 +962,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     } else {
         // ===================== MMA issuer (pair: rank 0 only) =====================
         if (lane == 0 && (!PAIR || rank == 0)) {
-            constexpr uint32_t idesc = make_idesc(1u /*BF16*/, PAIR ? 2 * BM : BM, Cfg::UMMA_N);
+            constexpr uint32_t idesc = make_idesc(F32 ? 2u /*TF32*/ : 1u /*BF16*/, PAIR ? 2 * BM : BM, Cfg::UMMA_N);
             int q = 0;
             for (int o = 0; o < nseg; ++o) {
                 const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
@@ -889,21 +985,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         KT(5, q);
                     }
                     tc_fence_after();
-                    const uint32_t a_addr = smem_u32(sA + s * A_STAGE_BYTES);
+                    const uint32_t a_addr = smem_u32(sA + s * Cfg::A_STAGE_BYTES);
                     const uint32_t b_addr = smem_u32(sB + s * Cfg::B_STAGE_BYTES);
 #pragma unroll
-                    for (int kk = 0; kk < BK / 16; ++kk) {
+                    for (int kk = 0; kk < 4; ++kk) {   // 4 K steps of 32 bytes per 128-byte row
                         const uint64_t adesc = make_sw128_desc(a_addr + kk * 32);
 #pragma unroll
                         for (int h = 0; h < Cfg::N_MMA; ++h) {
                             const uint64_t bdesc =
                                 make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
-                            if (PAIR)
-                                mma_bf16_ss_pair(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
-                                                 (kt != sg.kb || kk != 0) ? 1u : 0u);
-                            else
-                                mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc,
-                                            (kt != sg.kb || kk != 0) ? 1u : 0u);
+                            const uint32_t acc = (kt != sg.kb || kk != 0) ? 1u : 0u;
+                            if (F32) {   // 3xTF32: lo*hi + hi*lo + hi*hi
+                                const uint64_t adesc_lo = make_sw128_desc(a_addr + A_PLANE + kk * 32);
+                                const uint64_t bdesc_lo =
+                                    make_sw128_desc(b_addr + Cfg::B_PLANE + h * Cfg::UMMA_N * 128 + kk * 32);
+                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc_lo, bdesc, idesc, acc);
+                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc_lo, idesc, 1u);
+                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, 1u);
+                            } else if (PAIR) {
+                                mma_bf16_ss_pair(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, acc);
+                            } else {
+                                mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, acc);
+                            }
                         }
                     }
                     if (PAIR) mma_commit_pair(&empty[s], 0x3);
@@ -957,12 +1060,12 @@ struct Plan {
 static int g_pair_units = 0;
 
 template <int BLOCK_N>
-Plan<BLOCK_N> make_plan(const DcnGeom& g, bool pair = false) {
+Plan<BLOCK_N> make_plan(const DcnGeom& g, bool pair = false, int cpi = BK) {
     Plan<BLOCK_N> p;
     const int rows = pair ? 2 * BM : BM;
     p.n_tiles_n = (g.Cout + BLOCK_N - 1) / BLOCK_N;
     p.n_tiles = ((g.M + rows - 1) / rows) * p.n_tiles_n;
-    p.ipt = (g.Cin / BK) * g.KK;
+    p.ipt = (g.Cin / cpi) * g.KK;
     p.total = (long long)p.n_tiles * p.ipt;
     // At least 4 k-iterations per CTA (pair); DEFCON_MAX_CTAS caps the grid (tests use it to
     // force long persistent ranges and many whole tiles per CTA).
@@ -998,6 +1101,29 @@ size_t workspace_impl(const DcnGeom& g) {
     return partials_region() + make_plan<BLOCK_N>(g, false).counters_bytes;
 }
 
+// fp32 path: W's tf32 hi / lo planes ([Cout][Kd] fp32 each) sit INSIDE the partial region,
+// behind the partial tiles of the fp32 plan (BLOCK_N <= 128 needs a quarter of the region), so
+// the counters keep their shape-independent offset and no plane ever lands on a counter.
+size_t w_split_offset(size_t partial_bytes) { return (partial_bytes + 1023) & ~size_t(1023); }
+size_t w_split_bytes(const DcnGeom& g) { return 2 * (size_t)g.Cout * g.KK * g.Cin * sizeof(float); }
+
+// W -> tf32 hi plane (low 13 mantissa bits cleared) and lo plane (w - hi), both exact.
+__global__ void __launch_bounds__(256) dcn_w_split_kernel(const float* __restrict__ w, float* __restrict__ whi,
+                                                          float* __restrict__ wlo, long n) {
+    griddep_wait();   // the previous launch may still read the planes of this workspace
+    griddep_launch_dependents();
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n / 4; i += (long)gridDim.x * blockDim.x) {
+        const float4 v = __ldg(reinterpret_cast<const float4*>(w) + i);
+        float4 h, l;
+        h.x = __uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u); l.x = v.x - h.x;
+        h.y = __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u); l.y = v.y - h.y;
+        h.z = __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u); l.z = v.z - h.z;
+        h.w = __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u); l.w = v.w - h.w;
+        reinterpret_cast<float4*>(whi)[i] = h;
+        reinterpret_cast<float4*>(wlo)[i] = l;
+    }
+}
+
 #ifndef DEFCON_PAIR_DEFAULT
 #define DEFCON_PAIR_DEFAULT 0
 #endif
@@ -1008,12 +1134,14 @@ bool use_pair(const DcnGeom& g, const TexPlan* tex) {
     return DEFCON_PAIR_DEFAULT != 0;
 }
 
-template <int BLOCK_N, int STAGES, bool PAIR = false>
+template <int BLOCK_N, int STAGES, bool PAIR = false, bool F32 = false>
 cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
                         const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
-    using Cfg = TcCfg<BLOCK_N, PAIR>;
+    using Cfg = TcCfg<BLOCK_N, PAIR, F32>;
+    using E = Elem<F32>;
+    constexpr int EPI_W = epi_scratch_per_warp<F32>();
     if (PAIR && g_pair_units == 0) {   // how many pairs fit at once (one CTA per SM)
-        auto kp = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR>;
+        auto kp = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>;
         const size_t smem_q = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
                               (size_t)BM * g.KK * META_ENTRY + bias_smem_offset(STAGES, Cfg::NBUF) +
                               (size_t)BIAS_SMEM_MAX * 4;
@@ -1036,9 +1164,10 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
         g_pair_units = std::min(nclusters, num_sms() / 2);
         if (getenv("DEFCON_DEBUG")) fprintf(stderr, "defcon: %d co-resident 2-CTA clusters\n", nclusters);
     }
-    auto plan = make_plan<BLOCK_N>(g, PAIR);
+    auto plan = make_plan<BLOCK_N>(g, PAIR, E::CPI);
+    const size_t wsplit_off = w_split_offset(plan.partial_bytes);
     if (ws_bytes < partials_region() + plan.counters_bytes || ws == nullptr ||
-        plan.partial_bytes > partials_region()) {
+        plan.partial_bytes > partials_region() || (F32 && wsplit_off + w_split_bytes(g) > partials_region())) {
         *detail = "workspace too small for the stream-K partials and counters";
         return cudaErrorInvalidValue;
     }
@@ -1048,37 +1177,59 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
         return cudaErrorNotSupported;
     }
     const int Kd = g.KK * g.Cin;
-    CUtensorMap wmap;
+    const auto dt = F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
+    // W: bf16 as given, or (fp32) its tf32 hi / lo planes split into the workspace first
+    void* w_hi = const_cast<void*>(p.weight);
+    void* w_lo = w_hi;
+    if (F32) {
+        w_hi = static_cast<uint8_t*>(ws) + wsplit_off;
+        w_lo = static_cast<float*>(w_hi) + (size_t)g.Cout * Kd;
+        const long n = (long)g.Cout * Kd;   // a multiple of 4 (Cin % 32 == 0)
+        const unsigned nb = (unsigned)std::min<long>((n / 4 + 255) / 256, 4L * num_sms());
+        cudaError_t es = launch_pdl(dcn_w_split_kernel, dim3(nb), dim3(256), 0, stream,
+                                    static_cast<const float*>(p.weight), static_cast<float*>(w_hi),
+                                    static_cast<float*>(w_lo), n);
+        if (es != cudaSuccess) {
+            *detail = "dcn_w_split_kernel launch failed";
+            return es;
+        }
+    }
+    CUtensorMap wmap, wmap_lo;
     cuuint64_t dims[2] = {(cuuint64_t)Kd, (cuuint64_t)g.Cout};
-    cuuint64_t strides[1] = {(cuuint64_t)Kd * 2};
-    cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)Cfg::TMA_BOX_N};
+    cuuint64_t strides[1] = {(cuuint64_t)Kd * E::ES};
+    cuuint32_t box[2] = {(cuuint32_t)E::CPI, (cuuint32_t)Cfg::TMA_BOX_N};
     cuuint32_t estr[2] = {1, 1};
-    CUresult cr = encode(&wmap, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(p.weight),
-                         dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+    CUresult cr = encode(&wmap, dt, 2, w_hi, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                          CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (cr == CUDA_SUCCESS)
+        cr = encode(&wmap_lo, dt, 2, w_lo, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                    CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (cr != CUDA_SUCCESS) {
         *detail = "cuTensorMapEncodeTiled failed for the weight tensor";
         return cudaErrorInvalidValue;
     }
-    // y [M][Cout] bf16, stored by the epilogue in 32 x 32 boxes (64-byte swizzle)
+    // y [M][Cout], stored by the epilogue in 32 x 32 boxes (bf16: 64-byte swizzle; fp32: 128-byte)
     CUtensorMap ymap;
     cuuint64_t ydims[2] = {(cuuint64_t)g.Cout, (cuuint64_t)g.M};
-    cuuint64_t ystrides[1] = {(cuuint64_t)g.Cout * 2};
+    cuuint64_t ystrides[1] = {(cuuint64_t)g.Cout * E::ES};
     cuuint32_t ybox[2] = {(cuuint32_t)CS, 32u};
-    cr = encode(&ymap, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, p.y, ydims, ystrides, ybox, estr,
-                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+    cr = encode(&ymap, dt, 2, p.y, ydims, ystrides, ybox, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                F32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (cr != CUDA_SUCCESS) {
         *detail = "cuTensorMapEncodeTiled failed for the output tensor";
         return cudaErrorInvalidValue;
     }
     TcArgs a;
-    a.x = static_cast<const __nv_bfloat16*>(p.x);
+    a.x = p.x;
     a.offset = p.offset;
     a.mask = p.mask;
     a.bias = p.bias;
-    a.y = static_cast<__nv_bfloat16*>(p.y);
+    a.y = p.y;
+    a.es = E::ES;
+    a.cpi = E::CPI;
     a.partials = static_cast<float*>(ws);
     a.counters = reinterpret_cast<int*>(static_cast<uint8_t*>(ws) + partials_region());
     a.H = g.H; a.W = g.W; a.Cin = g.Cin; a.Cout = g.Cout; a.Kw = g.Kw; a.Ho = g.Ho; a.Wo = g.Wo;
@@ -1093,13 +1244,13 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.pair = PAIR ? 1 : 0;
     // Stream-K tile counters are NOT reset here: the workspace is zero-filled once by its
     // owner and every launch leaves it zeroed (the finisher of each split tile resets it).
-    const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
-                        (size_t)BM * g.KK * META_ENTRY +
+    const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_W + (size_t)BM * g.KK * META_ENTRY +
                         bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0);
-    auto kern = PAIR ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR>
-                : !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false>
-                : hybrid ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW / 2, false>
-                         : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW, false>;
+    auto kern = F32 ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false, F32>
+                : PAIR ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>
+                : !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false, false>
+                : hybrid ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW / 2, false, false>
+                         : dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, NPW, false, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) {
         *detail = "cudaFuncSetAttribute(MaxDynamicSharedMemorySize) failed";
@@ -1121,9 +1272,9 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
         attr[1].val.programmaticStreamSerializationAllowed = 1;
         cfg.attrs = attr;
         cfg.numAttrs = 2;
-        e = cudaLaunchKernelEx(&cfg, kern, wmap, ymap, a);
+        e = cudaLaunchKernelEx(&cfg, kern, wmap, wmap_lo, ymap, a);
     } else {
-        e = launch_pdl(kern, dim3(plan.grid), dim3(NUM_THREADS), smem, stream, wmap, ymap, a);
+        e = launch_pdl(kern, dim3(plan.grid), dim3(NUM_THREADS), smem, stream, wmap, wmap_lo, ymap, a);
     }
     if (e != cudaSuccess) *detail = "dcn_fwd_bf16_tc_kernel launch failed";
     return e;
@@ -1183,6 +1334,36 @@ cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, siz
         return launch_impl<256, DEFCON_STAGES_PAIR, true>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     if (g.Cout <= 256) return launch_impl<256, DEFCON_STAGES_256>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+}
+
+// ---- fp32 on the tensor cores (DEFCON_FP32_3XTF32): same kernel, kind::tf32 with the 3xTF32
+// split, 32 channels per k-iteration, N tiles of <= 128 columns (the B stage holds two planes).
+template <int BLOCK_N>
+static bool f32_planes_fit(const DcnGeom& g) {
+    return w_split_offset(make_plan<BLOCK_N>(g, false, 32).partial_bytes) + w_split_bytes(g) <= partials_region();
+}
+
+bool dcn_tc_f32_supported(const DcnGeom& g) {
+    if (g.Cin % 32 != 0 || g.Cg % 32 != 0) return false;
+    if (g.Cout % 16 != 0) return false;
+    if ((long)BM * g.KK * META_ENTRY > 48 * 1024) return false;
+    return g.Cout <= 64 ? f32_planes_fit<64>(g) : f32_planes_fit<128>(g);   // Cout * Kd up to ~7M
+}
+
+size_t dcn_tc_f32_workspace(const DcnGeom& g) {
+    return partials_region() + (g.Cout <= 64 ? make_plan<64>(g, false, 32).counters_bytes
+                                              : make_plan<128>(g, false, 32).counters_bytes);
+}
+
+void dcn_tc_f32_workspace_counters(const DcnGeom& g, size_t* offset, size_t* bytes) {
+    *offset = partials_region();
+    *bytes = g.Cout <= 64 ? make_plan<64>(g, false, 32).counters_bytes : make_plan<128>(g, false, 32).counters_bytes;
+}
+
+cudaError_t launch_dcn_tc_f32(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes, cudaStream_t stream,
+                              const char** detail) {
+    if (g.Cout <= 64) return launch_impl<64, 3, false, true>(g, p, ws, ws_bytes, nullptr, false, stream, detail);
+    return launch_impl<128, 2, false, true>(g, p, ws, ws_bytes, nullptr, false, stream, detail);
 }
 
 }  // namespace defcon

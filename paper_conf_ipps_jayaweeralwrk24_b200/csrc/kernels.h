@@ -79,6 +79,13 @@ struct TexPlan;
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
                                const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail);
 
+// ---- step 2 on the tensor cores in fp32: kind::tf32 3xTF32 (same fused kernel, dcn_tc_bf16.cu)
+bool dcn_tc_f32_supported(const DcnGeom& g);
+size_t dcn_tc_f32_workspace(const DcnGeom& g);   // partials + counters + W's tf32 hi / lo planes
+void dcn_tc_f32_workspace_counters(const DcnGeom& g, size_t* offset, size_t* bytes);
+cudaError_t launch_dcn_tc_f32(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes, cudaStream_t stream,
+                              const char** detail);
+
 // ---- texture sampler resources (tex_plan.cu)
 struct TexPlan;
 cudaError_t tex_plan_create(int N, int H, int W, int C, bool half, TexPlan** out);

@@ -115,6 +115,11 @@ def test_workspace_size_and_layer_size(lib):
     # fp32 CUDA-core path needs none
     assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(), 0, 0, 1, ctypes.byref(out)) == 0
     assert out.value == 0
+    # fp32 on the tensor cores (3xTF32): counters + partials (W's tf32 planes inside them)
+    assert lib.defcon_dcn_workspace_size(2, 8, 8, 64, 64, 3, 3, _conv(), 0, 0, 0, ctypes.byref(out)) == 0
+    assert out.value > 0
+    # ... which needs Cin/G % 32 == 0 (one 128-byte fp32 row per k-iteration)
+    assert lib.defcon_dcn_workspace_size(2, 8, 8, 48, 64, 3, 3, _conv(), 0, 0, 0, ctypes.byref(out)) == 2
     assert lib.defcon_layer_workspace_size(2, 8, 8, 64, 1, 64, 3, _conv(), 1, 0, 1, ctypes.byref(out)) == 0
     # x (2*8*8*64*2) + offsets + mask + y, each 256-aligned
     assert out.value >= 2 * 8 * 8 * 64 * 2 * 2 + 2 * 64 * 9 * 3 * 4

@@ -245,6 +245,76 @@ def test_dcn_pair_full_size_sampled(oracle_mod, d, dev, monkeypatch, c):
     assert ulp_close(y2, y1, np.max(np.abs(ref)))
 
 
+# fp32 on the tensor cores (DEFCON_FP32_3XTF32): kind::tf32 with the 3xTF32 split.  Dropping
+# lo*lo and truncating the lo parts to tf32 leaves ~2^-20 relative per product, so the fp32
+# gates (1e-4 contract, 1e-5 regression) hold as for the CUDA-core fp32 kernels.
+F32TC = [
+    small("tf32x3_cout64", dtype="f32", Cin=64, Cout=64),                 # BLOCK_N 64, 3 stages
+    small("tf32x3_cout128_g2", dtype="f32", Cin=64, Cout=128, G=2),       # Cg = 32
+    small("tf32x3_cout48_v1", dtype="f32", Cin=32, Cout=48, modulated=False),   # N tile not full
+    small("tf32x3_cout256_s2", dtype="f32", Cin=64, Cout=256, stride=2, H=23, W=21),   # 2 N tiles
+    small("tf32x3_cout272_dil2", dtype="f32", Cin=32, Cout=272, dil=2, pad=2, H=11, W=9),  # ragged N
+    small("tf32x3_k1", dtype="f32", Cin=96, Cout=80, K=1, pad=0),
+    small("tf32x3_g4", dtype="f32", Cin=128, Cout=32, G=4),                # 4 offset groups, Cg = 32
+]
+
+
+@pytest.mark.parametrize("c", F32TC, ids=lambda c: c.name)
+def test_dcn_3xtf32_parity(oracle_mod, d, dev, c):
+    L = inputs.gen_layer(c)
+    y = run_dcn(d, dev, c, L, fp32_mode="3xtf32")
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
+                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    err = normwise(y, ref)
+    print(f"{c.name}: normwise error {err:.3e}")
+    assert err < REG["f32"], err
+
+
+@pytest.mark.parametrize("c", [configs.C4_F32, configs.C4_G4_F32], ids=lambda c: c.name)
+def test_dcn_3xtf32_full_size_sampled(oracle_mod, d, dev, c):
+    """The 3xTF32 tensor-core path at the BASELINE.json fp32 configs (C4, C4 G=4), sampled."""
+    L = inputs.gen_layer(c)
+    y = run_dcn(d, dev, c, L, fp32_mode="3xtf32").reshape(c.M, c.Cout)
+    r = np.random.default_rng(7)
+    idx = np.unique(np.concatenate([np.arange(0, 130), np.arange(c.M - 130, c.M), r.integers(0, c.M, 300)]))
+    ref = oracle_mod.dcn_pixels(L["x"], L["offset"], L["weight"], idx, L["bias"], mask=L["mask"],
+                                stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    err = normwise(y[idx], ref)
+    print(f"{c.name} 3xtf32: normwise error {err:.3e}")
+    assert err < REG["f32"], err
+
+
+def test_dcn_3xtf32_stream_k_and_workspace_reuse(oracle_mod, d, dev, monkeypatch):
+    """Forced stream-K splits (DEFCON_MAX_CTAS) on the 3xTF32 path, and one zero-filled
+    workspace shared by a bf16 and an fp32 call of different shapes (the W planes live in the
+    partial region, never on a counter)."""
+    c = small("tf32x3_sk", dtype="f32", Cin=64, Cout=128)
+    cb = small("bf16_sk", Cin=64, Cout=256, H=37, W=29)
+    L, Lb = inputs.gen_layer(c), inputs.gen_layer(cb)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
+    nb = d.defcon_dcn_workspace_size(cb.N, cb.H, cb.W, cb.Cin, cb.Cout, 3, 3, 1, 1, 1, 1, torch.bfloat16)
+    nf = d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, 3, 3, 1, 1, 1, 1, torch.float32,
+                                     fp32_mode="3xtf32")
+    ws = torch.zeros(max(nb, nf), dtype=torch.uint8, device=dev)
+    # counters start at the device-wide partial-region size: nb minus the bf16 shape's counters
+    ctr_bytes = -(-max(-(-cb.M // 128), 2 * -(-cb.M // 256)) * 4 // 256) * 256
+    ctrs = ws[nb - ctr_bytes:]
+    for ctas in (7, 64):
+        monkeypatch.setenv("DEFCON_MAX_CTAS", str(ctas))
+        for _ in range(2):
+            yb = d.defcon_dcn_forward(to_dev(Lb["x"], torch.bfloat16, dev), to_dev(Lb["offset"], torch.float32, dev),
+                                      to_dev(Lb["mask"], torch.float32, dev), to_dev(Lb["weight"], torch.bfloat16, dev),
+                                      to_dev(Lb["bias"], torch.float32, dev), workspace=ws)
+            y = d.defcon_dcn_forward(to_dev(L["x"], torch.float32, dev), to_dev(L["offset"], torch.float32, dev),
+                                     to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], torch.float32, dev),
+                                     to_dev(L["bias"], torch.float32, dev), fp32_mode="3xtf32", workspace=ws)
+            torch.cuda.synchronize()
+            assert normwise(y.cpu().numpy(), ref) < REG["f32"]
+    refb = oracle_mod.dcn_forward(Lb["x"], Lb["offset"], Lb["weight"], Lb["bias"], mask=Lb["mask"])
+    assert normwise(yb.float().cpu().numpy(), refb) < REG["bf16"]
+    assert int(ctrs.count_nonzero()) == 0
+
+
 def test_dcn_deterministic(d, dev):
     c = small("det")
     L = inputs.gen_layer(c)

@@ -16,6 +16,9 @@ import paper_conf_ipps_jayaweeralwrk24_b200 as d  # noqa: E402
 
 
 def time_cfg(c, sampler, reps=200):
+    """sampler: ldg / tex / hybrid, or (fp32 configs) the fp32 mode simt / 3xtf32."""
+    fp32_mode = sampler if sampler in ("simt", "3xtf32") else "simt"
+    sampler = "ldg" if sampler in ("simt", "3xtf32") else sampler
     dev = torch.device("cuda")
     L = inputs.gen_layer(c)
     dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
@@ -26,12 +29,13 @@ def time_cfg(c, sampler, reps=200):
     b = torch.from_numpy(L["bias"]).to(dev)
     y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
     ws = torch.zeros(max(16, d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K,
-                                                         c.stride, c.pad, c.dil, c.G, dt, sampler)),
+                                                         c.stride, c.pad, c.dil, c.G, dt, sampler,
+                                                         fp32_mode)),
                      dtype=torch.uint8, device=dev)
     plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler in ("tex", "hybrid") else None
     fn = lambda: d.defcon_dcn_forward(x, off, msk, w, b, stride=c.stride, pad=c.pad, dil=c.dil,
                                       offset_groups=c.G, y=y, workspace=ws, sampler=sampler,
-                                      tex_plan=plan)
+                                      tex_plan=plan, fp32_mode=fp32_mode)
     for _ in range(5):
         fn()
     g = torch.cuda.CUDAGraph()
