@@ -1,16 +1,22 @@
 #!/usr/bin/env python3
 """DEFCON hot-path benchmark on B200 (contract: one JSON line from rank 0).
 
-Workload (BASELINE.json configs[2], the north-star target): YOLACT++ ResNet-101 C4 DCNv2
-3x3 layer, N=16 images per GPU, C=256, 35x35, offset_groups=1, bf16 storage, fed by the
-paper's lightweight depthwise offset branch.  One "step" = one pass of the
-whole hot path over one batch: defcon_offset_dw_conv (step 1) + defcon_dcn_forward (step 2).
+Default workload (BASELINE.json configs[2], the north-star target): YOLACT++ ResNet-101 C4
+DCNv2 3x3 layer, N=16 images per GPU, C=256, 35x35, offset_groups=1, bf16 storage, fed by the
+paper's lightweight depthwise offset branch.  One "step" = one pass of the whole
+hot path over one batch: defcon_offset_dw_conv (step 1) + defcon_dcn_forward (step 2).
+
+--workload picks another BASELINE.json config: c3, c4_g4, c5 (bf16), c4_f32 / c4_g4_f32 (fp32 on
+the tensor cores, 3xTF32), c4_f32_simt (the CUDA-core fp32 anchor), or stack -- config 5, the
+11-layer interval-placed DCN stack of YOLACT++ R101 C3-C5 at a GLOBAL batch of 64 images
+sharded over the GPUs (strong scaling: 64/N images per GPU); a step is then the whole stack.
 
 metric: contraction TFLOP/s (2*M*Cout*K^2*Cin per layer), higher is better;
-ms_per_step gives the layer latency.  value = FLOPs of all ranks / max-over-ranks time.
+ms_per_step gives the layer (stack) latency.  value = FLOPs of all ranks / max-over-ranks time.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
-Multi-GPU: launched by torchrun (one rank per GPU, NCCL, weak scaling by image).
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl reference]
+Multi-GPU: launched by torchrun (one rank per GPU, NCCL, images sharded, no data-path
+collective).
 """
 from __future__ import annotations
 
@@ -31,17 +37,49 @@ sys.path.insert(0, ROOT)
 
 from defcon_workloads import configs, inputs, sharding  # noqa: E402
 
-WORKLOAD = configs.C4
+# name -> (layers at the per-GPU batch of a 1-GPU run, fp32 mode, strong scaling)
+WORKLOADS = {
+    "c4": ([configs.C4], "simt", False),
+    "c3": ([configs.C3], "simt", False),
+    "c4_g4": ([configs.C4_G4], "simt", False),
+    "c5": ([configs.C5], "simt", False),
+    "c4_f32": ([configs.C4_F32], "3xtf32", False),
+    "c4_g4_f32": ([configs.C4_G4_F32], "3xtf32", False),
+    "c4_f32_simt": ([configs.C4_F32], "simt", False),
+    "stack": (configs.stack_layers(64), "simt", True),
+}
+STACK_GLOBAL_BATCH = 64
 L2_BYTES = 126 * 2**20
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 NCU_SUMMARY_GLOB = os.path.join(ROOT, "profiles", "r*_ncu_summary.json")
 
 
-def metric_name():
-    return "DCNv2 layer TFLOP/s (contraction) at YOLACT++ C4 shape, incl. offset branch"
+def metric_name(name="c4"):
+    if name == "stack":
+        return ("DEFCON interval-placed DCN stack (11 DCNv2 layers, YOLACT++ R101 C3-C5) TFLOP/s "
+                "(contraction) at global batch 64, incl. offset branches")
+    c = WORKLOADS[name][0][0]
+    shape = {"yolact_r101_c3_v2": "C3", "yolact_r101_c4_v2": "C4", "yolact_r101_c4_v2_g4": "C4 G=4",
+             "yolact_r101_c5_v2": "C5", "yolact_r101_c4_v2_f32": "C4 fp32",
+             "yolact_r101_c4_v2_g4_f32": "C4 G=4 fp32"}[c.name]
+    return f"DCNv2 layer TFLOP/s (contraction) at YOLACT++ {shape} shape, incl. offset branch"
 
 
-def workload_config(c, world, extra=None):
+def workload_config(c, world, extra=None, name="c4", per_rank=None):
+    if name == "stack":
+        d = {
+            "workload": "stack: config 5, DEFCON interval-3 DCNv2 stack of R101 C3-C5 (11 layers: "
+                        + ", ".join(f"{l.name} {l.H}x{l.W}x{l.Cin}->{l.Ho}x{l.Wo}x{l.Cout} s{l.stride}"
+                                    for l in configs.stack_layers(1))
+                        + "), bf16, each layer fed by its lightweight offset branch",
+            "global_batch": STACK_GLOBAL_BATCH,
+            "per_gpu_batch": per_rank,
+            "parallelism": f"dp{world} (global batch 64 split by image, strong scaling, no data-path "
+                           "collective)",
+        }
+        if extra:
+            d.update(extra)
+        return d
     d = {
         "workload": f"{c.name}: N={c.N}/GPU Cin=Cout={c.Cin} {c.H}x{c.W} K={c.K} stride={c.stride} "
                     f"G={c.G} DCNv2 {c.dtype} + lightweight offset branch (dw3x3+BN+ReLU+1x1)",
@@ -123,10 +161,13 @@ class ClockSampler:
 
 # ------------------------------------------------------------------ GPU arm
 class Layer:
-    """Device-resident inputs/outputs of one buffer set (one batch of the workload)."""
+    """Device-resident inputs/outputs of one layer's buffer set (one batch of the workload)."""
 
-    def __init__(self, c, images, dev, branch_dev, weight, bias):
+    def __init__(self, c, images, dev, branch_dev, weight, bias, fp32_mode):
+        import paper_conf_ipps_jayaweeralwrk24_b200 as d
         dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
+        self.c = c
+        self.fp32_mode = fp32_mode
         self.x = torch.from_numpy(inputs.gen_x(c, images)).to(dev, dt)
         KK = c.K * c.K
         self.off = torch.empty((c.N, c.Ho, c.Wo, c.G, KK, 2), device=dev, dtype=torch.float32)
@@ -135,9 +176,8 @@ class Layer:
         self.branch = branch_dev
         self.weight = weight
         self.bias = bias
-        import paper_conf_ipps_jayaweeralwrk24_b200 as d
         nws = d.defcon_dcn_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, c.K, c.K, c.stride, c.pad,
-                                          c.dil, c.G, dt)
+                                          c.dil, c.G, dt, fp32_mode=fp32_mode)
         self.ws = torch.zeros(max(nws, 16), dtype=torch.uint8, device=dev)   # zero before first use
         self.tws = torch.empty(d.defcon_offset_workspace_size(c.N, c.H, c.W, c.Cin, c.K, c.stride,
                                                               c.pad, c.dil, c.G),
@@ -148,16 +188,17 @@ class Layer:
                                                            self.weight))
 
 
-def step1(d, c, L):
-    B = L.branch
+def step1(d, L):
+    c, B = L.c, L.branch
     d.defcon_offset_dw_conv(L.x, B["dw_w"], B["dw_scale"], B["dw_shift"], B["pw_w"], B["pw_b"],
                             K=c.K, stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
                             with_mask=c.modulated, offset=L.off, mask=L.msk, workspace=L.tws)
 
 
-def step2(d, c, L):
+def step2(d, L):
+    c = L.c
     d.defcon_dcn_forward(L.x, L.off, L.msk, L.weight, L.bias, stride=c.stride, pad=c.pad,
-                         dil=c.dil, offset_groups=c.G, y=L.y, workspace=L.ws)
+                         dil=c.dil, offset_groups=c.G, y=L.y, workspace=L.ws, fp32_mode=L.fp32_mode)
 
 
 def capture(fn, stream):
@@ -167,39 +208,59 @@ def capture(fn, stream):
     return g
 
 
+def launches_per_layer(c, fp32_mode):
+    """Kernels one layer launches: the offset branch (weight-pack + one-pass kernel, or the
+    two-pass dw + 1x1 kernels: 2 either way) + the DCN kernel (+ the W tf32 split for 3xTF32)."""
+    return 2 + 1 + (1 if c.dtype == "f32" and fp32_mode == "3xtf32" else 0)
+
+
 def gpu_arm(args, rank, world, local_rank, dist):
     import paper_conf_ipps_jayaweeralwrk24_b200 as d
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     d.load_library()
-    c = WORKLOAD
-    # per-rank images: weak scaling, each rank regenerates exactly its own shard
-    images = sharding.shard_images(rank, world, c.N)
-    P = inputs.gen_offset_branch(c)
-    w, b = inputs.gen_weight(c)
-    dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
+    base_layers, fp32_mode, strong = WORKLOADS[args.workload]
+    if strong:   # config 5: global batch 64 split over the ranks
+        images = sharding.shard_strong(rank, world, STACK_GLOBAL_BATCH)
+    else:        # weak scaling: each rank regenerates exactly its own shard of N images
+        images = sharding.shard_images(rank, world, base_layers[0].N)
+    layers = [l.replace(N=len(images)) for l in base_layers]
+    c0 = layers[0]
+
+    def make_set():
+        out = []
+        for c in layers:
+            dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
+            P = {k: torch.from_numpy(v).to(dev) for k, v in inputs.gen_offset_branch(c).items()}
+            w, b = inputs.gen_weight(c)
+            out.append(Layer(c, images, dev, P, torch.from_numpy(w).to(dev, dt), torch.from_numpy(b).to(dev),
+                             fp32_mode))
+        return out
 
     # Rotate buffer sets so the sets touched between two visits exceed L2 (cold-L2 timing).
-    probe_bytes = (c.N * c.H * c.W * c.Cin * 2 + c.M * c.Cout * 2 + c.M * 27 * 4 +
-                   c.Cout * 9 * c.Cin * 2)
-    R = max(2, int(np.ceil(1.5 * L2_BYTES / probe_bytes)))
-    sets = []
-    for r in range(R):
-        Pd = {k: torch.from_numpy(v).to(dev) for k, v in P.items()}
-        sets.append(Layer(c, images, dev, Pd, torch.from_numpy(w).to(dev, dt),
-                          torch.from_numpy(b).to(dev)))
-    rot_bytes = sum(L.nbytes() for L in sets)
+    sets = [make_set()]
+    set_bytes = sum(L.nbytes() for L in sets[0])
+    R = max(2, int(np.ceil(1.5 * L2_BYTES / set_bytes))) if set_bytes < 1.5 * L2_BYTES else 1
+    sets += [make_set() for _ in range(R - 1)]
+    rot_bytes = set_bytes * R
 
     stream = torch.cuda.Stream(device=dev)
     with torch.cuda.stream(stream):
-        for L in sets:          # eager warm-up outside capture (module load, attributes)
-            step1(d, c, L)
-            step2(d, c, L)
+        for S in sets:          # eager warm-up outside capture (module load, attributes)
+            for L in S:
+                step1(d, L)
+                step2(d, L)
     torch.cuda.synchronize()
-    g_step = [capture(lambda L=L: (step1(d, c, L), step2(d, c, L)), stream) for L in sets]
-    g_dcn = [capture(lambda L=L: step2(d, c, L), stream) for L in sets]
-    g_br = [capture(lambda L=L: step1(d, c, L), stream) for L in sets]
+
+    def whole(S):
+        for L in S:
+            step1(d, L)
+            step2(d, L)
+
+    g_step = [capture(lambda S=S: whole(S), stream) for S in sets]
+    g_dcn = [capture(lambda S=S: [step2(d, L) for L in S], stream) for S in sets]
+    g_br = [capture(lambda S=S: [step1(d, L) for L in S], stream) for S in sets]
     torch.cuda.synchronize()
 
     def run(graphs, n):
@@ -235,7 +296,7 @@ def gpu_arm(args, rank, world, local_rank, dist):
         t_ext = time.time()
         with torch.cuda.stream(stream):
             while time.time() - t_ext < 0.6:
-                run(g_step, 200)
+                run(g_step, 20)
                 torch.cuda.synchronize()
         t_wall1 = time.time()
 
@@ -250,43 +311,53 @@ def gpu_arm(args, rank, world, local_rank, dist):
         torch.cuda.synchronize()
         return a.elapsed_time(bq) / n
 
-    n_k = max(args.steps, 200)
+    n_k = max(args.steps, 200 // len(layers))
     ms_dcn = time_graphs(g_dcn, n_k)
     ms_branch = time_graphs(g_br, n_k)
     clk.stop()
     clocks = clk.summary(t_wall0, t_wall1)
 
-    # ---------------- end to end through the C ABI with pinned host buffers
-    ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, K=c.K,
-                                                   stride=c.stride, pad=c.pad, dil=c.dil,
-                                                   offset_groups=c.G, dtype=dt,
-                                                   modulated=c.modulated),
-                     dtype=torch.uint8, device=dev)
-    xh = sets[0].x.cpu().pin_memory()
-    yh = torch.empty(tuple(sets[0].y.shape), dtype=dt).pin_memory()
-    L0 = sets[0]
-    e2e_steps = max(3, min(args.steps, 50))
+    # ---------------- end to end through the C ABI with pinned host buffers: every layer's x
+    # from pinned host memory, its y back (defcon_layer_forward_host, one call per layer)
+    e2e_in = []
+    for L in sets[0]:
+        c = L.c
+        dt = L.x.dtype
+        ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout, K=c.K,
+                                                       stride=c.stride, pad=c.pad, dil=c.dil,
+                                                       offset_groups=c.G, dtype=dt,
+                                                       modulated=c.modulated, fp32_mode=fp32_mode),
+                         dtype=torch.uint8, device=dev)
+        e2e_in.append((L, L.x.cpu().pin_memory(), torch.empty(tuple(L.y.shape), dtype=dt).pin_memory(), ws))
+
+    def e2e_step():
+        for L, xh, yh, ws in e2e_in:
+            c = L.c
+            d.defcon_layer_forward_host(xh, L.branch, L.weight, L.bias, yh, ws, K=c.K,
+                                        stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
+                                        modulated=c.modulated, fp32_mode=fp32_mode, stream=stream)
+
+    e2e_steps = max(3, min(args.steps, 50 // len(layers)))
     with torch.cuda.stream(stream):
         for _ in range(2):
-            d.defcon_layer_forward_host(xh, L0.branch, L0.weight, L0.bias, yh, ws, K=c.K,
-                                        stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
-                                        modulated=c.modulated, stream=stream)
+            e2e_step()
         barrier()
         a, bq = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         for _ in range(e2e_steps):
-            d.defcon_layer_forward_host(xh, L0.branch, L0.weight, L0.bias, yh, ws, K=c.K,
-                                        stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G,
-                                        modulated=c.modulated, stream=stream)
+            e2e_step()
         bq.record(stream)
     torch.cuda.synchronize()
     ms_e2e = a.elapsed_time(bq) / e2e_steps
+    h2d = sum(xh.numel() * xh.element_size() for _, xh, _, _ in e2e_in)
+    d2h = sum(yh.numel() * yh.element_size() for _, _, yh, _ in e2e_in)
+    del e2e_in
 
     # ---------------- collectives outside the timed region: per-image fp64
-    # checksums of y all-gathered (invariance: an image's y does not depend on its rank), and
-    # every rank's y gathered into rank 0, timed on its own
+    # checksums of the last layer's y all-gathered (invariance: an image's y does not depend on
+    # its rank), and every rank's y gathered into rank 0, timed on its own
     with torch.cuda.stream(stream):
-        y0 = sets[0].y
+        y0 = sets[0][-1].y
         cks = sharding.gather_checksums(dist, sharding.image_checksums(y0))
         barrier()
         ga, gb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -302,21 +373,40 @@ def gpu_arm(args, rank, world, local_rank, dist):
     ms_total, ms_e2e, ms_dcn, ms_branch, ms_gather = sharding.max_over_ranks(
         dist, [ms_total, ms_e2e, ms_dcn, ms_branch, ms_gather], dev)
 
-    flops = configs.contraction_flops(c)
+    flops = sum(configs.contraction_flops(c) for c in layers)       # per rank, per step
     ms_step = ms_total / args.steps
     value = world * flops * args.steps / (ms_total * 1e-3) / 1e12
     peaks, peak_src = load_peaks()
     achieved = flops / (ms_dcn * 1e-3) / 1e12
+    f32 = c0.dtype == "f32"
+    if f32 and fp32_mode == "3xtf32":   # 3 tf32 MMAs per product; tf32 peak = bf16 peak / 2 (nominal ratio)
+        peak, peak_unit_note = peaks["bf16_tflops"] / 2 / 3, "bf16 burst / 2 (tf32) / 3 (3xTF32 products)"
+    elif f32:                           # FFMA: 148 SMs x 128 lanes x 2 flop x max SM clock
+        peak, peak_unit_note = 148 * 128 * 2 * 1.965e9 / 1e12, "fp32 FFMA (148 x 128 x 2 x 1965 MHz)"
+    else:
+        peak, peak_unit_note = peaks["bf16_tflops"], "bf16 burst"
     traffic = None
-    try:   # dram read+write bytes per launch of the DCN kernel, latest committed ncu capture
-        import glob
-        latest = sorted(glob.glob(NCU_SUMMARY_GLOB))[-1]
-        with open(latest) as f:
-            traffic = json.load(f).get("dcn_dram_bytes_per_launch")
-    except Exception:
-        pass
+    if args.workload == "c4":
+        try:   # dram read+write bytes per launch of the DCN kernel, latest committed ncu capture
+            import glob
+            latest = sorted(glob.glob(NCU_SUMMARY_GLOB))[-1]
+            with open(latest) as f:
+                js = json.load(f)
+            traffic = js.get("dcn_dram_bytes_per_launch")
+            traffic_note = js.get("dcn_dram_bytes_note")
+        except Exception:
+            traffic_note = None
+    kernel = ("dcn_fwd_bf16_tc_kernel<F32> (fused gather + tcgen05 kind::tf32 3xTF32 implicit GEMM)"
+              if f32 and fp32_mode == "3xtf32" else
+              "dcn_fwd_f32 CUDA-core kernel (FFMA)" if f32 else
+              "dcn_fwd_bf16_tc_kernel (fused gather + tcgen05 implicit GEMM)")
+    if len(layers) > 1:
+        kernel += f", summed over the {len(layers)} layers of the stack"
+    per_layer = {}
+    if len(layers) > 1:
+        per_layer = {"layers": [c.name for c in layers]}
     line = {
-        "metric": metric_name(),
+        "metric": metric_name(args.workload),
         "value": round(value, 3),
         "unit": "TFLOP/s",
         "n_gpus": world,
@@ -324,42 +414,41 @@ def gpu_arm(args, rank, world, local_rank, dist):
         "warmup": args.warmup,
         "ms_per_step": round(ms_step, 5),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong" if strong else "weak",
         "vs_baseline": None,
-        "dtype": "bf16",
-        "data": "synthetic (seeded; x=ReLU(N(0,1)) bf16, offsets from the dw offset branch, "
+        "dtype": "f32" if f32 else "bf16",
+        "data": "synthetic (seeded; x=ReLU(N(0,1)), offsets from the dw offset branch, "
                 "random-init weights)",
-        "config": workload_config(c, world, {
-            "l2": f"rotating {R} buffer sets ({rot_bytes / 2**20:.0f} MiB > 126 MiB L2), CUDA graphs",
-            "us_per_layer": round(ms_step * 1e3, 2),
-            "us_dcn_kernel": round(ms_dcn * 1e3, 2),
-            "us_offset_branch_kernel": round(ms_branch * 1e3, 2),
-        }),
+        "config": workload_config(c0, world, dict({
+            "l2": (f"rotating {R} buffer sets ({rot_bytes / 2**20:.0f} MiB > 126 MiB L2), CUDA graphs"
+                   if R > 1 else f"inputs larger than L2 ({set_bytes / 2**20:.0f} MiB per step), CUDA graphs"),
+            "us_per_step": round(ms_step * 1e3, 2),
+            "us_dcn_kernels": round(ms_dcn * 1e3, 2),
+            "us_offset_branch_kernels": round(ms_branch * 1e3, 2),
+            "fp32_mode": fp32_mode if f32 else None,
+        }, **per_layer), name=args.workload, per_rank=len(images)),
         "roofline": {
-            "kernel": "dcn_fwd_bf16_tc_kernel (fused gather + tcgen05 implicit GEMM)",
-            "bound": "tensor",
+            "kernel": kernel,
+            "bound": "tensor" if not (f32 and fp32_mode == "simt") else "alu",
             "achieved": round(achieved, 2),
-            "peak": peaks["bf16_tflops"],
-            "peak_source": f"{peak_src} bf16 burst (MEASURED_PEAKS.json)" if peak_src == "measured"
-                           else "fallback bf16 burst (B200_PROFILING.md)",
+            "peak": round(peak, 1),
+            "peak_source": (f"{peak_src} {peak_unit_note} (MEASURED_PEAKS.json)" if peak_src == "measured"
+                            else f"fallback {peak_unit_note} (B200_PROFILING.md)"),
             "unit": "TFLOP/s",
-            "frac": round(achieved / peaks["bf16_tflops"], 4),
+            "frac": round(achieved / peak, 4),
             "traffic": traffic,
-            # context: the measured sustained bf16 figure (cuBLAS back to back for 4 s)
-            "peak_sustained": peaks.get("bf16_tflops_sustained"),
-            "frac_sustained": (round(achieved / peaks["bf16_tflops_sustained"], 4)
-                               if peaks.get("bf16_tflops_sustained") else None),
         },
         "clocks": clocks,
         "e2e": {
             "value": round(world * flops / (ms_e2e * 1e-3) / 1e12, 3),
             "unit": "TFLOP/s",
-            "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
-            "d2h_bytes_per_step": int(yh.numel() * yh.element_size()),
+            "h2d_bytes_per_step": int(h2d),
+            "d2h_bytes_per_step": int(d2h),
             "ms_per_step": round(ms_e2e, 4),
-            "api": "defcon_layer_forward_host (C ABI, pinned host x -> y)",
+            "api": "defcon_layer_forward_host (C ABI, pinned host x -> y)"
+                   + (", one call per layer" if len(layers) > 1 else ""),
         },
-        "gpu_launches": 3 * args.steps,   # dw_bn_relu + 1x1 (step 1) + dcn_fwd (step 2)
+        "gpu_launches": args.steps * sum(launches_per_layer(c, fp32_mode) for c in layers),
         "collectives": {                  # outside the timed region
             "checksum_images": int(cks.shape[0]),
             "y_checksum_image0": [round(float(v), 6) for v in cks[0].tolist()],
@@ -367,45 +456,65 @@ def gpu_arm(args, rank, world, local_rank, dist):
             "y_gather_bytes": gather_bytes,
         },
     }
+    if traffic is not None:
+        line["roofline"]["traffic_note"] = traffic_note
+    if not f32:   # context: the measured sustained bf16 figure (cuBLAS back to back for 4 s)
+        line["roofline"]["peak_sustained"] = peaks.get("bf16_tflops_sustained")
+        line["roofline"]["frac_sustained"] = (round(achieved / peaks["bf16_tflops_sustained"], 4)
+                                              if peaks.get("bf16_tflops_sustained") else None)
     return line
 
 
 # ------------------------------------------------------------------ oracle (CPU) legs
-def oracle_sample(c, target_s, images=4):
-    """Time the oracle as it stands on a bounded sample of the workload: the offset branch
-    of `images` images plus the DCN at n_pix of their output pixels (calibrated so the sample
-    takes about target_s seconds); returns (TFLOP/s, seconds, description, n_pix)."""
+def oracle_sample(layers, target_s, images=4):
+    """Time the oracle as it stands on a bounded sample of the workload: for every layer, the
+    offset branch of `images` images plus the DCN at n_pix of their output pixels (n_pix
+    calibrated so the sample takes about target_s seconds); returns (TFLOP/s, seconds,
+    description, n_pix, step function)."""
     import oracle
     oracle.build()
-    ci = c.replace(N=images)
-    x = inputs.gen_x(ci, images=list(range(images)))
-    P = inputs.gen_offset_branch(c)
-    w, b = inputs.gen_weight(c)
+    prep = []
+    for c in layers:
+        ci = c.replace(N=images)
+        x = inputs.gen_x(ci, images=list(range(images)))
+        P = inputs.gen_offset_branch(c)
+        w, b = inputs.gen_weight(c)
+        prep.append((c, ci, x, P, w, b))
+
+    def step(n_pix):
+        for c, ci, x, P, w, b in prep:
+            off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
+                                            P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated,
+                                            stride=c.stride, pad=c.pad, dil=c.dil)
+            idx = np.arange(n_pix) % ci.M
+            oracle.dcn_pixels(x, off, w, idx, b, mask=msk, stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
 
     def once(n_pix):
         t0 = time.perf_counter()
-        off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
-                                        P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated,
-                                        stride=c.stride, pad=c.pad, dil=c.dil)
-        idx = np.arange(n_pix) % ci.M
-        oracle.dcn_pixels(x, off, w, idx, b, mask=msk, stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+        step(n_pix)
         return time.perf_counter() - t0
 
     t_small = once(256)
     t_big = once(2048)
     per_pix = max((t_big - t_small) / (2048 - 256), 1e-7)
     fixed = max(t_small - 256 * per_pix, 0.0)
-    n_pix = int(np.clip((target_s - fixed) / per_pix, 256, 50 * ci.M))
+    n_pix = int(np.clip((target_s - fixed) / per_pix, 256, 50 * min(l.replace(N=images).M for l in layers)))
     dt = once(n_pix)
-    flops = 2 * n_pix * c.Cout * c.K * c.K * c.Cin
-    sample = (f"{c.name}: offset branch of {images} images + DCN at {n_pix} of their output "
+    flops = sum(2 * n_pix * c.Cout * c.K * c.K * c.Cin for c in layers)
+    what = layers[0].name if len(layers) == 1 else f"each of the {len(layers)} stack layers"
+    sample = (f"{what}: offset branch of {images} image(s) + DCN at {n_pix} of their output "
               f"pixels ({flops / 1e9:.1f} GFLOP contraction), fp64 C oracle, OpenMP")
-    return flops / dt / 1e12, dt, sample, n_pix
+    return flops / dt / 1e12, dt, sample, n_pix, step, flops
 
 
-def cpu_baseline(c):
+def sample_images(name):
+    return 1 if name == "stack" else 4
+
+
+def cpu_baseline(name):
     import oracle
-    v, dt, sample, _ = oracle_sample(c, target_s=10.0)
+    layers = WORKLOADS[name][0]
+    v, dt, sample, _, _, _ = oracle_sample(layers, target_s=10.0, images=sample_images(name))
     out = {"value": v, "unit": "TFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
            "sample": sample, "seconds": round(dt, 2)}
     # SURVEY 8(d): the oracle also single-core on config 1 (the tiny DCNv1 fp32 layer)
@@ -429,33 +538,21 @@ def reference_arm(args, world):
     Each step is a bounded sample of the workload (see oracle_sample), sized so that the
     whole --steps/--warmup run finishes within a few minutes."""
     import oracle
-    c = WORKLOAD
+    layers, _, strong = WORKLOADS[args.workload]
     per_step_s = float(np.clip(150.0 / max(args.steps + args.warmup, 1), 1.0, 10.0))
-    _, _, _, n_pix = oracle_sample(c, target_s=per_step_s)
-    images = 4
-    ci = c.replace(N=images)
-    x = inputs.gen_x(ci, images=list(range(images)))
-    P = inputs.gen_offset_branch(c)
-    w, b = inputs.gen_weight(c)
-
-    def step():
-        off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
-                                        P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated)
-        oracle.dcn_pixels(x, off, w, np.arange(n_pix) % ci.M, b, mask=msk, G=c.G)
-
+    _, _, sample, n_pix, step, flops = oracle_sample(layers, target_s=per_step_s,
+                                                     images=sample_images(args.workload))
     for _ in range(args.warmup):
-        step()
+        step(n_pix)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        step()
+        step(n_pix)
     dt = time.perf_counter() - t0
-    flops = 2 * n_pix * c.Cout * c.K * c.K * c.Cin
     value = flops * args.steps / dt / 1e12
-    sample = (f"{c.name}: per step the offset branch of {images} images + DCN at {n_pix} of their "
-              f"output pixels, fp64 C oracle with OpenMP")
+    sample = "per step: " + sample
     return {
         "impl": "reference",
-        "metric": metric_name(),
+        "metric": metric_name(args.workload),
         "value": value,
         "unit": "TFLOP/s",
         "n_gpus": world,
@@ -463,11 +560,12 @@ def reference_arm(args, world):
         "warmup": args.warmup,
         "ms_per_step": dt / args.steps * 1e3,
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong" if strong else "weak",
         "vs_baseline": None,
         "dtype": "f64",
         "data": "synthetic (seeded)",
-        "config": workload_config(c, world, {"sample": sample}),
+        "config": workload_config(layers[0], world, {"sample": sample}, name=args.workload,
+                                  per_rank=STACK_GLOBAL_BATCH // world if strong else None),
         "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": oracle.num_threads(),
                          "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -480,6 +578,7 @@ def main():
     ap.add_argument("--steps", type=int, default=2000)
     ap.add_argument("--warmup", type=int, default=50)
     ap.add_argument("--impl", default="defcon", choices=["defcon", "reference"])
+    ap.add_argument("--workload", default="c4", choices=sorted(WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
@@ -503,7 +602,7 @@ def main():
     line = gpu_arm(args, rank, world, local_rank, dist)
     if rank == 0:
         if not args.no_cpu_baseline and world == 1:
-            line["cpu_baseline"] = cpu_baseline(WORKLOAD)
+            line["cpu_baseline"] = cpu_baseline(args.workload)
         print(json.dumps(line), flush=True)
     if dist is not None:
         dist.barrier()

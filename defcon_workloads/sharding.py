@@ -19,6 +19,16 @@ def shard_images(rank: int, world: int, per_rank: int):
     return list(range(rank * per_rank, (rank + 1) * per_rank))
 
 
+def shard_strong(rank: int, world: int, global_batch: int):
+    """Strong scaling (config 5: a fixed global batch): contiguous image blocks, the first
+    global_batch % world ranks take one extra image."""
+    if not (0 <= rank < world) or global_batch < world:
+        raise ValueError("bad shard")
+    base, extra = divmod(global_batch, world)
+    start = rank * base + min(rank, extra)
+    return list(range(start, start + base + (1 if rank < extra else 0)))
+
+
 def max_over_ranks(dist, values, device):
     """Element-wise max of a list of floats over all ranks (the job's wall time is the
     slowest rank's).  dist=None means single process."""

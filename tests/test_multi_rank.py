@@ -73,3 +73,57 @@ def test_shard_images():
     assert sharding.shard_images(1, 4, 16) == list(range(16, 32))
     with pytest.raises(ValueError):
         sharding.shard_images(4, 4, 16)
+
+
+def test_shard_strong():
+    """Config 5 (global batch 64, strong scaling): contiguous blocks covering every image once."""
+    for world in (1, 2, 3, 4, 8):
+        parts = [sharding.shard_strong(r, world, 64) for r in range(world)]
+        assert sum(parts, []) == list(range(64))
+        assert max(map(len, parts)) - min(map(len, parts)) <= 1
+    assert sharding.shard_strong(1, 8, 64) == list(range(8, 16))
+    with pytest.raises(ValueError):
+        sharding.shard_strong(0, 8, 4)
+
+
+def _stack_worker(rank, world, port, out_dir):
+    """Two-layer stack (stride-2 then stride-1, each fed by its offset branch) on a strong shard
+    of a global batch of 4 images; rank 0 gathers the last layer's y."""
+    import oracle
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    oracle.set_num_threads(1)
+    imgs = sharding.shard_strong(rank, world, 4)
+    ys = []
+    for c in _tiny_stack(len(imgs)):
+        x = inputs.gen_x(c, imgs)
+        P = inputs.gen_offset_branch(c)
+        off, msk = oracle.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"], P["pw_b"],
+                                        K=c.K, G=c.G, with_mask=True, stride=c.stride, pad=c.pad)
+        w, b = inputs.gen_weight(c)
+        ys.append(oracle.dcn_forward(x, off, w, b, mask=msk, stride=c.stride, pad=c.pad))
+    t = torch.from_numpy(np.ascontiguousarray(ys[-1]))
+    yall = sharding.gather_outputs(dist, t)
+    if rank == 0:
+        np.save(os.path.join(out_dir, "stack.npy"), yall.numpy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def _tiny_stack(n):
+    return [configs.LayerConfig("ts0", N=n, Cin=8, Cout=8, H=9, W=7, stride=2, config_id=12),
+            configs.LayerConfig("ts1", N=n, Cin=8, Cout=8, H=5, W=4, config_id=12)]
+
+
+def test_gloo_strong_sharding_stack(tmp_path, oracle_mod):
+    world = 2
+    mp.spawn(_stack_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    c = _tiny_stack(4)[-1]
+    x = inputs.gen_x(c)
+    P = inputs.gen_offset_branch(c)
+    off, msk = oracle_mod.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"], P["pw_b"],
+                                        K=c.K, G=c.G, with_mask=True, stride=c.stride, pad=c.pad)
+    w, b = inputs.gen_weight(c)
+    ref = oracle_mod.dcn_forward(x, off, w, b, mask=msk, stride=c.stride, pad=c.pad)
+    assert np.array_equal(np.load(tmp_path / "stack.npy"), ref)
