@@ -204,7 +204,7 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
         return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
     const size_t need = offset_branch_workspace(N, H, W, C, Ho, Wo, K, cv.offset_groups, cv.stride_h, cv.stride_w,
                                                 cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, x_dtype == DEFCON_BF16);
-    if (!workspace || workspace_bytes < need)
+    if (workspace_bytes < need || (need && !workspace))
         return fail(DEFCON_ERR_LIMIT, "workspace of %zu bytes < required %zu", workspace_bytes, need);
     cudaError_t e = launch_offset_branch(x, x_dtype == DEFCON_BF16, N, H, W, C, dw_w, dw_scale,
                                          dw_shift, pw_w, pw_b, K, G, mask != nullptr, cv.stride_h,

@@ -8,8 +8,8 @@
 // Per 32-channel chunk:
 //   * TMA brings the tile's input window (IR rows x IC columns x 32 channels of NHWC x, box
 //     coordinates starting at -pad: the unit zero-fills everything outside the image, which
-//     IS the depthwise conv's zero padding) into a swizzled shared-memory stage (SWIZZLE_64B
-//     for bf16's 64-byte rows, SWIZZLE_128B for fp32's 128-byte rows), XS chunks ahead;
+//     IS the depthwise conv's zero padding) into an unswizzled shared-memory stage whose
+//     position stride (80 / 144 bytes) keeps the dw loads free of bank conflicts, XS chunks ahead;
 //   * the 8 warps compute t on the CUDA cores: task = (8 channels, output row, run of RUN
 //     adjacent pixels); for stride 1 / dilation 1 each input column of a tap row is loaded and
 //     widened once and used by every output of the run that covers it (packed FFMA2, fp32);
@@ -34,11 +34,23 @@ namespace defcon {
 namespace {
 
 constexpr int OP_KC = 32;              // channels per chunk = one 128-byte tf32 operand row
+// x stage: one input position = op_kb(ES) channels (the chunk's 32 + 8 / 4 of the next chunk,
+// unused), i.e. 80 bytes (bf16) or 144 bytes (fp32), unswizzled.  Pixel p then starts at bank
+// 20p / 4p (mod 32): the 8 pixel pairs a warp reads in one instruction hit every bank the same
+// number of times (a 64- / 128-byte position would put every even pixel on the same 16 banks).
+__host__ __device__ constexpr int op_kb(int es) { return es == 2 ? 40 : 36; }
 constexpr uint32_t TF32_HI = 0xFFFFE000u;
-constexpr int OP_MAXT = 256;           // threads = 2 * TP (TP <= 128 pixels per tile)
 
 #ifdef DEFCON_PROBE_OP_TIMELINE   // dev probe: per-CTA phase timestamps (globaltimer, ns)
-__device__ unsigned long long g_op_tl[1024][32];
+__device__ unsigned long long g_op_tl[1024][48];
+__device__ __forceinline__ void op_stamp_any(int i) {   // any thread (loader / issuer lanes)
+    if (blockIdx.x < 1024 && i < 48) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_op_tl[blockIdx.x][i] = t;
+    }
+}
+#define OPTL_ANY(i) op_stamp_any(i)
 __device__ __forceinline__ void op_stamp(int i) {
     if (threadIdx.x == 0 && blockIdx.x < 1024 && i < 32) {
         unsigned long long t;
@@ -49,6 +61,7 @@ __device__ __forceinline__ void op_stamp(int i) {
 #define OPTL(i) op_stamp(i)
 #else
 #define OPTL(i) ((void)0)
+#define OPTL_ANY(i) ((void)0)
 #endif
 
 struct OpArgs {
@@ -71,27 +84,6 @@ struct OpArgs {
     int x_stage;            // bytes per x stage (1024-aligned)
     int tmem_cols, a_col;   // TMEM allocation and first A column
 };
-
-// SWIZZLE_128B: 16-byte unit (bits 4-6) XOR the 128-byte row index (bits 7-9) within 1024 B.
-__device__ __forceinline__ uint32_t sw128(uint32_t byte) { return byte ^ (((byte >> 7) & 7u) << 4); }
-// SWIZZLE_64B: 16-byte unit (bits 4-5) XOR bits 7-8 within 512 B (the x stage of bf16 input,
-// whose 32-channel box rows are 64 bytes: the swizzle span must match the box row).
-__device__ __forceinline__ uint32_t sw64(uint32_t byte) { return byte ^ (((byte >> 7) & 3u) << 4); }
-
-// 8 channels at stage byte offset `byte` of stage base `b` -> 4 fp32 pairs.
-template <int ES>
-__device__ __forceinline__ void lds_x8(const uint8_t* b, uint32_t byte, uint64_t (&v)[4]) {
-    if (ES == 2) {
-        const uint4 u = *reinterpret_cast<const uint4*>(b + sw64(byte));
-        v[0] = bf16x2_to_f32x2(u.x); v[1] = bf16x2_to_f32x2(u.y);
-        v[2] = bf16x2_to_f32x2(u.z); v[3] = bf16x2_to_f32x2(u.w);
-    } else {
-        const uint4 u0 = *reinterpret_cast<const uint4*>(b + sw128(byte));
-        const uint4 u1 = *reinterpret_cast<const uint4*>(b + sw128(byte + 16u));
-        v[0] = ((uint64_t)u0.y << 32) | u0.x; v[1] = ((uint64_t)u0.w << 32) | u0.z;
-        v[2] = ((uint64_t)u1.y << 32) | u1.x; v[3] = ((uint64_t)u1.w << 32) | u1.z;
-    }
-}
 
 // ---- packed per-chunk parameters (written once per call by op_pack_kernel into the caller's
 // workspace, then bulk-copied into shared memory with each chunk's x stage): chunk k's block is
@@ -137,18 +129,23 @@ __global__ void __launch_bounds__(256) op_pack_kernel(const float* __restrict__ 
 
 // Warp roles.  Tile pixels are taken in pairs (virtual columns 2q, 2q+1 of a row: rows have
 // even virtual length Wv and tiles start at even pixels, so a pair never straddles a row); the
-// tile's nblk = TP/16 blocks of 8 pairs live in TMEM lane quarters: block b in lanes 32b .. 32b+15,
-// the left pixel of pair 8b+l in lane 32b+l and the right one in lane 32b+l+8 (the lane pattern
-// of tcgen05.st.16x256b).  Compute warp w (w % 4 = block, w / 4 = channel half) and lane t of it
-// work on pair l = t/4, channels 8g + 4*half .. +3 of the chunk's 32 (g = t%4): two warps per
-// block, so the warps per SM are not bounded by 16 pixels per warp.  The 4 input columns of a tap
+// tile's nblk = TP/16 <= 8 blocks of 8 pairs live in TMEM lane quarters: block b in lanes
+// L(b) = 32(b%4) + 16(b/4) .. +15, the left pixel of pair 8b+l in lane L(b)+l and the right one
+// in lane L(b)+l+8 (the lane pattern of tcgen05.st.16x256b).  Compute warp w (quarter w % 4,
+// channel half w / 4) handles block w%4 and then, for nblk > 4, block w%4 + 4 (the other half of
+// its lane quarter); lane t of it works on pair l = t/4, channels 8g + 4*half .. +3 of the
+// chunk's 32 (g = t%4).  The 4 input columns of a tap
 // row serve both pixels, the tap weights are read once for both.  t goes to the A operand in
-// TENSOR memory (tf32 hi / lo planes, 32 columns each), so the MMAs read only W2 from shared
-// memory.  The issuer warp (the first unused id) loads each chunk's x window (TMA) and packed
-// parameters (bulk copy) into a stage and issues the chunk's MMAs once the compute warps have
-// published its A operand.
+// TENSOR memory, one buffer per channel half (16 K positions: tf32 hi in 16 columns, lo in the
+// next 16), so the MMAs read only W2 from shared memory.  The two halves pipeline against each
+// other: the issuer warp runs a half's 6 MMAs (2 k-steps x 3xTF32) as soon as its 4 compute
+// warps have published it, and those warps compute the next chunk meanwhile, waiting only for
+// their own half's previous MMAs before overwriting its buffer.  The loader warp refills a stage
+// (x window by TMA + the chunk's packed parameters by bulk copy) once the chunk's last MMAs,
+// which follow both halves' reads of the stage, have completed.
+constexpr int OP_REGS = 64;            // registers per thread (__maxnreg__)
 template <int ES, bool S1>
-__global__ void __maxnreg__(80)
+__global__ void __maxnreg__(OP_REGS)
     offset_branch_onepass_kernel(const __grid_constant__ CUtensorMap xmap, const OpArgs a) {
     extern __shared__ __align__(1024) uint8_t op_raw[];
     // 1024-aligned base by pointer arithmetic on the __shared__ array (keeps every derived
@@ -159,17 +156,19 @@ __global__ void __maxnreg__(80)
     const int STG = a.x_stage + PBLK;                          // stage = [x window | packed params]
     uint8_t* st_base = smem;                                   // [XS] stages
     uint8_t* zero = st_base + a.XS * STG;                      // 1 KB of zeros
-    float* bias_s = reinterpret_cast<float*>(zero + 1024);     // [256] 1x1 bias (0 when absent)
-    uint64_t* xfull = reinterpret_cast<uint64_t*>(bias_s + 256);   // [XS] stage landed
-    uint64_t* afull = xfull + a.XS;                            // [2] chunk's A published
-    uint64_t* mma_done = afull + 2;                            // [2] chunk's MMAs complete
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(mma_done + 2);
+    uint64_t* xfull = reinterpret_cast<uint64_t*>(zero + 2048);    // [XS] stage landed
+    uint64_t* afull = xfull + a.XS;                            // [2] half h's A published
+    uint64_t* mma_done = afull + 2;                            // [2] half h's MMAs complete
+    uint64_t* sfree = mma_done + 2;                            // [XS] stage's last MMAs complete
+    uint64_t* acc_full = sfree + a.XS;                         // all MMAs complete
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_full + 1);
     float* out_s = reinterpret_cast<float*>(smem);             // epilogue staging (stages)
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int TP = a.TP;
     const int nblk = TP >> 4;                                  // 16-lane blocks (<= 4)
-    const int issuer_warp = nblk < 4 ? nblk : 8;
+    const int issuer_warp = nblk < 4 ? 3 : 8;                  // ids no compute warp uses
+    const int loader_warp = nblk < 4 ? 7 : 9;
     const int v0 = blockIdx.x * TP;                            // first virtual pixel of the tile
     const uint32_t tcols = a.tmem_cols;
     const uint32_t ACOL = a.a_col;                             // first A column (after the accumulator)
@@ -177,14 +176,17 @@ __global__ void __maxnreg__(80)
     OPTL(0);
     for (int e = tid; e < 256; e += blockDim.x) {
         reinterpret_cast<float*>(zero)[e] = 0.f;
-        bias_s[e] = (a.pw_b && e < a.OC) ? __ldg(a.pw_b + e) : 0.f;
     }
     if (tid == 0) {
-        for (int s = 0; s < a.XS; ++s) mbar_init(&xfull[s], 1);
+        for (int s = 0; s < a.XS; ++s) {
+            mbar_init(&xfull[s], 1);
+            mbar_init(&sfree[s], 1);
+        }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&afull[b], 1);
             mbar_init(&mma_done[b], 1);
         }
+        mbar_init(acc_full, 1);
         fence_barrier_init();
         tma_prefetch_desc(&xmap);
     }
@@ -206,10 +208,10 @@ __global__ void __maxnreg__(80)
     const int n0 = v0 / HoWv, ho0 = (v0 - n0 * HoWv) / a.Wv;
     const int Y0 = n0 * a.H + ho0 * a.sh - a.ph;              // window origin (stacked rows)
 
-    if (warp == issuer_warp) {
-        // ===================== TMA + MMA issuer =====================
+    if (warp == loader_warp) {
+        // ===================== stage loader (TMA x window + bulk-copied parameters) =========
         if (lane == 0) {
-            const uint32_t tx = (uint32_t)(a.IR * a.IC * OP_KC * ES + PBLK);
+            const uint32_t tx = (uint32_t)(a.IR * a.IC * op_kb(ES) * ES + PBLK);
             auto load_stage = [&](int k, int s) {
                 uint8_t* st = st_base + s * STG;
                 mbar_arrive_expect_tx(&xfull[s], tx);
@@ -217,60 +219,83 @@ __global__ void __maxnreg__(80)
                 bulk_load(st + a.x_stage, a.packed + (size_t)k * PBLK, (uint32_t)PBLK, &xfull[s]);
             };
             for (int k = 0; k < a.XS && k < a.nch; ++k) load_stage(k, k);
-            const uint32_t idesc = make_idesc(2u /*TF32*/, 128, (uint32_t)a.OCN);
-            int s = 0;
-            for (int k = 0; k < a.nch; ++k) {
-                const int ab = k & 1;
-                mbar_wait(&afull[ab], (uint32_t)(k >> 1) & 1u);   // A of chunk k published
-                tc_fence_after();
-                const uint32_t ah = tmem + ACOL, al = ah + 32u;
-                const uint32_t bh = smem_u32(st_base + s * STG + a.x_stage), bl = bh + B_PLANE;
-#pragma unroll
-                for (int kk = 0; kk < OP_KC / 8; ++kk) {
-                    const uint64_t dbh = make_sw128_desc(bh + kk * 32), dbl = make_sw128_desc(bl + kk * 32);
-                    mma_tf32_ts(tmem, al + kk * 8, dbh, idesc, (k | kk) != 0 ? 1u : 0u);
-                    mma_tf32_ts(tmem, ah + kk * 8, dbl, idesc, 1u);
-                    mma_tf32_ts(tmem, ah + kk * 8, dbh, idesc, 1u);
-                }
-                mma_commit(&mma_done[ab]);
-                if (k + a.XS < a.nch) {
-                    // stage s: x consumed (afull) and its W2 read by MMA(k): refill with chunk k+XS
-                    mbar_wait(&mma_done[ab], (uint32_t)(k >> 1) & 1u);
-                    load_stage(k + a.XS, s);
-                }
-                if (++s == a.XS) s = 0;
+            for (int k = a.XS; k < a.nch; ++k) {   // stage of chunk k - XS: its MMAs are done
+                const int s = k % a.XS;
+                mbar_wait(&sfree[s], (uint32_t)((k - a.XS) / a.XS) & 1u);
+                if (k < 8) OPTL_ANY(32 + k);
+                load_stage(k, s);
             }
         }
         return;
     }
-    if (warp >= 8 || (warp & 3) >= nblk) return;   // unused ids (small tiles)
+    if (warp == issuer_warp) {
+        // ===================== MMA issuer =====================
+        if (lane == 0) {
+            const uint32_t idesc = make_idesc(2u /*TF32*/, 128, (uint32_t)a.OCN);
+            int s = 0;
+            for (int k = 0; k < a.nch; ++k) {
+                const uint32_t bh = smem_u32(st_base + s * STG + a.x_stage), bl = bh + B_PLANE;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    mbar_wait(&afull[h], (uint32_t)k & 1u);         // half h of chunk k published
+                    if (h == 1 && k < 8) OPTL_ANY(40 + k);
+                    tc_fence_after();
+                    const uint32_t ah = tmem + ACOL + 32u * h, al = ah + 16u;
+#pragma unroll
+                    for (int kk = 0; kk < 2; ++kk) {               // K positions 16h + 8kk .. +7
+                        const uint32_t kb = (uint32_t)(2 * h + kk) * 32u;
+                        const uint64_t dbh = make_sw128_desc(bh + kb), dbl = make_sw128_desc(bl + kb);
+                        mma_tf32_ts(tmem, al + kk * 8, dbh, idesc, (k | h | kk) != 0 ? 1u : 0u);
+                        mma_tf32_ts(tmem, ah + kk * 8, dbl, idesc, 1u);
+                        mma_tf32_ts(tmem, ah + kk * 8, dbh, idesc, 1u);
+                    }
+                    mma_commit(&mma_done[h]);
+                }
+                mma_commit(&sfree[s]);
+                if (++s == a.XS) s = 0;
+            }
+            mma_commit(acc_full);
+        }
+        return;
+    }
+    const int NQ = nblk < 4 ? nblk : 4;                        // lane quarters in use
+    if (warp >= 8 || (warp & 3) >= NQ) return;                 // unused ids (small tiles)
 
     // ===================== compute warps =====================
-    const int NC = 64 * nblk;                                  // compute threads
-    const int ctid = ((warp >> 2) * nblk + (warp & 3)) * 32 + lane;   // 0 .. NC-1
-    const int blk = warp & 3, half = warp >> 2;
+    // warp (quarter qd, half) handles block qd (lanes 32qd .. +15) and, for nblk > 4, block
+    // qd + 4 (lanes 32qd + 16 .. +31), one after the other
+    const int NC = 64 * NQ;                                    // compute threads
+    const int ctid = ((warp >> 2) * NQ + (warp & 3)) * 32 + lane;   // 0 .. NC-1
+    const int qd = warp & 3, half = warp >> 2;
+    const int nsub = qd + 4 < nblk ? 2 : 1;                    // blocks of this warp
     const int l = lane >> 2, g = lane & 3;
-    const int q = 8 * blk + l;                                 // pixel pair within the tile
-    const int vp = v0 + 2 * q;                                 // virtual pixel of the left one
-    const bool pix_ok = vp < a.MV;
-    const int vpc = pix_ok ? vp : v0;
-    const int n = vpc / HoWv;
-    const int rem = vpc - n * HoWv;
-    const int ho = rem / a.Wv, wo = rem - ho * a.Wv;           // wo even
-    constexpr uint32_t PB = OP_KC * ES;                        // bytes per input position of a stage
+    constexpr uint32_t PB = op_kb(ES) * ES;                    // bytes per input position of a stage
     const uint32_t chb = (uint32_t)(8 * g + 4 * half) * ES;    // byte offset of this thread's 4 channels
-    uint32_t row_byte[3];   // stage byte offset of tap (i, 0) of the left pixel + channels
-    uint32_t row_ok = 0;    // tap rows in the zero padding (incl. a neighbouring image's rows)
+    uint32_t row_byte[2][3];   // stage byte offset of tap (i, 0) of the left pixel + channels
+    uint32_t row_ok[2];        // tap rows not in the zero padding (incl. a neighbouring image's rows)
 #pragma unroll
-    for (int i = 0; i < 3; ++i) {
-        const int yy = ho * a.sh - a.ph + i * a.dh;
-        const bool ok = pix_ok && yy >= 0 && yy < a.H;
-        row_ok |= ok ? 1u << i : 0u;
-        row_byte[i] = (ok ? (uint32_t)((n * a.H + yy - Y0) * a.IC + wo * a.sw) * PB : 0u) + chb;
+    for (int sb = 0; sb < 2; ++sb) {
+        const int q = 8 * (qd + 4 * sb) + l;                   // pixel pair within the tile
+        const int vp = v0 + 2 * q;                             // virtual pixel of the left one
+        const bool pix_ok = sb < nsub && vp < a.MV;
+        const int vpc = pix_ok ? vp : v0;
+        const int n = vpc / HoWv;
+        const int rem = vpc - n * HoWv;
+        const int ho = rem / a.Wv, wo = rem - ho * a.Wv;       // wo even
+        row_ok[sb] = 0;
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+            const int yy = ho * a.sh - a.ph + i * a.dh;
+            const bool ok = pix_ok && yy >= 0 && yy < a.H;
+            row_ok[sb] |= ok ? 1u << i : 0u;
+            row_byte[sb][i] = (ok ? (uint32_t)((n * a.H + yy - Y0) * a.IC + wo * a.sw) * PB : 0u) + chb;
+        }
     }
     const uint32_t col_step = (uint32_t)a.dw * PB;   // next tap column
     const uint32_t px_step = (uint32_t)a.sw * PB;    // the right pixel of the pair
-    const uint32_t a_addr = tmem + ((uint32_t)(32 * blk) << 16) + ACOL + 16u * half;
+    // this half's A buffer, lanes of block qd; block qd + 4 is 16 lanes further
+    const uint32_t a_addr = tmem + ((uint32_t)(32 * qd) << 16) + ACOL + 32u * half;
+    const bool half_lead = qd == 0 && lane == 0;
     const int wofs = 2 * B_PLANE / 4 + 8 * g + 4 * half;       // this thread's dw weights in a stage (floats)
 
     int s = 0;                          // stage of chunk k (k mod XS)
@@ -280,94 +305,97 @@ __global__ void __maxnreg__(80)
         const float* wk = reinterpret_cast<const float*>(xst + a.x_stage) + wofs;
         mbar_wait(&xfull[s], xphase);
         if (k < 8) OPTL(4 + 2 * k);
-        // ---- depthwise 3x3 of 4 channels at two pixels, fp32 pairs (FFMA2)
-        uint64_t acc0[2] = {0ull, 0ull}, acc1[2] = {0ull, 0ull};
-#ifdef OP_PROBE_NO_DW   // dev probe: skip the depthwise work (garbage t)
-        if (row_ok == 0xFFu)
-#endif
+#pragma unroll 1
+        for (int sb = 0; sb < nsub; ++sb) {
+            const uint32_t rok = sb ? row_ok[1] : row_ok[0];
+            // ---- depthwise 3x3 of 4 channels at two pixels, fp32 pairs (FFMA2)
+            uint64_t acc0[2] = {0ull, 0ull}, acc1[2] = {0ull, 0ull};
 #pragma unroll
-        for (int i = 0; i < 3; ++i) {
-            const bool ok = (row_ok >> i) & 1u;
-            const uint8_t* rb = ok ? xst : zero;
-            uint64_t w[3][2];
-#pragma unroll
-            for (int jj = 0; jj < 3; ++jj) {
-                const float4 w0 = *reinterpret_cast<const float4*>(wk + (i * 3 + jj) * OP_KC);
-                w[jj][0] = f32x2_pack(w0.x, w0.y);
-                w[jj][1] = f32x2_pack(w0.z, w0.w);
-            }
-            auto ld4 = [&](uint32_t byte, uint64_t (&v)[2]) {   // 4 channels -> 2 fp32 pairs
-                if (ES == 2) {
-                    const uint2 u = *reinterpret_cast<const uint2*>(rb + sw64(byte));
-                    v[0] = bf16x2_to_f32x2(u.x);
-                    v[1] = bf16x2_to_f32x2(u.y);
-                } else {
-                    const uint4 u = *reinterpret_cast<const uint4*>(rb + sw128(byte));
-                    v[0] = ((uint64_t)u.y << 32) | u.x;
-                    v[1] = ((uint64_t)u.w << 32) | u.z;
-                }
-            };
-            if (S1) {
-                // stride-1 / dilation-1 columns: c = 0..3 feed the left pixel through tap c and
-                // the right one through tap c - 1
-#pragma unroll
-                for (int c = 0; c < 4; ++c) {
-                    uint64_t v[2];
-                    ld4(ok ? row_byte[i] + c * PB : chb, v);
-#pragma unroll
-                    for (int p = 0; p < 2; ++p) {
-                        if (c < 3) acc0[p] = f32x2_fma(w[c][p], v[p], acc0[p]);
-                        if (c > 0) acc1[p] = f32x2_fma(w[c - 1][p], v[p], acc1[p]);
-                    }
-                }
-            } else {
+            for (int i = 0; i < 3; ++i) {
+                const bool ok = (rok >> i) & 1u;
+                const uint8_t* rb = ok ? xst : zero;
+                const uint32_t rbyte = sb ? row_byte[1][i] : row_byte[0][i];
+                uint64_t w[3][2];
 #pragma unroll
                 for (int jj = 0; jj < 3; ++jj) {
-                    uint64_t v[2], u[2];
-                    ld4(ok ? row_byte[i] + jj * col_step : chb, v);
-                    ld4(ok ? row_byte[i] + jj * col_step + px_step : chb, u);
+                    const float4 w0 = *reinterpret_cast<const float4*>(wk + (i * 3 + jj) * OP_KC);
+                    w[jj][0] = f32x2_pack(w0.x, w0.y);
+                    w[jj][1] = f32x2_pack(w0.z, w0.w);
+                }
+                auto ld4 = [&](uint32_t byte, uint64_t (&v)[2]) {   // 4 channels -> 2 fp32 pairs
+                    if (ES == 2) {
+                        const uint2 u = *reinterpret_cast<const uint2*>(rb + byte);
+                        v[0] = bf16x2_to_f32x2(u.x);
+                        v[1] = bf16x2_to_f32x2(u.y);
+                    } else {
+                        const uint4 u = *reinterpret_cast<const uint4*>(rb + byte);
+                        v[0] = ((uint64_t)u.y << 32) | u.x;
+                        v[1] = ((uint64_t)u.w << 32) | u.z;
+                    }
+                };
+                if (S1) {
+                    // stride-1 / dilation-1 columns: c = 0..3 feed the left pixel through tap c and
+                    // the right one through tap c - 1
 #pragma unroll
-                    for (int p = 0; p < 2; ++p) {
-                        acc0[p] = f32x2_fma(w[jj][p], v[p], acc0[p]);
-                        acc1[p] = f32x2_fma(w[jj][p], u[p], acc1[p]);
+                    for (int c = 0; c < 4; ++c) {
+                        uint64_t v[2];
+                        ld4(ok ? rbyte + c * PB : chb, v);
+#pragma unroll
+                        for (int p = 0; p < 2; ++p) {
+                            if (c < 3) acc0[p] = f32x2_fma(w[c][p], v[p], acc0[p]);
+                            if (c > 0) acc1[p] = f32x2_fma(w[c - 1][p], v[p], acc1[p]);
+                        }
+                    }
+                } else {
+#pragma unroll
+                    for (int jj = 0; jj < 3; ++jj) {
+                        uint64_t v[2], u[2];
+                        ld4(ok ? rbyte + jj * col_step : chb, v);
+                        ld4(ok ? rbyte + jj * col_step + px_step : chb, u);
+#pragma unroll
+                        for (int p = 0; p < 2; ++p) {
+                            acc0[p] = f32x2_fma(w[jj][p], v[p], acc0[p]);
+                            acc1[p] = f32x2_fma(w[jj][p], u[p], acc1[p]);
+                        }
                     }
                 }
             }
-        }
-        // ---- folded BN + ReLU, tf32 hi / lo split; register 4c' + 2x + e = channel
-        // 8g + 4*half + 2c' + e of pixel x (the 16x256b.x2 store pattern)
-        uint32_t hv[8], lv[8];
-        {
-            const float4 sc = *reinterpret_cast<const float4*>(wk + 9 * OP_KC);
-            const float4 sf = *reinterpret_cast<const float4*>(wk + 10 * OP_KC);
-            const float scv[4] = {sc.x, sc.y, sc.z, sc.w};
-            const float sfv[4] = {sf.x, sf.y, sf.z, sf.w};
+            // ---- folded BN + ReLU, tf32 hi / lo split; register 4c' + 2x + e = channel
+            // 8g + 4*half + 2c' + e of pixel x (the 16x256b.x2 store pattern)
+            uint32_t hv[8], lv[8];
+            {
+                const float4 sc = *reinterpret_cast<const float4*>(wk + 9 * OP_KC);
+                const float4 sf = *reinterpret_cast<const float4*>(wk + 10 * OP_KC);
+                const float scv[4] = {sc.x, sc.y, sc.z, sc.w};
+                const float sfv[4] = {sf.x, sf.y, sf.z, sf.w};
 #pragma unroll
-            for (int x = 0; x < 2; ++x) {
-                const uint64_t* acc = x ? acc1 : acc0;
+                for (int x = 0; x < 2; ++x) {
+                    const uint64_t* acc = x ? acc1 : acc0;
 #pragma unroll
-                for (int c = 0; c < 2; ++c) {
+                    for (int c = 0; c < 2; ++c) {
 #pragma unroll
-                    for (int e = 0; e < 2; ++e) {
-                        const float v = __uint_as_float(e ? (uint32_t)(acc[c] >> 32) : (uint32_t)(acc[c] & 0xFFFFFFFFull));
-                        const float t = fmaxf(fmaf(scv[2 * c + e], v, sfv[2 * c + e]), 0.f);
-                        const uint32_t h = __float_as_uint(t) & TF32_HI;
-                        hv[4 * c + 2 * x + e] = h;
-                        lv[4 * c + 2 * x + e] = __float_as_uint(t - __uint_as_float(h));
+                        for (int e = 0; e < 2; ++e) {
+                            const float v = __uint_as_float(e ? (uint32_t)(acc[c] >> 32) : (uint32_t)(acc[c] & 0xFFFFFFFFull));
+                            const float t = fmaxf(fmaf(scv[2 * c + e], v, sfv[2 * c + e]), 0.f);
+                            const uint32_t h = __float_as_uint(t) & TF32_HI;
+                            hv[4 * c + 2 * x + e] = h;
+                            lv[4 * c + 2 * x + e] = __float_as_uint(t - __uint_as_float(h));
+                        }
                     }
                 }
             }
+            // this half's A buffer was last read by its MMAs of chunk k-1
+            if (sb == 0 && k >= 1) mbar_wait(&mma_done[half], (uint32_t)(k - 1) & 1u);
+            tc_fence_after();
+            const uint32_t ad = a_addr + ((uint32_t)(16 * sb) << 16);
+            tmem_st_16x256b_x2(ad, hv);
+            tmem_st_16x256b_x2(ad + 16u, lv);
         }
-        // the single A buffer was last read by MMA(k-1)
-        if (k >= 1) mbar_wait(&mma_done[(k - 1) & 1], (uint32_t)((k - 1) >> 1) & 1u);
-        tc_fence_after();
-        tmem_st_16x256b_x2(a_addr, hv);
-        tmem_st_16x256b_x2(a_addr + 32u, lv);
         tmem_st_wait();
         tc_fence_before();
-        named_bar_sync(1, NC);      // A of chunk k complete; stage s read
+        named_bar_sync(1 + half, NC / 2);      // this half's A of chunk k complete
         if (k < 8) OPTL(5 + 2 * k);
-        if (ctid == 0) mbar_arrive(&afull[k & 1]);
+        if (half_lead) mbar_arrive(&afull[half]);
         if (++s == a.XS) {
             s = 0;
             xphase ^= 1u;
@@ -375,10 +403,19 @@ __global__ void __maxnreg__(80)
     }
     // ---- epilogue: accumulator lane = tile pixel (pair layout above), column = output channel;
     // + b2, sigmoid on the mask channels, staged in shared memory in the global layout (the tile's
-    // real pixels are one contiguous range of m), then copied out coalesced.  Warp w reads lanes
-    // 32*(w%4) .. +15 and the column half w/4.
+    // real pixels are one contiguous range of m), then copied out coalesced.  Warp (qd, half)
+    // reads lanes 32qd .. +31 (blocks qd and qd + 4) and the 16-column groups half, half + 2, ..
     OPTL(20);
-    mbar_wait(&mma_done[(a.nch - 1) & 1], (uint32_t)((a.nch - 1) >> 1) & 1u);
+    float bias_r[16];
+    {
+        const int cg0 = half;                                  // the first column group (bias prefetch)
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+            const int o = 16 * cg0 + u;
+            bias_r[u] = (a.pw_b && o < a.OC) ? __ldg(a.pw_b + o) : 0.f;
+        }
+    }
+    mbar_wait(acc_full, 0u);
     tc_fence_after();
     OPTL(21);
     const int vl = min(v0 + TP, a.MV) - 1;
@@ -392,34 +429,38 @@ __global__ void __maxnreg__(80)
     float* off_s = out_s;
     float* msk_s = out_s + nreal * a.n_off;
     {
-        const int li = lane & 15;
-        const int v = v0 + 2 * (8 * blk + (li & 7)) + (li >> 3);   // virtual pixel of lane 32*blk + li
+        const int li = lane & 15, bb = qd + 4 * (lane >> 4);
+        const int v = v0 + 2 * (8 * bb + (li & 7)) + (li >> 3);   // virtual pixel of lane 32*qd + lane
         const int rr = v / a.Wv, cc = v - rr * a.Wv;
-        const bool ok = lane < 16 && v < a.MV && cc < a.Wo;
+        const bool ok = bb < nblk && v < a.MV && cc < a.Wo;
         const int dm = rr * a.Wo + cc - mf;                   // real-pixel index within the tile
         const int ngrp = a.OCN >> 4;                           // 16-column groups
         for (int cg = half; cg < ngrp; cg += 2) {
             uint32_t vv[16];
-            tmem_ld_32x32b_x16(tmem + ((uint32_t)(32 * blk) << 16) + (uint32_t)(16 * cg), vv);
+            tmem_ld_32x32b_x16(tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(16 * cg), vv);
             tmem_ld_wait();
             if (!ok) continue;
 #pragma unroll
             for (int u = 0; u < 16; ++u) {
                 const int o = 16 * cg + u;
-                const float val = __uint_as_float(vv[u]) + bias_s[o];
+                const float val = __uint_as_float(vv[u]) +
+                                  (cg == half ? bias_r[u] : (a.pw_b && o < a.OC) ? __ldg(a.pw_b + o) : 0.f);
                 if (o < a.n_off) off_s[dm * a.n_off + o] = val;
                 else if (o < a.OC) msk_s[dm * a.n_msk + (o - a.n_off)] = __fdividef(1.f, 1.f + __expf(-val));
             }
         }
     }
+    OPTL(23);
     tc_fence_before();
-    named_bar_sync(1, NC);   // staged; TMEM no longer read
+    named_bar_sync(3, NC);   // staged; TMEM no longer read
+    OPTL(30);
     if (warp == 0) {
         tc_fence_after();
         if (tcols == 128) tmem_dealloc<128>(tmem);
         else if (tcols == 256) tmem_dealloc<256>(tmem);
         else tmem_dealloc<512>(tmem);
     }
+    OPTL(31);
     {
         float* go = a.offset + (long)mf * a.n_off;
         for (int e = ctid; e < nreal * a.n_off; e += NC) go[e] = off_s[e];
@@ -445,7 +486,7 @@ constexpr size_t OP_SMEM_TWO = 113 * 1024;   // two CTAs per SM
 #endif
 
 size_t op_smem(const OpArgs& a) {
-    return 1024 + (size_t)a.XS * (a.x_stage + op_block_bytes(a.OCN)) + 2048 + (a.XS + 4) * 8 + 16;
+    return 1024 + (size_t)a.XS * (a.x_stage + op_block_bytes(a.OCN)) + 2048 + (2 * a.XS + 5) * 8 + 16;
 }
 
 // Tile = TP consecutive pixels of the virtual [N][Ho][Wv] grid (a tile may run across an image
@@ -477,14 +518,17 @@ bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, in
     }
     long best = LONG_MAX;
     bool found = false;
-    for (int TP = 16; TP <= 64; TP += 16) {
+    for (int TP = 16; TP <= 128; TP += 16) {
         if (TP > Ho * a.Wv && TP > 16) break;     // a tile spans at most two images
+#ifdef OP_PROBE_TP   // dev probe: force the tile size
+        if (TP != OP_PROBE_TP) continue;
+#endif
         OpArgs t = a;
         t.TP = TP;
         const int orows = (a.Wv - 2 + TP + a.Wv - 1) / a.Wv;          // output rows a tile can touch
         t.IR = (orows - 1) * sh + std::max(0, H - Ho * sh) + 2 * dh + 1;
         if (t.IR > 256) continue;
-        t.x_stage = (int)(((size_t)t.IR * t.IC * OP_KC * es + 1023) & ~size_t(1023));
+        t.x_stage = (int)(((size_t)t.IR * t.IC * op_kb(es) * es + 1023) & ~size_t(1023));
         // epilogue staging ([TP][OC] fp32) reuses the x stages
         t.XS = 3;
         while (op_smem(t) > OP_SMEM_CAP / 3 && t.XS > 2) --t.XS;
@@ -492,10 +536,10 @@ bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, in
         const size_t sm = op_smem(t);
         if (sm > OP_SMEM_CAP) continue;
         // CTAs per SM: shared memory, TMEM columns (512 per SM), registers
-        const int nwarps = TP == 64 ? 9 : (TP / 16 < 4 ? 4 + TP / 16 : 9);
+        const int nwarps = TP >= 64 ? 10 : 8;
         int cps = (int)std::min<size_t>(OP_SMEM_CAP / sm, 512 / t.tmem_cols);
-        // 80 registers per thread (__maxnreg__): 6 warps per SM sub-partition (16K registers each)
-        cps = std::min(cps, 24 / nwarps);
+        // OP_REGS registers per thread: 4 sub-partitions x 16K registers per SM
+        cps = std::min(cps, 4 * (16384 / (OP_REGS * 32)) / nwarps);
         if (cps < 1) continue;
         const long tiles = (MV + TP - 1) / TP;
         const long rounds = (tiles + (long)sms * cps - 1) / ((long)sms * cps);
@@ -522,7 +566,8 @@ cudaError_t launch_op(const OpPlan& p, const CUtensorMap& xmap, cudaStream_t str
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
     if (e != cudaSuccess) return e;
     const int nblk = p.a.TP / 16;
-    const int threads = 32 * (nblk < 4 ? 4 + nblk : 9);   // compute warps 0..nblk-1, 4..3+nblk + issuer
+    // compute warps 0..nblk-1 (half 0), 4..3+nblk (half 1); issuer + loader: 3, 7 or 8, 9
+    const int threads = 32 * (nblk < 4 ? 8 : 10);
     return launch_pdl(kern, dim3(p.tiles), dim3(threads), p.smem, stream, xmap, p.a);
 }
 
@@ -571,11 +616,11 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
     CUtensorMap xmap;
     cuuint64_t dims[3] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)N * H};
     cuuint64_t strides[2] = {(cuuint64_t)C * es, (cuuint64_t)W * C * es};
-    cuuint32_t box[3] = {(cuuint32_t)OP_KC, (cuuint32_t)a.IC, (cuuint32_t)a.IR};
+    cuuint32_t box[3] = {(cuuint32_t)op_kb(es), (cuuint32_t)a.IC, (cuuint32_t)a.IR};
     cuuint32_t estr[3] = {1, 1, 1};
     CUresult cr = encode(&xmap, x_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
                          const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                         x_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_SWIZZLE_NONE,
                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (cr != CUDA_SUCCESS) return cudaErrorInvalidValue;
     return x_bf16 ? launch_op<2>(p, xmap, stream) : launch_op<4>(p, xmap, stream);

@@ -25,7 +25,7 @@ P = {k: torch.from_numpy(v).to(dev) for k, v in inputs.gen_offset_branch(c).item
 for _ in range(3):
     d.defcon_offset_dw_conv(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"], P["pw_b"], offset_groups=c.G)
 torch.cuda.synchronize()
-buf = np.zeros((1024, 32), dtype=np.uint64)
+buf = np.zeros((1024, 48), dtype=np.uint64)
 lib.defcon_debug_op_timeline(buf.ctypes.data_as(ctypes.c_void_p))
 grid = int((buf[:, 0] > 0).sum())
 b = buf[:grid].astype(np.int64)
@@ -36,6 +36,10 @@ names = {0: "start", 1: "setup", 2: "griddep"}
 for k in range(8):
     names[4 + 2 * k] = f"x{k} ready"
     names[5 + 2 * k] = f"bar{k}"
+for k in range(3, 8):
+    names[32 + k] = f"ld{k} issued"
+for k in range(8):
+    names[40 + k] = f"mma{k} go"
 names.update({20: "loop end", 21: "mma done", 22: "epi end", 24: "k3 top", 25: "k3 A free", 26: "epi ld0 beg",
               27: "epi ld0 end", 28: "epi pre", 29: "epi cb0 done", 23: "epi staged", 30: "epi bar", 31: "dealloc"})
 for i, nm in names.items():
