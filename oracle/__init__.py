@@ -64,6 +64,7 @@ def _load():
                                                   ctypes.POINTER(ctypes.c_int64), ctypes.c_long, dp]
         lib.oracle_offset_branch_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, dp,
                                                  i, i, i, i, i, i, dp, dp]
+        lib.oracle_bound_offsets_f64.argtypes = [dp, ctypes.c_long, i, i, i, i, i, i, dp]
         lib.oracle_bilinear_f64.argtypes = [dp, i, i, ctypes.c_long, ctypes.c_double,
                                             ctypes.c_double]
         lib.oracle_bilinear_f64.restype = ctypes.c_double
@@ -239,3 +240,25 @@ def offset_branch(x, dw_w, dw_scale, dw_shift, pw_w, pw_b, K=3, G=1, with_mask=T
     if rc:
         raise ValueError(f"oracle_offset_branch_f64 rc={rc}")
     return off, msk
+
+
+def bound_offsets(offset, P, K=3, dil=1):
+    """Bounded deformation (section III-A-c; reading R12): each offset restricted so the
+    sampling point of tap (i, j) stays in the P x P window centred on the output pixel's centre
+    tap (P = 7 in the paper, Fig. 5).  P <= 0 (or None): unbounded, offsets returned as is.
+
+    offset [..., G, Kh*Kw, 2] (dy, dx); K = (Kh, Kw) or int; dil = (dh, dw) or int.
+    Returns the bounded offsets (fp64, same shape); feed them to dcn_forward / dcn_pixels.
+    """
+    off = _f64(offset)
+    Kh, Kw = _pair(K)
+    dh, dw = _pair(dil)
+    if off.shape[-1] != 2 or off.shape[-2] != Kh * Kw:
+        raise ValueError("offset shape")
+    G = off.shape[-3]
+    n_pix = int(np.prod(off.shape[:-3]))
+    out = np.empty_like(off)
+    rc = _load().oracle_bound_offsets_f64(_p(off), n_pix, G, Kh, Kw, dh, dw, int(P or 0), _p(out))
+    if rc:
+        raise ValueError(f"oracle_bound_offsets_f64 rc={rc}")
+    return out

@@ -29,6 +29,7 @@
  *   oracle_offset_branch_f64    lightweight offset branch (dw3x3, BN, ReLU, 1x1) P:170
  *   oracle_dcn_forward_texq_f64 Eq.2 with the texture unit's fixed-point filter
  *                               weights (texture model; NOT from the paper, R14)
+ *   oracle_bound_offsets_f64    bounded deformation, P x P window (R12)
  */
 #include <math.h>
 #include <stddef.h>
@@ -422,5 +423,39 @@ int oracle_deform_columns_f64(const double *x, int N, int H, int W, int Cin,
                       mask ? mask + pix * G * Kh * Kw : NULL, Kh, Kw, sh, sw, ph, pw, dh, dw, G,
                       n, ho, wo, 0, cols + t * KKC);
     }
+    return 0;
+}
+
+/* Bounded deformation (section III-A-c, reading R12): before the deformable kernel is
+ * applied, each learned offset is restricted so that the sampling point of tap (i, j) stays in
+ * the P x P window centred on the output pixel's centre tap.  Written per axis: with the tap's
+ * regular displacement from the centre tap r = (i - (Kh-1)/2) * dh (resp. (j - (Kw-1)/2) * dw)
+ * and h = (P - 1) / 2, the bounded offset is clamp(r + d, -h, h) - r.  P <= 0: unbounded (the
+ * offsets are copied).  A NaN offset stays NaN.  offset / out: [n_pix][G][Kh*Kw][2] (dy, dx);
+ * out may alias offset.  Returns 0, or 1 on invalid arguments. */
+int oracle_bound_offsets_f64(const double *offset, long n_pix, int G, int Kh, int Kw, int dh, int dw,
+                             int P, double *out) {
+    if (n_pix < 0 || G <= 0 || Kh <= 0 || Kw <= 0 || dh <= 0 || dw <= 0) return 1;
+    const double h = 0.5 * (P - 1);
+    for (long p = 0; p < n_pix; ++p)
+        for (int g = 0; g < G; ++g)
+            for (int i = 0; i < Kh; ++i)
+                for (int j = 0; j < Kw; ++j) {
+                    const long e = ((p * G + g) * Kh * Kw + (long)i * Kw + j) * 2;
+                    const double ry = (i - 0.5 * (Kh - 1)) * dh;   /* regular displacement */
+                    const double rx = (j - 0.5 * (Kw - 1)) * dw;
+                    double dy = offset[e], dx = offset[e + 1];
+                    if (P > 0) {
+                        double sy = ry + dy, sx = rx + dx;        /* point relative to the centre */
+                        if (sy < -h) sy = -h;
+                        if (sy > h) sy = h;
+                        if (sx < -h) sx = -h;
+                        if (sx > h) sx = h;
+                        dy = sy - ry;
+                        dx = sx - rx;
+                    }
+                    out[e] = dy;
+                    out[e + 1] = dx;
+                }
     return 0;
 }

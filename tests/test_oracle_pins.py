@@ -423,3 +423,61 @@ def test_columns_times_weight_is_dcn(oracle_mod):
     cols = oracle_mod.deform_columns(x, off, 3, pix_idx=idx, mask=m, G=2)
     yy = cols @ w.reshape(w.shape[0], -1).T + b
     assert np.max(np.abs(yy - y.reshape(-1, w.shape[0])[idx])) < 1e-12
+
+
+# ---------------------------------------------------------------- P15: bounded deformation
+# P:182 (section III-A-c) restricts the learned offsets before the deformable kernel; reading
+# R12: the sampling point of every tap is kept in the P x P window centred on the output
+# pixel's centre tap (P = 7, Fig. 5).
+def _off1(taps, K=3, G=1):
+    """One pixel's offsets [1, 1, 1, G, K*K, 2] with the given {tap: (dy, dx)} set."""
+    o = np.zeros((1, 1, 1, G, K * K, 2))
+    for k, d in taps.items():
+        o[0, 0, 0, 0, k] = d
+    return o
+
+
+@pytest.mark.parametrize("K,dil,P,tap,d,want", [
+    # hand-worked: tap (i, j) sits r = ((i-1)d, (j-1)d) from the centre tap; h = (P-1)/2
+    (3, 1, 7, 0, (-5.0, 2.5), (-2.0, 2.5)),     # r=(-1,-1): -6 -> -3 ; 1.5 inside
+    (3, 1, 7, 7, (2.5, -4.0), (2.0, -3.0)),     # r=(1,0): 3.5 -> 3 ; -4 -> -3
+    (3, 1, 7, 4, (0.25, 7.5), (0.25, 3.0)),     # centre tap: 7.5 -> 3
+    (3, 2, 7, 2, (-1.5, 0.5), (-1.0, 0.5)),     # dil 2, r=(-2, 2): -3.5 -> -3 ; 2.5 inside
+    (3, 1, 3, 0, (-0.5, 0.0), (0.0, 0.0)),      # P=3 (h=1), r=(-1,-1): -1.5 -> -1 ; -1 on the edge
+    (2, 1, 2, 0, (-1.0, 0.2), (0.0, 0.2)),      # even K: r=(-0.5,-0.5), h=0.5: -1.5 -> -0.5
+    (5, 1, 7, 24, (1.5, -9.0), (1.0, -5.0)),    # K=5, r=(2,2): 3.5 -> 3 ; -7 -> -3
+])
+def test_p15_bound_hand_values(oracle_mod, K, dil, P, tap, d, want):
+    out = oracle_mod.bound_offsets(_off1({tap: d}, K=K), P, K=K, dil=dil)
+    assert tuple(out[0, 0, 0, 0, tap]) == want
+
+
+def test_p15_unbounded_and_inside_are_identity(oracle_mod):
+    r = np.random.default_rng(15)
+    off = r.uniform(-9, 9, (2, 3, 4, 2, 9, 2))
+    assert np.array_equal(oracle_mod.bound_offsets(off, 0), off)          # P <= 0: unbounded
+    inside = r.uniform(-2, 2, (2, 3, 4, 2, 9, 2))                          # |r + d| <= 3 for K=3
+    assert np.array_equal(oracle_mod.bound_offsets(inside, 7), inside)
+    b = oracle_mod.bound_offsets(off, 7)
+    assert np.array_equal(oracle_mod.bound_offsets(b, 7), b)               # idempotent
+    assert np.isnan(oracle_mod.bound_offsets(np.full((1, 1, 9, 2), np.nan), 7)).all()
+
+
+@pytest.mark.parametrize("sign", [1, -1])
+def test_p15_far_offsets_sample_the_window_corner(oracle_mod, sign):
+    """Offsets of +-100 on every tap: bounded, every tap samples the window corner
+    (centre + sign*3, centre + sign*3) exactly, so y = b + sum_k sum_c W[o,k,c] m_k x[corner, c]
+    (0 outside the image) -- a closed form independent of the oracle's sampler."""
+    x, w, b, _, m, Ho, Wo = rand_layer(H=9, W=8, Cin=4, Cout=3, seed=15)
+    off = np.full((x.shape[0], Ho, Wo, 1, 9, 2), 100.0 * sign)
+    y = oracle_mod.dcn_forward(x, oracle_mod.bound_offsets(off, 7), w, b, mask=m)
+    ref = np.empty_like(y)
+    N, H, W, _ = x.shape
+    for n in range(N):
+        for ho in range(Ho):
+            for wo in range(Wo):
+                yy, xx = ho + 3 * sign, wo + 3 * sign         # centre tap (ho, wo) with pad 1
+                v = x[n, yy, xx] if (0 <= yy < H and 0 <= xx < W) else np.zeros(x.shape[3])
+                wm = np.einsum("okc,k->oc", w.reshape(w.shape[0], 9, -1), m[n, ho, wo, 0])
+                ref[n, ho, wo] = b + wm @ v
+    np.testing.assert_allclose(y, ref, rtol=0, atol=1e-12)
