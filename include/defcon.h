@@ -43,7 +43,7 @@
 extern "C" {
 #endif
 
-#define DEFCON_ABI_VERSION 1
+#define DEFCON_ABI_VERSION 2   /* 2: defcon_conv_t.bound */
 
 typedef enum {
     DEFCON_OK = 0,
@@ -85,6 +85,12 @@ typedef struct {
     int pad_h, pad_w;
     int dil_h, dil_w;
     int offset_groups;
+    /* Bounded deformation (section III-A-c; reading R12): P > 0 restricts every offset
+     * so that the sampling point of tap (i, j) stays in the P x P window centred on the output
+     * pixel's centre tap: per axis, with r = (i - (Kh-1)/2) * dil_h (resp. j, Kw, dil_w) and
+     * h = (P-1)/2, the offset d is used as clamp(r + d, -h, h) - r (NaN stays NaN).  The paper
+     * picks P = 7 (Fig. 5).  0 = unbounded.  Read by the DCN / columns calls only. */
+    int bound;
 } defcon_conv_t;
 
 /* Opaque texture plan: owns one layered cudaArray + texture object per image. */

@@ -45,7 +45,8 @@ class defcon_conv_t(ctypes.Structure):
     _fields_ = [("stride_h", ctypes.c_int), ("stride_w", ctypes.c_int),
                 ("pad_h", ctypes.c_int), ("pad_w", ctypes.c_int),
                 ("dil_h", ctypes.c_int), ("dil_w", ctypes.c_int),
-                ("offset_groups", ctypes.c_int)]
+                ("offset_groups", ctypes.c_int),
+                ("bound", ctypes.c_int)]   # bounded deformation P (R12); 0 = unbounded
 
 
 _lib = None
@@ -100,11 +101,11 @@ def _check(rc: int, where: str):
         raise DefconError(rc, where, load_library().defcon_last_error_detail().decode())
 
 
-def _conv(stride, pad, dil, groups) -> defcon_conv_t:
+def _conv(stride, pad, dil, groups, bound=0) -> defcon_conv_t:
     s = (stride, stride) if isinstance(stride, int) else tuple(stride)
     p = (pad, pad) if isinstance(pad, int) else tuple(pad)
     d = (dil, dil) if isinstance(dil, int) else tuple(dil)
-    return defcon_conv_t(s[0], s[1], p[0], p[1], d[0], d[1], int(groups))
+    return defcon_conv_t(s[0], s[1], p[0], p[1], d[0], d[1], int(groups), int(bound or 0))
 
 
 def _out(n, k, s, p, d):
@@ -215,8 +216,9 @@ def defcon_dcn_workspace_size(N, H, W, Cin, Cout, Kh, Kw, stride=1, pad=1, dil=1
 
 def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=1, offset_groups=1,
                        sampler="ldg", fp32_mode="simt", y=None, workspace=None, tex_plan=None,
-                       stream=None):
-    """Step 2 (Eq.2 P:58 + Eq.3): deformable conv forward, NHWC.  Returns y."""
+                       stream=None, bound=0):
+    """Step 2 (Eq.2 P:58 + Eq.3): deformable conv forward, NHWC.  Returns y.
+    bound = P > 0: bounded deformation (reading R12; the paper's P = 7)."""
     lib = load_library()
     _dev_tensor(x, "x")
     if x.dtype not in _DTYPES:
@@ -226,7 +228,7 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
     Cout, Kh, Kw, Cw = weight.shape
     if Cw != Cin:
         raise ValueError("weight Cin mismatch")
-    cv = _conv(stride, pad, dil, offset_groups)
+    cv = _conv(stride, pad, dil, offset_groups, bound)
     Ho, Wo = _out(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w)
     G = int(offset_groups)
     _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
@@ -252,7 +254,7 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
 
 
 def defcon_deform_columns(x, offset, mask, K=3, stride=1, pad=1, dil=1, offset_groups=1, columns=None,
-                          stream=None):
+                          stream=None, bound=0):
     """Sampling step alone (Eq.3 P:63-67 + mask, the "two-step" split P:69-76): returns the
     deformable columns [N*Ho*Wo, K*K*Cin] in x's dtype."""
     lib = load_library()
@@ -261,7 +263,7 @@ def defcon_deform_columns(x, offset, mask, K=3, stride=1, pad=1, dil=1, offset_g
         raise ValueError("x must be float32 or bfloat16")
     N, H, W, Cin = x.shape
     Kh, Kw = (K, K) if isinstance(K, int) else K
-    cv = _conv(stride, pad, dil, offset_groups)
+    cv = _conv(stride, pad, dil, offset_groups, bound)
     Ho, Wo = _out(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w)
     G = int(offset_groups)
     _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
@@ -291,7 +293,7 @@ def defcon_layer_workspace_size(N, H, W, Cin, Cout, K=3, stride=1, pad=1, dil=1,
 
 def defcon_layer_forward_host(x_host, branch, weight, bias, y_host, dev_workspace, K=3, stride=1,
                               pad=1, dil=1, offset_groups=1, modulated=True, sampler="ldg",
-                              fp32_mode="simt", stream=None):
+                              fp32_mode="simt", stream=None, bound=0):
     """Whole layer from pinned host x to pinned host y (H2D, step 1, step 2, D2H, sync).
 
     branch: dict of device tensors dw_w, dw_scale, dw_shift, pw_w, pw_b (resident weights).
@@ -305,7 +307,7 @@ def defcon_layer_forward_host(x_host, branch, weight, bias, y_host, dev_workspac
         _ptr(x_host), N, H, W, Cin, _DTYPES[x_host.dtype], _ptr(branch["dw_w"]),
         _ptr(branch["dw_scale"]), _ptr(branch["dw_shift"]), _ptr(branch["pw_w"]),
         _ptr(branch.get("pw_b")), _ptr(weight), _ptr(bias), Cout, K,
-        _conv(stride, pad, dil, offset_groups), int(modulated), _SAMPLERS[sampler],
+        _conv(stride, pad, dil, offset_groups, bound), int(modulated), _SAMPLERS[sampler],
         _FP32_MODES[fp32_mode], _ptr(y_host), _ptr(dev_workspace),
         dev_workspace.numel() * dev_workspace.element_size(), _stream_handle(stream))
     _check(rc, "defcon_layer_forward_host")

@@ -59,6 +59,7 @@ static int check_conv(const defcon_conv_t& cv) {
         return fail(DEFCON_ERR_INVALID_ARG, "stride and dilation must be positive");
     if (cv.pad_h < 0 || cv.pad_w < 0) return fail(DEFCON_ERR_INVALID_ARG, "padding must be >= 0");
     if (cv.offset_groups <= 0) return fail(DEFCON_ERR_INVALID_ARG, "offset_groups must be > 0");
+    if (cv.bound < 0) return fail(DEFCON_ERR_INVALID_ARG, "bound must be >= 0 (0 = unbounded)");
     return DEFCON_OK;
 }
 
@@ -79,6 +80,7 @@ static int make_geom(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
     g->dh = cv.dil_h; g->dw = cv.dil_w;
     g->G = cv.offset_groups;
     g->Cg = Cin / cv.offset_groups;
+    g->bound_h = cv.bound > 0 ? 0.5f * (float)(cv.bound - 1) : -1.f;
     g->KK = Kh * Kw;
     const long M = (long)N * g->Ho * g->Wo;
     if ((long)N * H * W * Cin >= (1L << 31) || M * Cout >= (1L << 31) ||

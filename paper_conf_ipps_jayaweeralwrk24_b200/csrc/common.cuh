@@ -77,6 +77,15 @@ DEFCON_DEVICE void mbar_wait(uint64_t* bar, uint32_t parity) {
     }
 }
 
+// ------------------------------------------------------------------ bounded deformation
+// P:182 (section III-A-c), reading R12: the offset d of a tap at regular displacement r from the
+// centre tap, restricted so that r + d stays in [-h, h] (the P x P window, h = (P-1)/2).
+// h < 0: unbounded.  A NaN offset stays NaN (the samplers turn it into zeros).
+DEFCON_DEVICE float bound_offset(float d, float r, float h) {
+    if (h < 0.f || d != d) return d;
+    return fminf(fmaxf(r + d, -h), h) - r;
+}
+
 // ------------------------------------------------------------------ fences
 // Make this thread's generic-proxy smem writes visible to the async proxy
 // (tcgen05.mma operand reads, TMA).

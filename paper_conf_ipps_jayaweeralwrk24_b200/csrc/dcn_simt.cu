@@ -80,8 +80,10 @@ __global__ void __launch_bounds__(THREADS) dcn_fwd_simt_kernel(const SimtArgs a)
                 const int ho = rem / g.Wo, wo = rem - (rem / g.Wo) * g.Wo;
                 const int i = tap / g.Kw, j = tap - (tap / g.Kw) * g.Kw;
                 const long pix = (long)m * g.G + grp;
-                const float dy = a.offset[(pix * g.KK + tap) * 2];
-                const float dx = a.offset[(pix * g.KK + tap) * 2 + 1];
+                const float dy = bound_offset(a.offset[(pix * g.KK + tap) * 2], (i - 0.5f * (g.Kh - 1)) * g.dh,
+                                              g.bound_h);   // bounded deformation (R12)
+                const float dx = bound_offset(a.offset[(pix * g.KK + tap) * 2 + 1], (j - 0.5f * (g.Kw - 1)) * g.dw,
+                                              g.bound_h);
                 const float mk = a.mask ? a.mask[pix * g.KK + tap] : 1.f;
                 float py = (float)(ho * g.sh - g.ph + i * g.dh) + dy;
                 float px = (float)(wo * g.sw - g.pw + j * g.dw) + dx;
@@ -219,10 +221,12 @@ __global__ void __launch_bounds__(THREADS, 2) dcn_fwd_f32_tiled_kernel(const Sim
                 for (int q = 0; q < 4; ++q) { off[q] = 0; wt[q] = 0.f; }
                 if (gok) {
                     const long pix = (long)gm * g.G + grp;
-                    const float dy = __ldg(a.offset + (pix * g.KK + tap) * 2);
-                    const float dx = __ldg(a.offset + (pix * g.KK + tap) * 2 + 1);
-                    const float mk = a.mask ? __ldg(a.mask + pix * g.KK + tap) : 1.f;
                     const int i = tap / g.Kw, j = tap - (tap / g.Kw) * g.Kw;
+                    const float dy = bound_offset(__ldg(a.offset + (pix * g.KK + tap) * 2),
+                                                  (i - 0.5f * (g.Kh - 1)) * g.dh, g.bound_h);   // P:182, R12
+                    const float dx = bound_offset(__ldg(a.offset + (pix * g.KK + tap) * 2 + 1),
+                                                  (j - 0.5f * (g.Kw - 1)) * g.dw, g.bound_h);
+                    const float mk = a.mask ? __ldg(a.mask + pix * g.KK + tap) : 1.f;
                     float py = (float)(gyb + i * g.dh) + dy;
                     float px = (float)(gxb + j * g.dw) + dx;
                     py = fminf(fmaxf(py, -2.f), (float)g.H + 1.f);

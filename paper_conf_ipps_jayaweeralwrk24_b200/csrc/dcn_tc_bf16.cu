@@ -94,6 +94,7 @@ struct TcArgs {
     int H, W, Cin, Cout, Kw, Ho, Wo;
     int sh, sw, ph, pw, dh, dw;
     int G, Cg, M, KK;
+    float bound_h;         // bounded deformation half-window (R12); < 0: unbounded
     int ipt;               // k-iterations per tile = (Cin / CPI) * KK
     int es, cpi;           // element bytes, channels per k-iteration
     int n_tiles_n;         // tiles along Cout
@@ -181,7 +182,12 @@ __device__ __forceinline__ RowPos row_pos(const TcArgs& a, int m) {
 
 __device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& rp, int i, int j, const MetaIn& in,
                                                  uint8_t* e, bool tex_row) {
-    const float2 d = in.d;
+    float2 d = in.d;
+    if (a.bound_h >= 0.f) {   // bounded deformation (R12)
+        const int Kh = a.KK / a.Kw;
+        d.x = bound_offset(d.x, (i - 0.5f * (Kh - 1)) * a.dh, a.bound_h);
+        d.y = bound_offset(d.y, (j - 0.5f * (a.Kw - 1)) * a.dw, a.bound_h);
+    }
     const float mk = in.mk;
     if (tex_row) {
         // texture sampler: unnormalised texel coordinates (texel centres at +0.5, R7) in the
@@ -1235,6 +1241,7 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.H = g.H; a.W = g.W; a.Cin = g.Cin; a.Cout = g.Cout; a.Kw = g.Kw; a.Ho = g.Ho; a.Wo = g.Wo;
     a.sh = g.sh; a.sw = g.sw; a.ph = g.ph; a.pw = g.pw; a.dh = g.dh; a.dw = g.dw;
     a.G = g.G; a.Cg = g.Cg; a.M = g.M; a.KK = g.KK;
+    a.bound_h = g.bound_h;
     a.ipt = plan.ipt;
     a.n_tiles_n = plan.n_tiles_n;
     a.total_iters = plan.total;

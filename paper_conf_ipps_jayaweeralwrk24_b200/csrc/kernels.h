@@ -16,6 +16,7 @@ struct DcnGeom {
     int G, Cg;   // offset groups, channels per group
     int M;       // N * Ho * Wo output pixels
     int KK;      // Kh * Kw taps
+    float bound_h;   // bounded deformation half-window (P-1)/2 (R12); < 0: unbounded
 };
 
 struct DcnPtrs {

@@ -27,6 +27,7 @@ struct ColArgs {
     int H, W, Cin, Kw, Ho, Wo;
     int sh, sw, ph, pw, dh, dw;
     int G, Cg, M, KK;
+    float bound_h;       // bounded deformation half-window (R12); < 0: unbounded
     int pieces;          // 32-byte pieces per (pixel, tap) row = Cin * ES / 32
     long long total;     // M * KK * pieces
 };
@@ -56,7 +57,9 @@ __device__ __forceinline__ void piece_issue(const ColArgs& a, long long u, Piece
     const int wo = rem - ho * a.Wo;
     const int i = k / a.Kw, j = k - (k / a.Kw) * a.Kw;
     const long pix = (long)m * a.G + g;
-    const float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + k) * 2));
+    float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + k) * 2));
+    d.x = bound_offset(d.x, (i - 0.5f * (a.KK / a.Kw - 1)) * a.dh, a.bound_h);   // P:182, R12
+    d.y = bound_offset(d.y, (j - 0.5f * (a.Kw - 1)) * a.dw, a.bound_h);
     const float mv = a.mask ? __ldg(a.mask + pix * a.KK + k) : 1.f;
     float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
     float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
@@ -178,7 +181,9 @@ __device__ __forceinline__ void row_issue(const ColArgs& a, int r, int piece, co
     const int ho = rem / a.Wo;
     const int wo = rem - ho * a.Wo;
     const int i = k / a.Kw, j = k - (k / a.Kw) * a.Kw;
-    const float2 d = rm.d;
+    float2 d = rm.d;
+    d.x = bound_offset(d.x, (i - 0.5f * (a.KK / a.Kw - 1)) * a.dh, a.bound_h);   // P:182, R12
+    d.y = bound_offset(d.y, (j - 0.5f * (a.Kw - 1)) * a.dw, a.bound_h);
     const float mv = rm.mv;
     float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
     float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
@@ -242,6 +247,7 @@ cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* 
     a.H = g.H; a.W = g.W; a.Cin = g.Cin; a.Kw = g.Kw; a.Ho = g.Ho; a.Wo = g.Wo;
     a.sh = g.sh; a.sw = g.sw; a.ph = g.ph; a.pw = g.pw; a.dh = g.dh; a.dw = g.dw;
     a.G = g.G; a.Cg = g.Cg; a.M = g.M; a.KK = g.KK;
+    a.bound_h = g.bound_h;
     a.pieces = g.Cin * (bf16 ? 2 : 4) / 32;
     a.total = (long long)g.M * g.KK * a.pieces;
     int dev = 0, nsm = 148;

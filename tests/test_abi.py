@@ -36,14 +36,14 @@ def test_header_symbols_exported(lib):
 
 
 def test_status_strings(lib):
-    assert lib.defcon_abi_version() == 1
+    assert lib.defcon_abi_version() == 2
     assert lib.defcon_status_string(0) == b"DEFCON_OK"
     assert lib.defcon_status_string(5) == b"DEFCON_ERR_LIMIT"
 
 
 def _conv(**kw):
     from paper_conf_ipps_jayaweeralwrk24_b200._binding import defcon_conv_t
-    d = dict(stride_h=1, stride_w=1, pad_h=1, pad_w=1, dil_h=1, dil_w=1, offset_groups=1)
+    d = dict(stride_h=1, stride_w=1, pad_h=1, pad_w=1, dil_h=1, dil_w=1, offset_groups=1, bound=0)
     d.update(kw)
     return defcon_conv_t(**d)
 
@@ -69,9 +69,10 @@ def _fwd(lib, x=FAKE, N=2, H=8, W=8, Cin=64, off=FAKE, mask=FAKE, w=FAKE, b=FAKE
     (dict(x=FAKE + 8), 3), (dict(mask=FAKE + 4), 3), (dict(w=FAKE + 2), 3),
     (dict(x=FAKE + 16), 3),               # tensor-core path: x is gathered in 32-byte vectors
     (dict(cv="g16_bf16"), 2),             # Cin/G = 4, not a multiple of 8 for bf16
+    (dict(cv="neg_bound"), 1),            # bounded deformation P must be >= 0
 ])
 def test_dcn_forward_validation(lib, kw, status):
-    cvs = {"g3": _conv(offset_groups=3), "s0": _conv(stride_h=0),
+    cvs = {"g3": _conv(offset_groups=3), "s0": _conv(stride_h=0), "neg_bound": _conv(bound=-1),
            "tiny": _conv(pad_h=0, pad_w=0), "g16_bf16": _conv(offset_groups=16)}
     if kw.get("cv") in cvs:
         name = kw.pop("cv")

@@ -605,3 +605,72 @@ def test_unfused_columns_gemm_matches_fused(oracle_mod, d, dev):
     ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"]).reshape(-1, c.Cout)
     assert normwise(y2.cpu().numpy(), ref) < REG["bf16"]
     assert normwise(y1.float().cpu().numpy().reshape(-1, c.Cout), ref) < REG["bf16"]
+
+
+# ---------------------------------------------------------------- bounded deformation (NEXT 2)
+# P:182 (section III-A-c), reading R12, P = 7: every kernel clamps the sampling points into the
+# P x P window around the centre tap; the oracle applies bound_offsets (pinned, P15) and then the
+# plain DCN.  Offsets U(-7, 7) (off_dist "local") put most taps outside the window.
+BOUNDED = [
+    (small("bnd_tc_g1", N=1, H=21, W=19), "ldg", "simt"),
+    (small("bnd_tc_g2_dil2", N=1, G=2, dil=2, pad=2, H=17, W=23), "ldg", "simt"),
+    (small("bnd_tc_s2_v1", N=1, stride=2, modulated=False, H=25, W=21), "ldg", "simt"),
+    (small("bnd_tex", N=1, Cin=64, Cout=64, H=21, W=19), "tex", "simt"),
+    (small("bnd_f32_simt", N=1, dtype="f32", Cin=32, Cout=40), "ldg", "simt"),
+    (small("bnd_f32_3xtf32", N=1, dtype="f32", Cin=64, Cout=64), "ldg", "3xtf32"),
+]
+
+
+@pytest.mark.parametrize("c,sampler,fp32_mode", BOUNDED, ids=lambda v: v.name if hasattr(v, "name") else str(v))
+@pytest.mark.parametrize("P", [7, 3])
+def test_dcn_bounded_parity(oracle_mod, d, dev, c, sampler, fp32_mode, P):
+    L = inputs.gen_layer(c, off_dist="local")
+    dt = TDT[c.dtype]
+    plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler == "tex" else None
+    y = d.defcon_dcn_forward(to_dev(L["x"], dt, dev), to_dev(L["offset"], torch.float32, dev),
+                             to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], dt, dev),
+                             to_dev(L["bias"], torch.float32, dev), stride=c.stride, pad=c.pad, dil=c.dil,
+                             offset_groups=c.G, sampler=sampler, fp32_mode=fp32_mode, tex_plan=plan,
+                             bound=P).float().cpu().numpy()
+    ob = oracle_mod.bound_offsets(L["offset"], P, K=c.K, dil=c.dil)
+    ref = oracle_mod.dcn_forward(L["x"], ob, L["weight"], L["bias"], mask=L["mask"], stride=c.stride,
+                                 pad=c.pad, dil=c.dil, G=c.G)
+    unb = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"],
+                                 stride=c.stride, pad=c.pad, dil=c.dil, G=c.G)
+    if sampler == "tex":   # the texture-model oracle on the bounded offsets (R14)
+        ref = oracle_mod.dcn_forward_texq(inputs.round_to(L["x"], "f16"), ob, L["weight"], L["bias"],
+                                          mask=L["mask"], stride=c.stride, pad=c.pad, dil=c.dil, G=c.G,
+                                          quant="hw")
+    err = normwise(y, ref)
+    print(f"{c.name} P={P}: normwise error {err:.3e} (bounded vs unbounded oracle differ by "
+          f"{normwise(unb, ref):.2e})")
+    assert normwise(unb, ref) > 10 * REG[c.dtype]   # the bound is active
+    assert err < REG[c.dtype]
+
+
+def test_dcn_bounded_full_size_sampled(oracle_mod, d, dev):
+    """Bounded (P = 7) at the full C4 shape, sampled output pixels."""
+    c = configs.C4
+    L = inputs.gen_layer(c, off_dist="local")
+    y = d.defcon_dcn_forward(to_dev(L["x"], torch.bfloat16, dev), to_dev(L["offset"], torch.float32, dev),
+                             to_dev(L["mask"], torch.float32, dev), to_dev(L["weight"], torch.bfloat16, dev),
+                             to_dev(L["bias"], torch.float32, dev), bound=7).float().cpu().numpy()
+    y = y.reshape(c.M, c.Cout)
+    r = np.random.default_rng(9)
+    idx = np.unique(np.concatenate([np.arange(0, 130), np.arange(c.M - 130, c.M), r.integers(0, c.M, 300)]))
+    ob = oracle_mod.bound_offsets(L["offset"], 7)
+    ref = oracle_mod.dcn_pixels(L["x"], ob, L["weight"], idx, L["bias"], mask=L["mask"])
+    assert normwise(y[idx], ref) < REG["bf16"]
+
+
+def test_deform_columns_bounded(oracle_mod, d, dev):
+    c = small("cols_bnd", Cin=64, N=1)
+    L = inputs.gen_layer(c, off_dist="local")
+    cols = d.defcon_deform_columns(to_dev(L["x"], torch.bfloat16, dev), to_dev(L["offset"], torch.float32, dev),
+                                   to_dev(L["mask"], torch.float32, dev), K=3, bound=7)
+    torch.cuda.synchronize()
+    idx = np.arange(c.M)
+    ref = oracle_mod.deform_columns(L["x"], oracle_mod.bound_offsets(L["offset"], 7), 3, pix_idx=idx,
+                                    mask=L["mask"])
+    g = cols.float().cpu().numpy()
+    assert np.all(np.abs(g - ref) <= 2.0 ** -8 * np.abs(ref) + 1e-6 * np.max(np.abs(ref)))

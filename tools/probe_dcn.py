@@ -15,6 +15,9 @@ from defcon_workloads import configs, inputs  # noqa: E402
 import paper_conf_ipps_jayaweeralwrk24_b200 as d  # noqa: E402
 
 
+BOUND = int(os.environ.get("PROBE_BOUND", "0"))   # bounded deformation P (0 = unbounded)
+
+
 def time_cfg(c, sampler, reps=200):
     """sampler: ldg / tex / hybrid, or (fp32 configs) the fp32 mode simt / 3xtf32."""
     fp32_mode = sampler if sampler in ("simt", "3xtf32") else "simt"
@@ -35,7 +38,7 @@ def time_cfg(c, sampler, reps=200):
     plan = d.TexPlan(c.N, c.H, c.W, c.Cin, dt) if sampler in ("tex", "hybrid") else None
     fn = lambda: d.defcon_dcn_forward(x, off, msk, w, b, stride=c.stride, pad=c.pad, dil=c.dil,
                                       offset_groups=c.G, y=y, workspace=ws, sampler=sampler,
-                                      tex_plan=plan, fp32_mode=fp32_mode)
+                                      tex_plan=plan, fp32_mode=fp32_mode, bound=BOUND)
     for _ in range(5):
         fn()
     g = torch.cuda.CUDAGraph()
