@@ -322,8 +322,8 @@ cudaError_t launch_dcn_simt(const DcnGeom& g, const DcnPtrs& p, bool bf16, cudaS
     SimtArgs a{p.x, p.offset, p.mask, p.weight, p.bias, p.y, g};
     // fp32: the register-tiled kernel when the 16-channel steps stay inside one tap and one offset
     // group and the 16-byte vector loads are aligned (Cin, Cg multiples of 16; Cout multiple of 4);
-    // DEFCON_F32_ANCHOR=1 selects the simple anchor kernel below (A/B and tests).
-    if (!bf16 && g.Cin % FT_K == 0 && g.Cg % FT_K == 0 && g.Cout % 4 == 0 && !getenv("DEFCON_F32_ANCHOR")) {
+    // otherwise the simple anchor kernel below.
+    if (!bf16 && g.Cin % FT_K == 0 && g.Cg % FT_K == 0 && g.Cout % 4 == 0) {
         dim3 grid((g.M + FT_M - 1) / FT_M, (g.Cout + FT_N - 1) / FT_N);
         dcn_fwd_f32_tiled_kernel<<<grid, THREADS, 0, stream>>>(a);
         return cudaGetLastError();

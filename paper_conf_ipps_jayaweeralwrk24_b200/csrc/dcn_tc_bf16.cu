@@ -888,6 +888,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
         // segment's epilogue, which would otherwise be exposed at the end of the CTA's range.
+        // Its store scratch reuses the A stages other producer threads wrote: ordered already
+        // through full_a -> MMA -> tmem_full, a barrier the race checker can see makes it explicit.
+        named_bar_sync(1, NPT);
         if (nseg > 0) {
             const int o = nseg - 1;
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));

@@ -48,23 +48,6 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
                                          const float* pw_w, const float* pw_b, int n_off, int n_msk,
                                          int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                          float* offset, float* mask, void* ws, cudaStream_t stream);
-// single-launch branch: dw on CUDA cores -> t in smem -> 1x1 on tcgen05 (3xTF32)
-bool offset_branch_tc_supported(int C, int OC);
-cudaError_t launch_offset_branch_tc(const void* x, bool x_bf16, int N, int H, int W, int C,
-                                    const float* dw_w, const float* dw_scale, const float* dw_shift,
-                                    const float* pw_w, const float* pw_b, int n_off, int n_msk,
-                                    int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                    float* offset, float* mask, cudaStream_t stream);
-
-// single-launch branch, one output row per CTA: TMA-staged dw on CUDA cores -> t as tf32 hi/lo
-// operand planes in smem -> 1x1 on tcgen05 3xTF32 (offset_branch_fused.cu)
-bool offset_branch_fused_supported(int C, int OC, int Wo, int sw, int dw, int dh, bool x_bf16);
-cudaError_t launch_offset_branch_fused(const void* x, bool x_bf16, int N, int H, int W, int C,
-                                       const float* dw_w, const float* dw_scale, const float* dw_shift,
-                                       const float* pw_w, const float* pw_b, int n_off, int n_msk,
-                                       int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho,
-                                       int Wo, float* offset, float* mask, cudaStream_t stream);
-
 // ---- sampling step alone: deformable columns [M][KK*Cin] (sampler.cu)
 cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* offset, const float* mask,
                                   bool bf16, void* cols, cudaStream_t stream);

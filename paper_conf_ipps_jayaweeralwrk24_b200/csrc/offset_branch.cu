@@ -507,8 +507,9 @@ static size_t two_pass_workspace(int M, int C) { return (2 * (size_t)M * C + 2 *
 
 static bool use_onepass(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph, int pw,
                         int dh, int dw, bool x_bf16) {
-    const char* impl = getenv("DEFCON_OFFSET_IMPL");
-    if (impl && !strcmp(impl, "two_pass")) return false;
+#ifdef DEFCON_DEV_TWO_PASS   // dev builds (tools/build_variants.py): time the two-launch path
+    return false;
+#endif
     return offset_branch_onepass_plan(N, H, W, C, Ho, Wo, sh, sw, ph, pw, dh, dw, 3 * G * K * K, x_bf16);
 }
 
@@ -534,24 +535,14 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     a.n_msk = with_mask ? G * K * K : 0;
     a.OC = a.n_off + a.n_msk;
     if (a.OC > 256) return cudaErrorInvalidValue;   // api.cu maps this to DEFCON_ERR_LIMIT
-    // Two launches by default (measured fastest at the YOLACT++ shapes).
-    // DEFCON_OFFSET_IMPL=tc (or DEFCON_OFFSET_TC=1) selects the single-launch tcgen05 branch
-    // (offset_branch_tc.cu: t stays on chip), =row_tc the row-tile kernel with TMA-staged input
-    // (offset_branch_fused.cu).  All three are parity-tested.
+    // One pass per pixel tile (offset_branch_onepass.cu) wherever it tiles; the two-launch path
+    // (dw kernel -> t in HBM -> 1x1 kernel) covers input rows wider than its TMA box.
     if (use_onepass(N, H, W, C, Ho, Wo, K, G, s_h, s_w, p_h, p_w, d_h, d_w, x_bf16))
         return launch_offset_branch_onepass(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
                                             a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
                                             mask, t_ws, stream);
-    const char* impl = getenv("DEFCON_OFFSET_IMPL");
-    if (((impl && !strcmp(impl, "tc")) || getenv("DEFCON_OFFSET_TC")) && offset_branch_tc_supported(C, a.OC))
-        return launch_offset_branch_tc(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b, a.n_off,
-                                       a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset, mask, stream);
-    if (impl && !strcmp(impl, "row_tc") && offset_branch_fused_supported(C, a.OC, Wo, s_w, d_w, d_h, x_bf16))
-        return launch_offset_branch_fused(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
-                                          a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
-                                          mask, stream);
     // 1x1 on tcgen05 from TMA-loaded hi / lo planes, or the mma.sync 3xTF32 kernel (t in one
-    // plane; DEFCON_PW_MMA=1 or DEFCON_PW_IMPL=mma forces it)
+    // plane)
     // The tcgen05 kernel runs one 128-pixel tile per CTA, two CTAs per SM, each CTA a latency
     // chain over the channel chunks: it wins when its tiles fill whole rounds of CTAs, so a grid
     // whose last round would hold a few stragglers (C3: 298 tiles for 296 slots) keeps mma.sync.
@@ -564,9 +555,7 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     const int pw_tiles = (a.M + 127) / 128, pw_slots = 2 * sms;
     const int pw_rounds = (pw_tiles + pw_slots - 1) / pw_slots;
     const bool pw_fill = pw_rounds == 1 || pw_tiles - (pw_rounds - 1) * pw_slots >= pw_slots / 2;
-    const char* pw_env = getenv("DEFCON_PW_IMPL");   // "mma" / "tc" force a kernel
-    const bool pw_tc = C % 4 == 0 && get_encode_tiled() != nullptr && !getenv("DEFCON_PW_MMA") &&
-                       (pw_env ? !strcmp(pw_env, "tc") : pw_fill);
+    const bool pw_tc = C % 4 == 0 && get_encode_tiled() != nullptr && pw_fill;
     a.OCN = pw_tc_ocn(a.OC);
     if (pw_tc) {
         a.t_lo = t_ws + (size_t)a.M * C;

@@ -257,7 +257,7 @@ cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* 
     const int grid = (int)(blocks < (long long)nsm * 8 ? blocks : (long long)nsm * 8);
     // row-mapped kernel when a row is 8 / 16 / 32 pieces and every index fits 32 bits
     const bool rows32 = (long long)g.M * g.KK * g.Cin < (1ll << 31) &&
-                        (long long)g.N * g.H * g.W * g.Cin < (1ll << 31) && !getenv("DEFCON_COLUMNS_PIECEWISE");
+                        (long long)g.N * g.H * g.W * g.Cin < (1ll << 31);
     if (rows32 && (a.pieces == 8 || a.pieces == 16 || a.pieces == 32)) {
         auto pick = [&](auto kb, auto kf) { return bf16 ? kb : kf; };
         void (*kern)(ColArgs) =

@@ -114,18 +114,6 @@ def test_dcn_kernel_sizes(oracle_mod, d, dev, c):
     assert normwise(y, ref) < REG[c.dtype]
 
 
-def test_dcn_f32_anchor_matches_tiled(oracle_mod, d, dev, monkeypatch):
-    """The simple fp32 anchor kernel (DEFCON_F32_ANCHOR=1) and the register-tiled fp32 kernel
-    both reach fp32 accuracy against the oracle on the same inputs."""
-    c = small("f32_anchor", dtype="f32", Cin=32, Cout=40)
-    L = inputs.gen_layer(c)
-    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"])
-    y_tiled = run_dcn(d, dev, c, L)
-    monkeypatch.setenv("DEFCON_F32_ANCHOR", "1")
-    y_anchor = run_dcn(d, dev, c, L)
-    assert normwise(y_tiled, ref) < 1e-5 and normwise(y_anchor, ref) < 1e-5
-
-
 @pytest.mark.parametrize("dist", ["zeros", "integer", "half", "far", "border", "local"])
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 def test_dcn_special_offsets(oracle_mod, d, dev, dist, dtype):
@@ -375,18 +363,19 @@ def gen_branch_dev(c, dev):
     return P, {k: to_dev(v, torch.float32, dev) for k, v in P.items()}
 
 
-@pytest.mark.parametrize("path", ["row_tc", "tc", "two_pass", "two_pass_pw_tc", "two_pass_pw_mma"])
 @pytest.mark.parametrize("c", [configs.C3.replace(N=2), configs.C4_G4.replace(N=2),
                                small("branch_s2_f32", dtype="f32", stride=2, Cin=48, modulated=False),
                                small("branch_d2", dil=2, pad=2, Cin=40, H=15, W=23),
-                               configs.C5.replace(N=1), configs.C4],
+                               configs.C5.replace(N=1), configs.C4,
+                               # rows wider than the one-pass TMA box (256 columns): the two-launch
+                               # path, its 1x1 on tcgen05 (150 tiles: one full round) ...
+                               small("branch_wide_pw_tc", Cin=16, N=1, H=64, W=300),
+                               # ... and on mma.sync (300 tiles: a 2nd round of 4 stragglers)
+                               small("branch_wide_pw_mma", Cin=16, N=1, H=128, W=300, modulated=False)],
                          ids=lambda c: c.name)
-def test_offset_branch_parity(oracle_mod, d, dev, monkeypatch, c, path):
-    """All three branch kernels vs the oracle: the default two-launch path ("two_pass"), the
-    single-launch tcgen05 kernel ("tc") and the TMA-staged row-tile kernel ("row_tc")."""
-    monkeypatch.setenv("DEFCON_OFFSET_IMPL", path.split("_pw_")[0])
-    if "_pw_" in path:   # the two-launch path's 1x1: tcgen05 from hi / lo planes, or mma.sync
-        monkeypatch.setenv("DEFCON_PW_IMPL", path.split("_pw_")[1])
+def test_offset_branch_parity(oracle_mod, d, dev, c):
+    """The branch kernels vs the oracle: the one-pass kernel wherever it tiles, the two-launch
+    path (dw kernel, t in HBM, 1x1 on tcgen05 or mma.sync) for wide rows."""
     x = inputs.gen_x(c)
     P, Pd = gen_branch_dev(c, dev)
     off, msk = d.defcon_offset_dw_conv(to_dev(x, TDT[c.dtype], dev), Pd["dw_w"], Pd["dw_scale"],

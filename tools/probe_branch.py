@@ -1,8 +1,10 @@
 """Time the lightweight offset branch (defcon_offset_dw_conv) alone, graph-replayed, per config.
 
   python tools/probe_branch.py [config,...]
-Prints one JSON line per (config, path): the default one-pass kernel ("onepass") and the
-two-launch path ("two_pass", dw kernel + 1x1 kernel through an HBM intermediate).
+Prints one JSON line per config for the loaded library ("path" = PROBE_PATH, default
+"onepass"); the two-launch path (dw kernel + 1x1 kernel through an HBM intermediate) is timed
+with a dev build: python tools/build_variants.py two_pass=-DDEFCON_DEV_TWO_PASS, then
+DEFCON_LIB=tools/bin/libdefcon_two_pass.so PROBE_PATH=two_pass python tools/probe_branch.py
 """
 import json
 import os
@@ -50,10 +52,7 @@ if __name__ == "__main__":
     d.load_library()
     for n in names:
         c = configs.SINGLE_LAYER[n] if n in configs.SINGLE_LAYER else {l.name: l for l in configs.stack_layers(64)}[n]
-        for path in ("onepass", "two_pass"):
-            os.environ["DEFCON_OFFSET_IMPL"] = path
-            us = time_branch(c)
-            byt = configs.offset_branch_compulsory_bytes(c)
-            print(json.dumps({"config": n, "path": path, "us": round(us, 2),
-                              "GB/s(compulsory)": round(byt / (us * 1e-6) / 1e9, 1)}))
-    os.environ.pop("DEFCON_OFFSET_IMPL", None)
+        us = time_branch(c)
+        byt = configs.offset_branch_compulsory_bytes(c)
+        print(json.dumps({"config": n, "path": os.environ.get("PROBE_PATH", "onepass"), "us": round(us, 2),
+                          "GB/s(compulsory)": round(byt / (us * 1e-6) / 1e9, 1)}))

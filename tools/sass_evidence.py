@@ -16,8 +16,8 @@ OPS = {  # SASS mnemonic (as the first token of the instruction) -> meaning
     "FFMA2": "packed fp32 FMA", "FFMA": "fp32 FMA", "TEX": "texture fetch",
 }
 KERNELS = ["dcn_fwd_bf16_tc_kernel", "pw_tc_kernel", "pw_sigmoid_kernel", "dw_bn_relu_kernel",
-           "dcn_fwd_f32_tiled_kernel", "deform_columns_rows_kernel", "offset_branch_tc_kernel",
-           "offset_branch_row_tc_kernel", "dcn_fwd_simt_kernel"]
+           "dcn_fwd_f32_tiled_kernel", "deform_columns_rows_kernel", "offset_branch_onepass_kernel",
+           "dcn_fwd_simt_kernel"]
 
 sass = subprocess.run(["cuobjdump", "-sass", LIB], capture_output=True, text=True).stdout
 stats, cur = collections.OrderedDict(), None
