@@ -121,7 +121,11 @@ struct TcCfg {
     static constexpr int A_STAGE_BYTES = Elem<F32>::A_STAGE;
     static constexpr int STAGE_BYTES = A_STAGE_BYTES + B_STAGE_BYTES;
     static constexpr int NBUF = BLOCK_N <= 256 ? 2 : 1;      // TMEM accumulator buffers
-    static constexpr int TMEM_COLS = (BLOCK_N * NBUF) < 32 ? 32 : BLOCK_N * NBUF;
+    // F32: two accumulators per buffer -- hi*hi, and the small cross terms lo*hi + hi*lo in
+    // their own (ACC_STRIDE = BLOCK_N columns further) -- summed in the epilogue
+    static constexpr int NACC = F32 ? 2 : 1;
+    static constexpr int ACC_STRIDE = BLOCK_N * NACC;      // columns per accumulator buffer
+    static constexpr int TMEM_COLS = (ACC_STRIDE * NBUF) < 32 ? 32 : ACC_STRIDE * NBUF;
     static constexpr int TMA_BOX_N = B_ROWS > 256 ? 256 : B_ROWS;
 };
 
@@ -561,6 +565,13 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
         for (int c = col0; c < col0 + NCOLS; c += CH) {
             uint32_t v[CH];
             tmem_ld_32x32b_x16(tacc + c, v);
+            if (F32) {   // + the cross-term accumulator
+                uint32_t vx[CH];
+                tmem_ld_32x32b_x16(tacc + BLOCK_N + c, vx);
+                tmem_ld_wait();
+#pragma unroll
+                for (int u = 0; u < CH; ++u) v[u] = __float_as_uint(__uint_as_float(v[u]) + __uint_as_float(vx[u]));
+            }
             tmem_ld_wait();
 #pragma unroll
             for (int u = 0; u < CH / 4; ++u)
@@ -579,6 +590,13 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
         uint32_t v[CS];
         if (own_from_tmem) {
             tmem_ld_32x32b_x32(tacc + c, v);
+            if (F32) {   // + the cross-term accumulator
+                uint32_t vx[CS];
+                tmem_ld_32x32b_x32(tacc + BLOCK_N + c, vx);
+                tmem_ld_wait();
+#pragma unroll
+                for (int u = 0; u < CS; ++u) v[u] = __float_as_uint(__uint_as_float(v[u]) + __uint_as_float(vx[u]));
+            }
             tmem_ld_wait();
         }
         if (n0 + c >= a.Cout) return;      // warp-uniform
@@ -899,7 +917,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             tc_fence_after();
             const int qd = warp & 3;
             const int r = qd * 32 + lane;
-            const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
+            const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * Cfg::ACC_STRIDE);
             constexpr int SLICE = BLOCK_N / (NPW / 4);
             if (t == 0) TL(12);
             // idle pipeline buffers: A stages hold the per-warp store scratch, B stages the
@@ -919,7 +937,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const int buf = o % Cfg::NBUF;
             mbar_wait(&tmem_full[buf], (uint32_t)(o / Cfg::NBUF) & 1u);
             tc_fence_after();
-            const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * BLOCK_N);
+            const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * Cfg::ACC_STRIDE);
             epilogue_segment<BLOCK_N, BLOCK_N, PAIR, F32>(a, &ymap, sg, tacc, r, 0, 2, 128,
                                                     threadIdx.x == EPI_WARP0 * 32, fix_flag, T, nct,
                                                     a.bias_in_smem ? bias_s : nullptr,
@@ -979,7 +997,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 if (PAIR) mbar_wait_cluster(&tmem_empty[buf], ((uint32_t)(o / Cfg::NBUF) & 1u) ^ 1u);
                 else mbar_wait(&tmem_empty[buf], ((uint32_t)(o / Cfg::NBUF) & 1u) ^ 1u);
                 tc_fence_after();
-                const uint32_t d_base = tmem_base + (uint32_t)(buf * BLOCK_N);
+                const uint32_t d_base = tmem_base + (uint32_t)(buf * Cfg::ACC_STRIDE);
                 for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
                     const int s = q % STAGES;
                     const uint32_t ph = (uint32_t)(q / STAGES) & 1u;
@@ -1004,13 +1022,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                             const uint64_t bdesc =
                                 make_sw128_desc(b_addr + h * Cfg::UMMA_N * 128 + kk * 32);
                             const uint32_t acc = (kt != sg.kb || kk != 0) ? 1u : 0u;
-                            if (F32) {   // 3xTF32: lo*hi + hi*lo + hi*hi
+                            if (F32) {   // 3xTF32: lo*hi + hi*lo into the cross accumulator, hi*hi
+                                // into the main one (each MMA rounds its accumulator: the
+                                // tiny cross terms no longer cost the main sum two roundings)
                                 const uint64_t adesc_lo = make_sw128_desc(a_addr + A_PLANE + kk * 32);
                                 const uint64_t bdesc_lo =
                                     make_sw128_desc(b_addr + Cfg::B_PLANE + h * Cfg::UMMA_N * 128 + kk * 32);
-                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc_lo, bdesc, idesc, acc);
-                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc_lo, idesc, 1u);
-                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, 1u);
+                                const uint32_t dx = d_base + BLOCK_N + h * Cfg::UMMA_N;
+                                mma_tf32_ss(dx, adesc_lo, bdesc, idesc, acc);
+                                mma_tf32_ss(dx, adesc, bdesc_lo, idesc, 1u);
+                                mma_tf32_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, acc);
                             } else if (PAIR) {
                                 mma_bf16_ss_pair(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, acc);
                             } else {
