@@ -1073,6 +1073,47 @@ int num_sms() {
     return n;
 }
 
+// ---- schedule tuning (SURVEY NEXT 3, P:276 / P:286: the paper tunes its tile size per layer).
+// tools/autotune.py times every (BLOCK_N, CTA pair, grid cap) candidate per layer shape and per
+// per-GPU batch and writes the winners to tuning_table.inc, compiled in here.  Shapes not in
+// the table take the defaults (BLOCK_N from Cout, single CTAs, a full persistent grid).
+// DEFCON_BLOCK_N / DEFCON_DCN_PAIR / DEFCON_MAX_CTAS override the table (the sweep, tests).
+struct TcTuning {
+    int block_n;    // 0: from Cout
+    int pair;       // -1: default (single CTAs); 0 / 1 (BLOCK_N = 256 only)
+    int max_ctas;   // 0: every SM
+};
+struct TuneEntry {
+    int Cin, Cout, H, W, stride, G, nmin, nmax;
+    TcTuning t;
+};
+static const TuneEntry kTuneTable[] = {
+#include "tuning_table.inc"
+    {0, 0, 0, 0, 0, 0, 0, 0, {0, -1, 0}}   // terminator
+};
+
+TcTuning tc_tuning(const DcnGeom& g) {
+    TcTuning t{0, -1, 0};
+    for (const TuneEntry* e = kTuneTable; e->Cin; ++e)
+        if (e->Cin == g.Cin && e->Cout == g.Cout && e->H == g.H && e->W == g.W && e->stride == g.sh &&
+            g.sw == g.sh && e->G == g.G && g.KK == 9 && g.N >= e->nmin && g.N <= e->nmax) {
+            t = e->t;
+            break;
+        }
+    if (const char* env = getenv("DEFCON_BLOCK_N")) t.block_n = atoi(env);
+    if (const char* env = getenv("DEFCON_DCN_PAIR")) t.pair = atoi(env) != 0;
+    if (const char* env = getenv("DEFCON_MAX_CTAS")) t.max_ctas = atoi(env);
+    return t;
+}
+
+// BLOCK_N of the bf16 kernel for this shape: the tuned value, else the smallest tile of
+// 64 / 128 / 256 / 512 columns covering Cout.
+int tc_block_n(const DcnGeom& g) {
+    const int bn = tc_tuning(g).block_n;
+    if (bn == 64 || bn == 128 || bn == 256 || bn == 512) return bn;
+    return g.Cout <= 64 ? 64 : g.Cout <= 128 ? 128 : g.Cout <= 256 ? 256 : 512;
+}
+
 template <int BLOCK_N>
 struct Plan {
     int grid;
@@ -1097,13 +1138,13 @@ Plan<BLOCK_N> make_plan(const DcnGeom& g, bool pair = false, int cpi = BK) {
     p.n_tiles = ((g.M + rows - 1) / rows) * p.n_tiles_n;
     p.ipt = (g.Cin / cpi) * g.KK;
     p.total = (long long)p.n_tiles * p.ipt;
-    // At least 4 k-iterations per CTA (pair); DEFCON_MAX_CTAS caps the grid (tests use it to
-    // force long persistent ranges and many whole tiles per CTA).
+    // At least 4 k-iterations per CTA (pair); the tuning's grid cap (DEFCON_MAX_CTAS: tests use
+    // it to force long persistent ranges and many whole tiles per CTA).
     const int per = pair ? 2 : 1;
     const int max_units = pair && g_pair_units > 0 ? g_pair_units : num_sms() / per;
     long long units = std::min<long long>(max_units, (p.total + 3) / 4);
-    if (const char* env = getenv("DEFCON_MAX_CTAS")) {
-        const long long cap = atoll(env);
+    {
+        const long long cap = tc_tuning(g).max_ctas;
         if (cap > 0) units = std::min(units, std::max<long long>(cap / per, 1));
     }
     p.grid = (int)std::max<long long>(units, 1) * per;
@@ -1154,14 +1195,9 @@ __global__ void __launch_bounds__(256) dcn_w_split_kernel(const float* __restric
     }
 }
 
-#ifndef DEFCON_PAIR_DEFAULT
-#define DEFCON_PAIR_DEFAULT 0
-#endif
-// DEFCON_DCN_PAIR=0 / 1 forces the single-CTA / CTA-pair schedule of the N = 256 kernel.
+// CTA pairs (cta_group::2) for the BLOCK_N = 256 kernel when the tuning asks for them.
 bool use_pair(const DcnGeom& g, const TexPlan* tex) {
-    if (tex || g.Cout > 256 || g.Cout <= 128) return false;
-    if (const char* env = getenv("DEFCON_DCN_PAIR")) return atoi(env) != 0;
-    return DEFCON_PAIR_DEFAULT != 0;
+    return !tex && tc_block_n(g) == 256 && tc_tuning(g).pair == 1;
 }
 
 template <int BLOCK_N, int STAGES, bool PAIR = false, bool F32 = false>
@@ -1338,32 +1374,37 @@ bool dcn_tc_bf16_supported(const DcnGeom& g) {
 // no initialisation.
 void dcn_tc_bf16_workspace_counters(const DcnGeom& g, size_t* offset, size_t* bytes) {
     *offset = partials_region();
-    if (g.Cout <= 64) *bytes = make_plan<64>(g).counters_bytes;
-    else if (g.Cout <= 128) *bytes = make_plan<128>(g).counters_bytes;
-    else if (g.Cout <= 256) *bytes = make_plan<256>(g).counters_bytes;
-    else *bytes = make_plan<512>(g).counters_bytes;
+    switch (tc_block_n(g)) {
+        case 64: *bytes = make_plan<64>(g).counters_bytes; break;
+        case 128: *bytes = make_plan<128>(g).counters_bytes; break;
+        case 256: *bytes = make_plan<256>(g).counters_bytes; break;
+        default: *bytes = make_plan<512>(g).counters_bytes; break;
+    }
 }
 
 size_t dcn_tc_bf16_workspace(const DcnGeom& g) {
-    if (g.Cout <= 64) return workspace_impl<64>(g);
-    if (g.Cout <= 128) return workspace_impl<128>(g);
-    if (g.Cout <= 256) return workspace_impl<256>(g);
-    return workspace_impl<512>(g);
+    switch (tc_block_n(g)) {
+        case 64: return workspace_impl<64>(g);
+        case 128: return workspace_impl<128>(g);
+        case 256: return workspace_impl<256>(g);
+        default: return workspace_impl<512>(g);
+    }
 }
 
 cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_bytes,
                                const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
-    if (g.Cout <= 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
-    if (g.Cout <= 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+    const int bn = tc_block_n(g);
+    if (bn == 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+    if (bn == 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 #ifndef DEFCON_STAGES_256
 #define DEFCON_STAGES_256 2
 #endif
 #ifndef DEFCON_STAGES_PAIR
 #define DEFCON_STAGES_PAIR 4
 #endif
-    if (g.Cout <= 256 && use_pair(g, tex))
+    if (bn == 256 && use_pair(g, tex))
         return launch_impl<256, DEFCON_STAGES_PAIR, true>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
-    if (g.Cout <= 256) return launch_impl<256, DEFCON_STAGES_256>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+    if (bn == 256) return launch_impl<256, DEFCON_STAGES_256>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     return launch_impl<512, 2>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 }
 
