@@ -65,6 +65,7 @@ def _load():
         lib.oracle_offset_branch_f64.argtypes = [dp, i, i, i, i, dp, dp, dp, dp, dp,
                                                  i, i, i, i, i, i, dp, dp]
         lib.oracle_bound_offsets_f64.argtypes = [dp, ctypes.c_long, i, i, i, i, i, i, dp]
+        lib.oracle_round_f16_array.argtypes = [dp, ctypes.c_long, dp]
         lib.oracle_bilinear_f64.argtypes = [dp, i, i, ctypes.c_long, ctypes.c_double,
                                             ctypes.c_double]
         lib.oracle_bilinear_f64.restype = ctypes.c_double
@@ -261,4 +262,16 @@ def bound_offsets(offset, P, K=3, dil=1):
     rc = _load().oracle_bound_offsets_f64(_p(off), n_pix, G, Kh, Kw, dh, dw, int(P or 0), _p(out))
     if rc:
         raise ValueError(f"oracle_bound_offsets_f64 rc={rc}")
+    return out
+
+
+def round_f16(a):
+    """tex2D++ (reading R13): offsets / mask as stored in 16 bits (IEEE binary16, round to
+    nearest even), returned as fp64 -- the values a 16-bit-offset DCN computes its coordinates from.
+    None passes through."""
+    if a is None:
+        return None
+    a = _f64(a)
+    out = np.empty_like(a)
+    _load().oracle_round_f16_array(_p(a), int(a.size), _p(out))
     return out

@@ -30,6 +30,7 @@
  *   oracle_dcn_forward_texq_f64 Eq.2 with the texture unit's fixed-point filter
  *                               weights (texture model; NOT from the paper, R14)
  *   oracle_bound_offsets_f64    bounded deformation, P x P window (R12)
+ *   oracle_round_f16_array      16-bit offsets / mask of tex2D++ (R13)
  */
 #include <math.h>
 #include <stddef.h>
@@ -105,14 +106,18 @@ static double quant_frac(double f, int quant_mode) {
     return f;
 }
 
-/* Round to the nearest binary16 value, ties to even (normal and subnormal range; the
- * texels of the half4 texture are binary16, and so is the filter's result, R14). */
+/* Round to the nearest binary16 value, ties to even (normal and subnormal range; beyond the
+ * largest finite value 65504 -- after rounding -- +-infinity, as IEEE binary16 does).  The
+ * texels of the half4 texture are binary16, and so is the filter's result (R14); so are the
+ * 16-bit offsets / mask of tex2D++ (R13). */
 static double round_to_f16(double v) {
     if (v == 0.0 || v != v) return v;
     int e;
     frexp(v, &e);                          /* |v| = m * 2^e, 0.5 <= m < 1 */
     double q = ldexp(1.0, (e - 1 >= -14 ? e - 1 : -14) - 10);   /* 11 significant bits */
-    return rint(v / q) * q;                /* default rounding mode: to nearest, ties to even */
+    double r = rint(v / q) * q;            /* default rounding mode: to nearest, ties to even */
+    if (fabs(r) > 65504.0) r = copysign(INFINITY, v);
+    return r;
 }
 
 /* quant_mode 3 ("hw", the half4-texel filter as measured on B200, R14): both fractions and
@@ -457,5 +462,13 @@ int oracle_bound_offsets_f64(const double *offset, long n_pix, int G, int Kh, in
                     out[e] = dy;
                     out[e + 1] = dx;
                 }
+    return 0;
+}
+
+/* tex2D++ (reading R13): the offsets and mask stored in 16 bits -- IEEE binary16, round to
+ * nearest even (round_to_f16 above) -- before the deformable kernel forms its coordinates.
+ * out may alias in.  Returns 0. */
+int oracle_round_f16_array(const double *in, long n, double *out) {
+    for (long i = 0; i < n; ++i) out[i] = round_to_f16(in[i]);
     return 0;
 }

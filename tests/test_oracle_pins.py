@@ -481,3 +481,28 @@ def test_p15_far_offsets_sample_the_window_corner(oracle_mod, sign):
                 wm = np.einsum("okc,k->oc", w.reshape(w.shape[0], 9, -1), m[n, ho, wo, 0])
                 ref[n, ho, wo] = b + wm @ v
     np.testing.assert_allclose(y, ref, rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- P16: tex2D++ 16-bit offsets
+# tex2D++ "only use[s] 16 bits to compute the offset"; reading R13: IEEE binary16 with
+# round-to-nearest-even storage of offsets and mask.  Pinned to numpy's float16 conversion (a
+# library routine) over normal, subnormal, tie and overflow values.
+def test_p16_round_f16_matches_numpy(oracle_mod):
+    r = np.random.default_rng(16)
+    v = np.concatenate([r.uniform(-8, 8, 4000), r.standard_normal(2000) * 1e-5,       # subnormal range
+                        np.array([1 + 2.0 ** -11, 1 + 3 * 2.0 ** -11, 2049.0, 2051.0,  # ties -> even
+                                  65504.0, 65520.0, -70000.0, 2.0 ** -25, 0.0, -0.0])])
+    got = oracle_mod.round_f16(v)
+    want = v.astype(np.float16).astype(np.float64)
+    assert np.array_equal(got, want)
+
+
+def test_p16_f16_offsets_dcn_is_dcn_of_rounded(oracle_mod):
+    """The 16-bit-offset DCN is the plain DCN on the rounded offsets and mask: equal to the
+    torchvision-pinned DCN at those inputs, and within the rounding's effect of the fp32 one."""
+    x, w, b, off, m, Ho, Wo = rand_layer(seed=16)
+    o16, m16 = oracle_mod.round_f16(off), oracle_mod.round_f16(m)
+    assert np.all(np.abs(o16 - off) <= 2.0 ** -11 * np.abs(off) + 2.0 ** -25)
+    y16 = oracle_mod.dcn_forward(x, o16, w, b, mask=m16)
+    y = oracle_mod.dcn_forward(x, off, w, b, mask=m)
+    assert 0 < np.max(np.abs(y16 - y)) < 1e-2 * np.max(np.abs(y))
