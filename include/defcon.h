@@ -56,7 +56,9 @@ typedef enum {
 
 typedef enum {
     DEFCON_F32 = 0,   /* x, weight, y stored as float32                         */
-    DEFCON_BF16 = 1   /* x, weight, y stored as bfloat16 (fp32 accumulation)    */
+    DEFCON_BF16 = 1,  /* x, weight, y stored as bfloat16 (fp32 accumulation)    */
+    DEFCON_F16 = 2    /* offsets / mask only (defcon_conv_t.offset_dtype): the
+                         16-bit offsets of the paper's tex2D++ (R13)      */
 } defcon_dtype_t;
 
 typedef enum {
@@ -91,6 +93,10 @@ typedef struct {
      * h = (P-1)/2, the offset d is used as clamp(r + d, -h, h) - r (NaN stays NaN).  The paper
      * picks P = 7 (Fig. 5).  0 = unbounded.  Read by the DCN / columns calls only. */
     int bound;
+    /* Storage of the offset / mask tensors: DEFCON_F32 (0) or DEFCON_F16 -- tex2D++, "16 bits
+     * to compute the offset" (reading R13): the branch writes them as binary16 (round
+     * to nearest), the DCN reads them and forms the sampling coordinates in fp32. */
+    int offset_dtype;
 } defcon_conv_t;
 
 /* Opaque texture plan: owns one layered cudaArray + texture object per image. */

@@ -31,6 +31,8 @@ EXPORTED = (
 )
 
 _DTYPES = {torch.float32: DEFCON_F32, torch.bfloat16: DEFCON_BF16}
+DEFCON_F16 = 2
+_OFF_DTYPES = {torch.float32: DEFCON_F32, torch.float16: DEFCON_F16}   # offsets / mask storage
 _SAMPLERS = {"ldg": DEFCON_SAMPLER_LDG, "tex": DEFCON_SAMPLER_TEX, "hybrid": DEFCON_SAMPLER_HYBRID}
 _FP32_MODES = {"3xtf32": DEFCON_FP32_3XTF32, "simt": DEFCON_FP32_SIMT}
 
@@ -46,7 +48,8 @@ class defcon_conv_t(ctypes.Structure):
                 ("pad_h", ctypes.c_int), ("pad_w", ctypes.c_int),
                 ("dil_h", ctypes.c_int), ("dil_w", ctypes.c_int),
                 ("offset_groups", ctypes.c_int),
-                ("bound", ctypes.c_int)]   # bounded deformation P (R12); 0 = unbounded
+                ("bound", ctypes.c_int),   # bounded deformation P (R12); 0 = unbounded
+                ("offset_dtype", ctypes.c_int)]   # DEFCON_F32 / DEFCON_F16 (tex2D++, R13)
 
 
 _lib = None
@@ -101,11 +104,14 @@ def _check(rc: int, where: str):
         raise DefconError(rc, where, load_library().defcon_last_error_detail().decode())
 
 
-def _conv(stride, pad, dil, groups, bound=0) -> defcon_conv_t:
+def _conv(stride, pad, dil, groups, bound=0, offset_dtype=torch.float32) -> defcon_conv_t:
     s = (stride, stride) if isinstance(stride, int) else tuple(stride)
     p = (pad, pad) if isinstance(pad, int) else tuple(pad)
     d = (dil, dil) if isinstance(dil, int) else tuple(dil)
-    return defcon_conv_t(s[0], s[1], p[0], p[1], d[0], d[1], int(groups), int(bound or 0))
+    if offset_dtype not in _OFF_DTYPES:
+        raise ValueError("offsets / mask must be float32 or float16")
+    return defcon_conv_t(s[0], s[1], p[0], p[1], d[0], d[1], int(groups), int(bound or 0),
+                         _OFF_DTYPES[offset_dtype])
 
 
 def _out(n, k, s, p, d):
@@ -164,14 +170,15 @@ def defcon_offset_workspace_size(N, H, W, C, K=3, stride=1, pad=1, dil=1, offset
 
 def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, stride=1, pad=1,
                           dil=1, offset_groups=1, with_mask=True, offset=None, mask=None,
-                          workspace=None, stream=None):
-    """Step 1: lightweight offset branch.  Returns (offset, mask|None)."""
+                          workspace=None, stream=None, offset_dtype=torch.float32):
+    """Step 1: lightweight offset branch.  Returns (offset, mask|None), stored as
+    offset_dtype (torch.float16: the 16-bit offsets of tex2D++, R13)."""
     lib = load_library()
     _dev_tensor(x, "x")
     if x.dtype not in _DTYPES:
         raise ValueError("x must be float32 or bfloat16")
     N, H, W, C = x.shape
-    cv = _conv(stride, pad, dil, offset_groups)
+    cv = _conv(stride, pad, dil, offset_groups, 0, offset_dtype)
     Ho, Wo = _out(H, 3, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, 3, cv.stride_w, cv.pad_w, cv.dil_w)
     G, KK = int(offset_groups), K * K
     OC = G * KK * (3 if with_mask else 2)
@@ -182,16 +189,16 @@ def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, str
     _dev_tensor(pw_b, "pw_b", torch.float32, (OC,), allow_none=True)
     with _on(stream):
         if offset is None:
-            offset = torch.empty((N, Ho, Wo, G, KK, 2), device=x.device, dtype=torch.float32)
+            offset = torch.empty((N, Ho, Wo, G, KK, 2), device=x.device, dtype=offset_dtype)
         if with_mask and mask is None:
-            mask = torch.empty((N, Ho, Wo, G, KK), device=x.device, dtype=torch.float32)
+            mask = torch.empty((N, Ho, Wo, G, KK), device=x.device, dtype=offset_dtype)
         if workspace is None:
             workspace = torch.empty(defcon_offset_workspace_size(N, H, W, C, K, stride, pad, dil,
                                                                  offset_groups),
                                     dtype=torch.uint8, device=x.device)
-    _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, KK, 2))
+    _dev_tensor(offset, "offset", offset_dtype, (N, Ho, Wo, G, KK, 2))
     if with_mask:
-        _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, KK))
+        _dev_tensor(mask, "mask", offset_dtype, (N, Ho, Wo, G, KK))
     else:
         mask = None
     rc = lib.defcon_offset_dw_conv(_ptr(x), N, H, W, C, _DTYPES[x.dtype], _ptr(dw_w), _ptr(dw_scale),
@@ -228,11 +235,12 @@ def defcon_dcn_forward(x, offset, mask, weight, bias=None, stride=1, pad=1, dil=
     Cout, Kh, Kw, Cw = weight.shape
     if Cw != Cin:
         raise ValueError("weight Cin mismatch")
-    cv = _conv(stride, pad, dil, offset_groups, bound)
+    odt = offset.dtype if offset is not None else torch.float32   # float16: tex2D++ offsets (R13)
+    cv = _conv(stride, pad, dil, offset_groups, bound, odt)
     Ho, Wo = _out(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w)
     G = int(offset_groups)
-    _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
-    _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
+    _dev_tensor(offset, "offset", odt, (N, Ho, Wo, G, Kh * Kw, 2))
+    _dev_tensor(mask, "mask", odt, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
     _dev_tensor(bias, "bias", torch.float32, (Cout,), allow_none=True)
     with _on(stream):
         if y is None:
@@ -263,11 +271,12 @@ def defcon_deform_columns(x, offset, mask, K=3, stride=1, pad=1, dil=1, offset_g
         raise ValueError("x must be float32 or bfloat16")
     N, H, W, Cin = x.shape
     Kh, Kw = (K, K) if isinstance(K, int) else K
-    cv = _conv(stride, pad, dil, offset_groups, bound)
+    odt = offset.dtype if offset is not None else torch.float32
+    cv = _conv(stride, pad, dil, offset_groups, bound, odt)
     Ho, Wo = _out(H, Kh, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, Kw, cv.stride_w, cv.pad_w, cv.dil_w)
     G = int(offset_groups)
-    _dev_tensor(offset, "offset", torch.float32, (N, Ho, Wo, G, Kh * Kw, 2))
-    _dev_tensor(mask, "mask", torch.float32, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
+    _dev_tensor(offset, "offset", odt, (N, Ho, Wo, G, Kh * Kw, 2))
+    _dev_tensor(mask, "mask", odt, (N, Ho, Wo, G, Kh * Kw), allow_none=True)
     if columns is None:
         with _on(stream):
             columns = torch.empty((N * Ho * Wo, Kh * Kw * Cin), device=x.device, dtype=x.dtype)
@@ -280,11 +289,12 @@ def defcon_deform_columns(x, offset, mask, K=3, stride=1, pad=1, dil=1, offset_g
 
 def defcon_layer_workspace_size(N, H, W, Cin, Cout, K=3, stride=1, pad=1, dil=1, offset_groups=1,
                                 dtype=torch.bfloat16, modulated=True, sampler="ldg",
-                                fp32_mode="simt") -> int:
+                                fp32_mode="simt", bound=0, offset_dtype=torch.float32) -> int:
     lib = load_library()
     out = ctypes.c_size_t(0)
     rc = lib.defcon_layer_workspace_size(N, H, W, Cin, _DTYPES[dtype], Cout, K,
-                                         _conv(stride, pad, dil, offset_groups), int(modulated),
+                                         _conv(stride, pad, dil, offset_groups, bound, offset_dtype),
+                                         int(modulated),
                                          _SAMPLERS[sampler], _FP32_MODES[fp32_mode],
                                          ctypes.byref(out))
     _check(rc, "defcon_layer_workspace_size")
@@ -293,7 +303,7 @@ def defcon_layer_workspace_size(N, H, W, Cin, Cout, K=3, stride=1, pad=1, dil=1,
 
 def defcon_layer_forward_host(x_host, branch, weight, bias, y_host, dev_workspace, K=3, stride=1,
                               pad=1, dil=1, offset_groups=1, modulated=True, sampler="ldg",
-                              fp32_mode="simt", stream=None, bound=0):
+                              fp32_mode="simt", stream=None, bound=0, offset_dtype=torch.float32):
     """Whole layer from pinned host x to pinned host y (H2D, step 1, step 2, D2H, sync).
 
     branch: dict of device tensors dw_w, dw_scale, dw_shift, pw_w, pw_b (resident weights).
@@ -307,7 +317,7 @@ def defcon_layer_forward_host(x_host, branch, weight, bias, y_host, dev_workspac
         _ptr(x_host), N, H, W, Cin, _DTYPES[x_host.dtype], _ptr(branch["dw_w"]),
         _ptr(branch["dw_scale"]), _ptr(branch["dw_shift"]), _ptr(branch["pw_w"]),
         _ptr(branch.get("pw_b")), _ptr(weight), _ptr(bias), Cout, K,
-        _conv(stride, pad, dil, offset_groups, bound), int(modulated), _SAMPLERS[sampler],
+        _conv(stride, pad, dil, offset_groups, bound, offset_dtype), int(modulated), _SAMPLERS[sampler],
         _FP32_MODES[fp32_mode], _ptr(y_host), _ptr(dev_workspace),
         dev_workspace.numel() * dev_workspace.element_size(), _stream_handle(stream))
     _check(rc, "defcon_layer_forward_host")

@@ -60,6 +60,8 @@ static int check_conv(const defcon_conv_t& cv) {
     if (cv.pad_h < 0 || cv.pad_w < 0) return fail(DEFCON_ERR_INVALID_ARG, "padding must be >= 0");
     if (cv.offset_groups <= 0) return fail(DEFCON_ERR_INVALID_ARG, "offset_groups must be > 0");
     if (cv.bound < 0) return fail(DEFCON_ERR_INVALID_ARG, "bound must be >= 0 (0 = unbounded)");
+    if (cv.offset_dtype != DEFCON_F32 && cv.offset_dtype != DEFCON_F16)
+        return fail(DEFCON_ERR_INVALID_ARG, "offset_dtype must be DEFCON_F32 or DEFCON_F16");
     return DEFCON_OK;
 }
 
@@ -81,6 +83,7 @@ static int make_geom(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
     g->G = cv.offset_groups;
     g->Cg = Cin / cv.offset_groups;
     g->bound_h = cv.bound > 0 ? 0.5f * (float)(cv.bound - 1) : -1.f;
+    g->off_f16 = cv.offset_dtype == DEFCON_F16 ? 1 : 0;
     g->KK = Kh * Kw;
     const long M = (long)N * g->Ho * g->Wo;
     if ((long)N * H * W * Cin >= (1L << 31) || M * Cout >= (1L << 31) ||
@@ -212,7 +215,7 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
                                          dw_shift, pw_w, pw_b, K, G, mask != nullptr, cv.stride_h,
                                          cv.stride_w, cv.pad_h, cv.pad_w, cv.dil_h, cv.dil_w, Ho, Wo,
                                          offset, mask, static_cast<float*>(workspace),
-                                         static_cast<cudaStream_t>(stream));
+                                         static_cast<cudaStream_t>(stream), cv.offset_dtype == DEFCON_F16);
     if (e == cudaErrorInvalidValue) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d unsupported", OC);
     if (e != cudaSuccess) return cuda_fail(e, "offset_branch launch");
     return DEFCON_OK;
@@ -343,8 +346,9 @@ static ChunkCarve chunk_carve(const DcnGeom& g, int dtype, int Cout, int modulat
     ChunkCarve c;
     c.x = align_up((size_t)nc * g.H * g.W * g.Cin * es);
     c.y = align_up((size_t)nc * hw * Cout * es);
-    c.off = align_up((size_t)nc * hw * g.G * g.KK * 2 * sizeof(float));
-    c.msk = modulated ? align_up((size_t)nc * hw * g.G * g.KK * sizeof(float)) : 0;
+    const size_t oes = g.off_f16 ? 2 : 4;   // offsets / mask element bytes
+    c.off = align_up((size_t)nc * hw * g.G * g.KK * 2 * oes);
+    c.msk = modulated ? align_up((size_t)nc * hw * g.G * g.KK * oes) : 0;
     return c;
 }
 

@@ -86,6 +86,19 @@ DEFCON_DEVICE float bound_offset(float d, float r, float h) {
     return fminf(fmaxf(r + d, -h), h) - r;
 }
 
+// Offsets / mask in fp32 or binary16 (tex2D++, R13): element pair `i2` (dy, dx), mask `i`.
+DEFCON_DEVICE float2 ld_offset2(const float* base, long i2, bool f16) {
+    if (f16) return __half22float2(__ldg(reinterpret_cast<const __half2*>(base) + (i2 >> 1)));
+    return __ldg(reinterpret_cast<const float2*>(base + i2));
+}
+DEFCON_DEVICE float ld_mask1(const float* base, long i, bool f16) {
+    return f16 ? __half2float(__ldg(reinterpret_cast<const __half*>(base) + i)) : __ldg(base + i);
+}
+DEFCON_DEVICE void st_offset1(float* base, long i, float v, bool f16) {
+    if (f16) reinterpret_cast<__half*>(base)[i] = __float2half_rn(v);
+    else base[i] = v;
+}
+
 // ------------------------------------------------------------------ fences
 // Make this thread's generic-proxy smem writes visible to the async proxy
 // (tcgen05.mma operand reads, TMA).

@@ -80,11 +80,11 @@ __global__ void __launch_bounds__(THREADS) dcn_fwd_simt_kernel(const SimtArgs a)
                 const int ho = rem / g.Wo, wo = rem - (rem / g.Wo) * g.Wo;
                 const int i = tap / g.Kw, j = tap - (tap / g.Kw) * g.Kw;
                 const long pix = (long)m * g.G + grp;
-                const float dy = bound_offset(a.offset[(pix * g.KK + tap) * 2], (i - 0.5f * (g.Kh - 1)) * g.dh,
+                const float2 d = ld_offset2(a.offset, (pix * g.KK + tap) * 2, g.off_f16);
+                const float dy = bound_offset(d.x, (i - 0.5f * (g.Kh - 1)) * g.dh,
                                               g.bound_h);   // bounded deformation (R12)
-                const float dx = bound_offset(a.offset[(pix * g.KK + tap) * 2 + 1], (j - 0.5f * (g.Kw - 1)) * g.dw,
-                                              g.bound_h);
-                const float mk = a.mask ? a.mask[pix * g.KK + tap] : 1.f;
+                const float dx = bound_offset(d.y, (j - 0.5f * (g.Kw - 1)) * g.dw, g.bound_h);
+                const float mk = a.mask ? ld_mask1(a.mask, pix * g.KK + tap, g.off_f16) : 1.f;
                 float py = (float)(ho * g.sh - g.ph + i * g.dh) + dy;
                 float px = (float)(wo * g.sw - g.pw + j * g.dw) + dx;
                 py = fminf(fmaxf(py, -2.f), (float)g.H + 1.f);
@@ -222,11 +222,10 @@ __global__ void __launch_bounds__(THREADS, 2) dcn_fwd_f32_tiled_kernel(const Sim
                 if (gok) {
                     const long pix = (long)gm * g.G + grp;
                     const int i = tap / g.Kw, j = tap - (tap / g.Kw) * g.Kw;
-                    const float dy = bound_offset(__ldg(a.offset + (pix * g.KK + tap) * 2),
-                                                  (i - 0.5f * (g.Kh - 1)) * g.dh, g.bound_h);   // P:182, R12
-                    const float dx = bound_offset(__ldg(a.offset + (pix * g.KK + tap) * 2 + 1),
-                                                  (j - 0.5f * (g.Kw - 1)) * g.dw, g.bound_h);
-                    const float mk = a.mask ? __ldg(a.mask + pix * g.KK + tap) : 1.f;
+                    const float2 d = ld_offset2(a.offset, (pix * g.KK + tap) * 2, g.off_f16);
+                    const float dy = bound_offset(d.x, (i - 0.5f * (g.Kh - 1)) * g.dh, g.bound_h);   // P:182, R12
+                    const float dx = bound_offset(d.y, (j - 0.5f * (g.Kw - 1)) * g.dw, g.bound_h);
+                    const float mk = a.mask ? ld_mask1(a.mask, pix * g.KK + tap, g.off_f16) : 1.f;
                     float py = (float)(gyb + i * g.dh) + dy;
                     float px = (float)(gxb + j * g.dw) + dx;
                     py = fminf(fmaxf(py, -2.f), (float)g.H + 1.f);

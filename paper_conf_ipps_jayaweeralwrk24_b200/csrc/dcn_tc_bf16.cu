@@ -95,6 +95,7 @@ struct TcArgs {
     int sh, sw, ph, pw, dh, dw;
     int G, Cg, M, KK;
     float bound_h;         // bounded deformation half-window (R12); < 0: unbounded
+    int off_f16;           // offsets / mask in binary16 (tex2D++, R13)
     int ipt;               // k-iterations per tile = (Cin / CPI) * KK
     int es, cpi;           // element bytes, channels per k-iteration
     int n_tiles_n;         // tiles along Cout
@@ -265,8 +266,8 @@ __device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g,
             in[k].d = make_float2(0.f, 0.f);
             in[k].mk = 0.f;
             if (rp.ok && tk < a.KK) {
-                in[k].d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + tk) * 2));
-                in[k].mk = a.mask ? __ldg(a.mask + pix * a.KK + tk) : 1.0f;
+                in[k].d = ld_offset2(a.offset, (pix * a.KK + tk) * 2, a.off_f16);
+                in[k].mk = a.mask ? ld_mask1(a.mask, pix * a.KK + tk, a.off_f16) : 1.0f;
             }
         }
 #ifdef DEFCON_PROBE_TL_META
@@ -287,10 +288,11 @@ __device__ __forceinline__ void prefetch_meta_l2(const TcArgs& a, int m0, int t)
     if (m0 < 0) return;
     const int rows = min(BM, a.M - m0);
     const size_t per_pix = (size_t)a.G * a.KK;
-    const char* o0 = reinterpret_cast<const char*>(a.offset + (size_t)m0 * per_pix * 2);
-    const int o_lines = (int)((rows * per_pix * 8 + 127) / 128);
-    const char* k0 = a.mask ? reinterpret_cast<const char*>(a.mask + (size_t)m0 * per_pix) : nullptr;
-    const int k_lines = a.mask ? (int)((rows * per_pix * 4 + 127) / 128) : 0;
+    const size_t es = a.off_f16 ? 2 : 4;
+    const char* o0 = reinterpret_cast<const char*>(a.offset) + (size_t)m0 * per_pix * 2 * es;
+    const int o_lines = (int)((rows * per_pix * 2 * es + 127) / 128);
+    const char* k0 = a.mask ? reinterpret_cast<const char*>(a.mask) + (size_t)m0 * per_pix * es : nullptr;
+    const int k_lines = a.mask ? (int)((rows * per_pix * es + 127) / 128) : 0;
     for (int l = t; l < o_lines + k_lines; l += NPT) {
         const char* p = l < o_lines ? o0 + (size_t)l * 128 : k0 + (size_t)(l - o_lines) * 128;
         asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
@@ -1302,6 +1304,7 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     a.sh = g.sh; a.sw = g.sw; a.ph = g.ph; a.pw = g.pw; a.dh = g.dh; a.dw = g.dw;
     a.G = g.G; a.Cg = g.Cg; a.M = g.M; a.KK = g.KK;
     a.bound_h = g.bound_h;
+    a.off_f16 = g.off_f16;
     a.ipt = plan.ipt;
     a.n_tiles_n = plan.n_tiles_n;
     a.total_iters = plan.total;

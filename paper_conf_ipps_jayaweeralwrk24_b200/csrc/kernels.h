@@ -17,6 +17,7 @@ struct DcnGeom {
     int M;       // N * Ho * Wo output pixels
     int KK;      // Kh * Kw taps
     float bound_h;   // bounded deformation half-window (P-1)/2 (R12); < 0: unbounded
+    int off_f16;     // offsets / mask stored as binary16 (tex2D++, R13)
 };
 
 struct DcnPtrs {
@@ -33,7 +34,8 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                 float* offset, float* mask, float* t_ws, cudaStream_t stream);
+                                 float* offset, float* mask, float* t_ws, cudaStream_t stream,
+                                 bool out_f16 = false);
 // workspace of defcon_offset_dw_conv: the one-pass kernel's packed parameters when it can run
 // this shape (decided for the widest branch, OC = 3*G*K*K), else the two-pass t buffers
 size_t offset_branch_workspace(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph,
@@ -47,7 +49,8 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
                                          const float* dw_w, const float* dw_scale, const float* dw_shift,
                                          const float* pw_w, const float* pw_b, int n_off, int n_msk,
                                          int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                         float* offset, float* mask, void* ws, cudaStream_t stream);
+                                         float* offset, float* mask, void* ws, cudaStream_t stream,
+                                         bool out_f16);
 // ---- sampling step alone: deformable columns [M][KK*Cin] (sampler.cu)
 cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* offset, const float* mask,
                                   bool bf16, void* cols, cudaStream_t stream);

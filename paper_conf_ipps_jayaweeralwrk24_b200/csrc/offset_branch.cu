@@ -43,6 +43,7 @@ struct BranchArgs {
     int N, H, W, C, Ho, Wo, M;
     int sh, sw, ph, pw, dh, dw;
     int n_off, n_msk, OC;
+    int out_f16;       // offsets / mask written as binary16 (tex2D++, R13)
 };
 
 // ------------------------------------------------------------------ depthwise 3x3
@@ -331,9 +332,9 @@ __global__ void __launch_bounds__(PW_WARPS * 32) pw_sigmoid_kernel(const BranchA
                 if (o >= a.OC) continue;
                 const float val = acc[nt][h * 2 + u] + (a.pw_b ? __ldg(a.pw_b + o) : 0.f);
                 if (o < a.n_off)
-                    a.offset[(long)m * a.n_off + o] = val;
+                    st_offset1(a.offset, (long)m * a.n_off + o, val, a.out_f16);
                 else
-                    a.mask[(long)m * a.n_msk + (o - a.n_off)] = 1.f / (1.f + __expf(-val));
+                    st_offset1(a.mask, (long)m * a.n_msk + (o - a.n_off), 1.f / (1.f + __expf(-val)), a.out_f16);
             }
     }
 }
@@ -417,9 +418,9 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
                     if (o >= a.OC) break;
                     const float val = __uint_as_float(vv[u]) + (a.pw_b ? __ldg(a.pw_b + o) : 0.f);
                     if (o < a.n_off)
-                        a.offset[(long)m * a.n_off + o] = val;
+                        st_offset1(a.offset, (long)m * a.n_off + o, val, a.out_f16);
                     else
-                        a.mask[(long)m * a.n_msk + (o - a.n_off)] = 1.f / (1.f + __expf(-val));
+                        st_offset1(a.mask, (long)m * a.n_msk + (o - a.n_off), 1.f / (1.f + __expf(-val)), a.out_f16);
                 }
             }
         }
@@ -524,8 +525,10 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                 float* offset, float* mask, float* t_ws, cudaStream_t stream) {
+                                 float* offset, float* mask, float* t_ws, cudaStream_t stream,
+                                 bool out_f16) {
     BranchArgs a;
+    a.out_f16 = out_f16 ? 1 : 0;
     a.x = x; a.dw_w = dw_w; a.dw_scale = dw_scale; a.dw_shift = dw_shift;
     a.pw_w = pw_w; a.pw_b = pw_b; a.t = t_ws; a.t_lo = nullptr; a.w_hi = nullptr; a.w_lo = nullptr;
     a.offset = offset; a.mask = mask;
@@ -540,7 +543,7 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     if (use_onepass(N, H, W, C, Ho, Wo, K, G, s_h, s_w, p_h, p_w, d_h, d_w, x_bf16))
         return launch_offset_branch_onepass(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
                                             a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
-                                            mask, t_ws, stream);
+                                            mask, t_ws, stream, out_f16);
     // 1x1 on tcgen05 from TMA-loaded hi / lo planes, or the mma.sync 3xTF32 kernel (t in one
     // plane)
     // The tcgen05 kernel runs one 128-pixel tile per CTA, two CTAs per SM, each CTA a latency

@@ -73,6 +73,7 @@ struct OpArgs {
     const uint8_t* packed;  // per-chunk parameter blocks (op_pack_kernel)
     float* offset;          // [M][n_off]
     float* mask;            // [M][n_msk] or null
+    int out_f16;            // offsets / mask written as binary16 (tex2D++, R13)
     int H, W, C, Ho, Wo, Wv;   // Wv = Wo rounded up to even: virtual row length of the tiling
     int MV;                 // N * Ho * Wv virtual pixels
     int sh, sw, ph, pw, dh, dw;
@@ -462,11 +463,11 @@ __global__ void __maxnreg__(OP_REGS)
     }
     OPTL(31);
     {
-        float* go = a.offset + (long)mf * a.n_off;
-        for (int e = ctid; e < nreal * a.n_off; e += NC) go[e] = off_s[e];
+        const long go = (long)mf * a.n_off;
+        for (int e = ctid; e < nreal * a.n_off; e += NC) st_offset1(a.offset, go + e, off_s[e], a.out_f16);
         if (a.n_msk) {
-            float* gm = a.mask + (long)mf * a.n_msk;
-            for (int e = ctid; e < nreal * a.n_msk; e += NC) gm[e] = msk_s[e];
+            const long gm = (long)mf * a.n_msk;
+            for (int e = ctid; e < nreal * a.n_msk; e += NC) st_offset1(a.mask, gm + e, msk_s[e], a.out_f16);
         }
     }
     OPTL(22);
@@ -595,7 +596,8 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
                                          const float* dw_w, const float* dw_scale, const float* dw_shift,
                                          const float* pw_w, const float* pw_b, int n_off, int n_msk,
                                          int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
-                                         float* offset, float* mask, void* ws, cudaStream_t stream) {
+                                         float* offset, float* mask, void* ws, cudaStream_t stream,
+                                         bool out_f16) {
     const int es = x_bf16 ? 2 : 4;
     OpPlan p;
     if (!make_op_plan(N, H, W, C, Ho, Wo, s_h, s_w, p_h, p_w, d_h, d_w, n_off + n_msk, es, &p))
@@ -604,6 +606,7 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
     a.dw_w = dw_w; a.dw_scale = dw_scale; a.dw_shift = dw_shift;
     a.pw_w = pw_w; a.pw_b = pw_b; a.offset = offset; a.mask = mask;
     a.n_off = n_off; a.n_msk = n_msk;
+    a.out_f16 = out_f16 ? 1 : 0;
     a.packed = static_cast<const uint8_t*>(ws);
     // plain stream order (not PDL): measured faster behind a host-to-device copy in the host entry
     op_pack_kernel<<<dim3(a.nch, (a.OCN * OP_KC + 255) / 256), 256, 0, stream>>>(dw_w, dw_scale, dw_shift, pw_w, C,

@@ -28,6 +28,7 @@ struct ColArgs {
     int sh, sw, ph, pw, dh, dw;
     int G, Cg, M, KK;
     float bound_h;       // bounded deformation half-window (R12); < 0: unbounded
+    int off_f16;         // offsets / mask in binary16 (tex2D++, R13)
     int pieces;          // 32-byte pieces per (pixel, tap) row = Cin * ES / 32
     long long total;     // M * KK * pieces
 };
@@ -57,10 +58,10 @@ __device__ __forceinline__ void piece_issue(const ColArgs& a, long long u, Piece
     const int wo = rem - ho * a.Wo;
     const int i = k / a.Kw, j = k - (k / a.Kw) * a.Kw;
     const long pix = (long)m * a.G + g;
-    float2 d = __ldg(reinterpret_cast<const float2*>(a.offset + (pix * a.KK + k) * 2));
+    float2 d = ld_offset2(a.offset, (pix * a.KK + k) * 2, a.off_f16);
     d.x = bound_offset(d.x, (i - 0.5f * (a.KK / a.Kw - 1)) * a.dh, a.bound_h);   // P:182, R12
     d.y = bound_offset(d.y, (j - 0.5f * (a.Kw - 1)) * a.dw, a.bound_h);
-    const float mv = a.mask ? __ldg(a.mask + pix * a.KK + k) : 1.f;
+    const float mv = a.mask ? ld_mask1(a.mask, pix * a.KK + k, a.off_f16) : 1.f;
     float py = (float)(ho * a.sh - a.ph + i * a.dh) + d.x;
     float px = (float)(wo * a.sw - a.pw + j * a.dw) + d.y;
     py = fminf(fmaxf(py, -2.f), (float)a.H + 1.f);     // beyond one pixel out: zeros only
@@ -164,8 +165,8 @@ __device__ __forceinline__ RowMeta row_meta(const ColArgs& a, int r, int piece) 
     const int m = r / a.KK, k = r - (r / a.KK) * a.KK;
     const int g = piece * Piece<BF16>::CPP / a.Cg;
     const int pix = m * a.G + g;
-    q.d = __ldg(reinterpret_cast<const float2*>(a.offset) + pix * a.KK + k);
-    q.mv = a.mask ? __ldg(a.mask + pix * a.KK + k) : 1.f;
+    q.d = ld_offset2(a.offset, ((long)pix * a.KK + k) * 2, a.off_f16);
+    q.mv = a.mask ? ld_mask1(a.mask, (long)pix * a.KK + k, a.off_f16) : 1.f;
     return q;
 }
 
@@ -248,6 +249,7 @@ cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* 
     a.sh = g.sh; a.sw = g.sw; a.ph = g.ph; a.pw = g.pw; a.dh = g.dh; a.dw = g.dw;
     a.G = g.G; a.Cg = g.Cg; a.M = g.M; a.KK = g.KK;
     a.bound_h = g.bound_h;
+    a.off_f16 = g.off_f16;
     a.pieces = g.Cin * (bf16 ? 2 : 4) / 32;
     a.total = (long long)g.M * g.KK * a.pieces;
     int dev = 0, nsm = 148;

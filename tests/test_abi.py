@@ -43,7 +43,8 @@ def test_status_strings(lib):
 
 def _conv(**kw):
     from paper_conf_ipps_jayaweeralwrk24_b200._binding import defcon_conv_t
-    d = dict(stride_h=1, stride_w=1, pad_h=1, pad_w=1, dil_h=1, dil_w=1, offset_groups=1, bound=0)
+    d = dict(stride_h=1, stride_w=1, pad_h=1, pad_w=1, dil_h=1, dil_w=1, offset_groups=1, bound=0,
+             offset_dtype=0)
     d.update(kw)
     return defcon_conv_t(**d)
 
@@ -70,9 +71,10 @@ def _fwd(lib, x=FAKE, N=2, H=8, W=8, Cin=64, off=FAKE, mask=FAKE, w=FAKE, b=FAKE
     (dict(x=FAKE + 16), 3),               # tensor-core path: x is gathered in 32-byte vectors
     (dict(cv="g16_bf16"), 2),             # Cin/G = 4, not a multiple of 8 for bf16
     (dict(cv="neg_bound"), 1),            # bounded deformation P must be >= 0
+    (dict(cv="bf16_offsets"), 1),         # offsets / mask: DEFCON_F32 or DEFCON_F16 only
 ])
 def test_dcn_forward_validation(lib, kw, status):
-    cvs = {"g3": _conv(offset_groups=3), "s0": _conv(stride_h=0), "neg_bound": _conv(bound=-1),
+    cvs = {"g3": _conv(offset_groups=3), "s0": _conv(stride_h=0), "neg_bound": _conv(bound=-1), "bf16_offsets": _conv(offset_dtype=1),
            "tiny": _conv(pad_h=0, pad_w=0), "g16_bf16": _conv(offset_groups=16)}
     if kw.get("cv") in cvs:
         name = kw.pop("cv")

@@ -16,6 +16,7 @@ import paper_conf_ipps_jayaweeralwrk24_b200 as d  # noqa: E402
 
 
 BOUND = int(os.environ.get("PROBE_BOUND", "0"))   # bounded deformation P (0 = unbounded)
+OFF16 = os.environ.get("PROBE_OFF16", "0") == "1"  # tex2D++: binary16 offsets / mask
 
 
 def time_cfg(c, sampler, reps=200):
@@ -26,8 +27,9 @@ def time_cfg(c, sampler, reps=200):
     L = inputs.gen_layer(c)
     dt = torch.bfloat16 if c.dtype == "bf16" else torch.float32
     x = torch.from_numpy(L["x"]).to(dev, dt)
-    off = torch.from_numpy(L["offset"]).to(dev)
-    msk = torch.from_numpy(L["mask"]).to(dev) if L["mask"] is not None else None
+    odt = torch.float16 if OFF16 else torch.float32
+    off = torch.from_numpy(L["offset"]).to(dev, odt)
+    msk = torch.from_numpy(L["mask"]).to(dev, odt) if L["mask"] is not None else None
     w = torch.from_numpy(L["weight"]).to(dev, dt)
     b = torch.from_numpy(L["bias"]).to(dev)
     y = torch.empty((c.N, c.Ho, c.Wo, c.Cout), device=dev, dtype=dt)
