@@ -11,8 +11,16 @@ python bench.py > gpurun_out/${R}_bench.json 2> gpurun_out/${R}_bench.err
 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv \
     --log-file gpurun_out/${R}_launches.csv python bench.py --steps 4 --warmup 3 --no-cpu-baseline > /dev/null 2>&1
 # one full capture per hot-path kernel, same command
-ncu --set full --clock-control none --import-source on -k regex:"dcn_fwd|dw_bn|pw_" -s 3 -c 3 \
+ncu --set full --clock-control none --import-source on -k regex:"dcn_fwd|offset_branch_onepass|op_pack" -s 3 -c 3 \
     -o gpurun_out/${R}_full python bench.py --steps 4 --warmup 3 --no-cpu-baseline > /dev/null 2>&1
 ncu -i gpurun_out/${R}_full.ncu-rep --page details --csv > gpurun_out/${R}_full_details.csv 2>/dev/null
 ncu -i gpurun_out/${R}_full.ncu-rep --page raw --csv > gpurun_out/${R}_full_raw.csv 2>/dev/null
+# the sampling stage alone (defcon_deform_columns): dram bytes of the columns kernel
+ncu --set full --clock-control none -k regex:"deform_columns" -c 1 -o gpurun_out/${R}_columns \
+    python tools/probe_sampler.py yolact_r101_c5_v2 > /dev/null 2>&1
+ncu -i gpurun_out/${R}_columns.ncu-rep --page raw --csv > gpurun_out/${R}_columns_raw.csv 2>/dev/null
+# fp32 3xTF32 DCN (C4 fp32)
+ncu --set full --clock-control none -k regex:"dcn_fwd" -c 1 -o gpurun_out/${R}_f32 \
+    python tools/probe_dcn.py yolact_r101_c4_v2_f32 3xtf32 > /dev/null 2>&1
+ncu -i gpurun_out/${R}_f32.ncu-rep --page raw --csv > gpurun_out/${R}_f32_raw.csv 2>/dev/null
 echo done

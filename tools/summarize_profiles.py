@@ -19,7 +19,8 @@ for r in rows:
     if hdr and len(r) == len(hdr):
         d = dict(zip(hdr, r))
         launch.append((d["Kernel Name"].split("(")[0].replace("void ", ""), float(d["Metric Value"])))
-ours = [(k, v) for k, v in launch if any(s in k for s in ("dcn_fwd", "dw_bn", "pw_", "tex_stage"))]
+ours = [(k, v) for k, v in launch if any(s in k for s in ("dcn_fwd", "dw_bn", "pw_", "tex_stage", "offset_branch",
+                                                          "op_pack"))]
 tot = {}
 for k, v in ours:
     tot.setdefault(k, []).append(v)
@@ -64,5 +65,32 @@ summary = {"round": R, "launch_list_us": {k: [round(x / 1000, 2) for x in v] for
 dcn = [c for c in caps if "dcn_fwd" in c["kernel"]]
 if dcn:
     summary["dcn_dram_bytes_per_launch"] = dcn[0]["dram__bytes_read"] + dcn[0]["dram__bytes_write"]
+    summary["dcn_dram_bytes_note"] = (
+        "cold: ncu --cache-control all flushes L2 before the replay; y (M x Cout bf16) stays dirty "
+        "in the write-back L2 at kernel end, so dram__bytes_write under-counts it")
+
+
+def extra(name):   # the other captures of the round (columns kernel, fp32 DCN)
+    try:
+        rr = list(csv.reader(open(f"{G}/{R}_{name}_raw.csv")))
+    except OSError:
+        return []
+    hh, uu = rr[0], dict(zip(rr[0], rr[1]))
+    out = []
+    for r in rr[2:]:
+        d = dict(zip(hh, r))
+        rec = {"kernel": d.get("Kernel Name", "").split("(")[0].replace("void ", "")}
+        for k in want:
+            try:
+                v = float(str(d.get(k)).replace(",", "")) * SCALE.get(uu.get(k, ""), 1)
+            except (TypeError, ValueError):
+                v = d.get(k)
+            rec[k.replace(".sum", "").replace("gpu__time_duration", "duration_us")] = v
+        out.append(rec)
+    return out
+
+
+summary["columns_capture"] = extra("columns")
+summary["f32_3xtf32_capture"] = extra("f32")
 json.dump(summary, open(f"{P}/{R}_ncu_summary.json", "w"), indent=1)
 print(json.dumps(summary, indent=1)[:3000])
