@@ -398,6 +398,26 @@ DEFCON_DEVICE void mbar_arrive_cluster(uint64_t* bar, uint32_t cta) {
         "r"(cta)
         : "memory");
 }
+// Release-arrive (cluster scope) on the barrier at the same offset in CTA `cta`: orders this
+// thread's earlier distributed-shared-memory stores before the arrival.
+DEFCON_DEVICE void mbar_arrive_release_cluster(uint64_t* bar, uint32_t cta) {
+    asm volatile(
+        "{\n\t.reg .b32 ra;\n\t"
+        "mapa.shared::cluster.u32 ra, %0, %1;\n\t"
+        "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n\t}" ::"r"(smem_u32(bar)),
+        "r"(cta)
+        : "memory");
+}
+// 16-byte store into CTA `cta`'s shared memory at the offset of local address `laddr`.
+DEFCON_DEVICE void st_cluster_v4(uint32_t laddr, uint32_t cta, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+    asm volatile(
+        "{\n\t.reg .b32 ra;\n\t"
+        "mapa.shared::cluster.u32 ra, %0, %1;\n\t"
+        "st.shared::cluster.v4.b32 [ra], {%2, %3, %4, %5};\n\t}" ::"r"(laddr),
+        "r"(cta), "r"(a), "r"(b), "r"(c), "r"(d)
+        : "memory");
+}
+
 // Wait for a phase whose arrivals may come from the peer CTA (cluster-scope acquire).
 DEFCON_DEVICE void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
     uint32_t ok = 0;

@@ -84,6 +84,9 @@ struct OpArgs {
     int XS;                 // x stages in flight
     int x_stage;            // bytes per x stage (1024-aligned)
     int tmem_cols, a_col;   // TMEM allocation and first A column
+    int csplit;             // 1, or 2: a 2-CTA cluster per tile, each CTA half of the chunks
+    int ksplit;             // csplit 2: rank 0 takes chunks [0, ksplit), rank 1 [ksplit, nch)
+    int red_pitch;          // csplit 2: floats per row of the reduction buffer (OCN + 4)
 };
 
 // ---- packed per-chunk parameters (written once per call by op_pack_kernel into the caller's
@@ -162,7 +165,10 @@ __global__ void __maxnreg__(OP_REGS)
     uint64_t* mma_done = afull + 2;                            // [2] half h's MMAs complete
     uint64_t* sfree = mma_done + 2;                            // [XS] stage's last MMAs complete
     uint64_t* acc_full = sfree + a.XS;                         // all MMAs complete
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_full + 1);
+    uint64_t* red_full = acc_full + 1;                         // csplit 2: rank 1's partial landed
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(red_full + 1);
+    // csplit 2: rank 1's fp32 accumulator, stored into rank 0's copy of this buffer ([128][pitch])
+    float* red = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(tmem_slot) + 16 + 15) & ~uintptr_t(15));
     float* out_s = reinterpret_cast<float*>(smem);             // epilogue staging (stages)
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -170,7 +176,12 @@ __global__ void __maxnreg__(OP_REGS)
     const int nblk = TP >> 4;                                  // 16-lane blocks (<= 4)
     const int issuer_warp = nblk < 4 ? 3 : 8;                  // ids no compute warp uses
     const int loader_warp = nblk < 4 ? 7 : 9;
-    const int v0 = blockIdx.x * TP;                            // first virtual pixel of the tile
+    // channel split: the two CTAs of a cluster share the tile, each with half of the chunks
+    const int crank = a.csplit == 2 ? (int)cluster_ctarank() : 0;
+    const int tile = a.csplit == 2 ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+    const int kc0 = crank == 0 ? 0 : a.ksplit;
+    const int kc1 = a.csplit == 2 && crank == 0 ? a.ksplit : a.nch;
+    const int v0 = tile * TP;                                  // first virtual pixel of the tile
     const uint32_t tcols = a.tmem_cols;
     const uint32_t ACOL = a.a_col;                             // first A column (after the accumulator)
 
@@ -188,6 +199,7 @@ __global__ void __maxnreg__(OP_REGS)
             mbar_init(&mma_done[b], 1);
         }
         mbar_init(acc_full, 1);
+        mbar_init(red_full, 64 * (nblk < 4 ? nblk : 4));   // every compute thread of rank 1
         fence_barrier_init();
         tma_prefetch_desc(&xmap);
     }
@@ -198,6 +210,7 @@ __global__ void __maxnreg__(OP_REGS)
     }
     tc_fence_before();
     __syncthreads();
+    if (a.csplit == 2) cluster_sync_all();   // rank 0's red_full initialised before rank 1 arrives
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
     OPTL(1);
@@ -219,12 +232,13 @@ __global__ void __maxnreg__(OP_REGS)
                 tma_load_3d(st, &xmap, &xfull[s], k * OP_KC, -a.pw, Y0);
                 bulk_load(st + a.x_stage, a.packed + (size_t)k * PBLK, (uint32_t)PBLK, &xfull[s]);
             };
-            for (int k = 0; k < a.XS && k < a.nch; ++k) load_stage(k, k);
-            for (int k = a.XS; k < a.nch; ++k) {   // stage of chunk k - XS: its MMAs are done
-                const int s = k % a.XS;
-                mbar_wait(&sfree[s], (uint32_t)((k - a.XS) / a.XS) & 1u);
-                if (k < 8) OPTL_ANY(32 + k);
-                load_stage(k, s);
+            const int nk = kc1 - kc0;                // this CTA's chunks kc0 .. kc1-1
+            for (int i = 0; i < a.XS && i < nk; ++i) load_stage(kc0 + i, i);
+            for (int i = a.XS; i < nk; ++i) {      // stage of chunk i - XS: its MMAs are done
+                const int s = i % a.XS;
+                mbar_wait(&sfree[s], (uint32_t)((i - a.XS) / a.XS) & 1u);
+                if (i < 8) OPTL_ANY(32 + i);
+                load_stage(kc0 + i, s);
             }
         }
         return;
@@ -234,7 +248,7 @@ __global__ void __maxnreg__(OP_REGS)
         if (lane == 0) {
             const uint32_t idesc = make_idesc(2u /*TF32*/, 128, (uint32_t)a.OCN);
             int s = 0;
-            for (int k = 0; k < a.nch; ++k) {
+            for (int k = 0; k < kc1 - kc0; ++k) {   // local chunk index
                 const uint32_t bh = smem_u32(st_base + s * STG + a.x_stage), bl = bh + B_PLANE;
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {
@@ -301,7 +315,7 @@ __global__ void __maxnreg__(OP_REGS)
 
     int s = 0;                          // stage of chunk k (k mod XS)
     uint32_t xphase = 0;
-    for (int k = 0; k < a.nch; ++k) {
+    for (int k = 0; k < kc1 - kc0; ++k) {   // local chunk index (chunk kc0 + k)
         const uint8_t* xst = st_base + s * STG;
         const float* wk = reinterpret_cast<const float*>(xst + a.x_stage) + wofs;
         mbar_wait(&xfull[s], xphase);
@@ -419,6 +433,31 @@ __global__ void __maxnreg__(OP_REGS)
     mbar_wait(acc_full, 0u);
     tc_fence_after();
     OPTL(21);
+    if (a.csplit == 2 && crank == 1) {
+        // rank 1: its partial accumulator (its half of the channels) into rank 0's red buffer,
+        // one release-arrive per thread, then leave; rank 0 finishes the tile
+        const int ngrp = a.OCN >> 4;
+        const int row = 32 * qd + lane;                        // TMEM lane = red row
+        for (int cg = half; cg < ngrp; cg += 2) {
+            uint32_t vv[16];
+            tmem_ld_32x32b_x16(tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(16 * cg), vv);
+            tmem_ld_wait();
+            const uint32_t la = smem_u32(red + row * a.red_pitch + 16 * cg);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) st_cluster_v4(la + 16 * u, 0, vv[4 * u], vv[4 * u + 1], vv[4 * u + 2], vv[4 * u + 3]);
+        }
+        mbar_arrive_release_cluster(red_full, 0);
+        tc_fence_before();
+        named_bar_sync(3, NC);   // TMEM no longer read
+        if (warp == 0) {
+            tc_fence_after();
+            if (tcols == 128) tmem_dealloc<128>(tmem);
+            else if (tcols == 256) tmem_dealloc<256>(tmem);
+            else tmem_dealloc<512>(tmem);
+        }
+        return;
+    }
+    if (a.csplit == 2) mbar_wait_cluster(red_full, 0u);   // rank 1's partial is in red
     const int vl = min(v0 + TP, a.MV) - 1;
     auto real_m = [&](int v, bool up) {   // m of virtual pixel v (dead column: next / previous real)
         const int r = v / a.Wv, c = v - r * a.Wv;
@@ -445,6 +484,7 @@ __global__ void __maxnreg__(OP_REGS)
             for (int u = 0; u < 16; ++u) {
                 const int o = 16 * cg + u;
                 const float val = __uint_as_float(vv[u]) +
+                                  (a.csplit == 2 ? red[(32 * qd + lane) * a.red_pitch + o] : 0.f) +
                                   (cg == half ? bias_r[u] : (a.pw_b && o < a.OC) ? __ldg(a.pw_b + o) : 0.f);
                 if (o < a.n_off) off_s[dm * a.n_off + o] = val;
                 else if (o < a.OC) msk_s[dm * a.n_msk + (o - a.n_off)] = __fdividef(1.f, 1.f + __expf(-val));
@@ -487,13 +527,24 @@ constexpr size_t OP_SMEM_TWO = 113 * 1024;   // two CTAs per SM
 #endif
 
 size_t op_smem(const OpArgs& a) {
-    return 1024 + (size_t)a.XS * (a.x_stage + op_block_bytes(a.OCN)) + 2048 + (2 * a.XS + 5) * 8 + 16;
+    return 1024 + (size_t)a.XS * (a.x_stage + op_block_bytes(a.OCN)) + 2048 + (2 * a.XS + 6) * 8 + 16 +
+           (a.csplit == 2 ? (size_t)128 * a.red_pitch * 4 + 16 : 0);
 }
 
 // Tile = TP consecutive pixels of the virtual [N][Ho][Wv] grid (a tile may run across an image
 // boundary: its input window covers the stacked N*H rows, and taps in another image's rows are
 // masked as zero padding).  TP (a multiple of 16, <= 128 = the UMMA M) spreads the pixels evenly
 // over the CTA slots: minimise rounds x CTAs-per-SM x TP, the pixels one SM processes.
+// Tile size / channel split measured per layer shape and per-GPU batch by tools/autotune.py
+// (branch_tuning_table.inc, compiled in); shapes not in it take the time model below.
+struct OpTuneEntry {
+    int C, H, W, stride, OC, nmin, nmax, TP, csplit;
+};
+static const OpTuneEntry kOpTuneTable[] = {
+#include "branch_tuning_table.inc"
+    {0, 0, 0, 0, 0, 0, 0, 0, 0}   // terminator
+};
+
 bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, int ph, int pw, int dh, int dw,
                   int OC, int es, OpPlan* p) {
     OpArgs& a = p->a;
@@ -517,15 +568,32 @@ bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, in
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     }
-    long best = LONG_MAX;
+    double best = 1e30;
     bool found = false;
+    int force_split = 0, force_tp = 0;
+    for (const OpTuneEntry* e = kOpTuneTable; e->C; ++e)
+        if (e->C == C && e->H == H && e->W == W && e->stride == sh && sw == sh && e->OC == OC && N >= e->nmin &&
+            N <= e->nmax && dh == 1 && dw == 1) {
+            force_tp = e->TP;
+            force_split = e->csplit;
+            break;
+        }
+    // DEFCON_OP_TP / DEFCON_OP_CSPLIT override the table (the autotune sweep, tests)
+    if (const char* env = getenv("DEFCON_OP_TP")) force_tp = atoi(env);
+    if (const char* env = getenv("DEFCON_OP_CSPLIT")) force_split = atoi(env);
+    OpArgs best_t = a;
+    auto search = [&](int ftp, int fsplit) {
+    for (int cs = 1; cs <= 2; ++cs)
     for (int TP = 16; TP <= 128; TP += 16) {
+        if (fsplit && cs != fsplit) break;
+        if (cs == 2 && a.nch < 2) break;
         if (TP > Ho * a.Wv && TP > 16) break;     // a tile spans at most two images
-#ifdef OP_PROBE_TP   // dev probe: force the tile size
-        if (TP != OP_PROBE_TP) continue;
-#endif
+        if (ftp && TP != ftp) continue;
         OpArgs t = a;
         t.TP = TP;
+        t.csplit = cs;
+        t.ksplit = (a.nch + 1) / 2;
+        t.red_pitch = a.OCN + 4;
         const int orows = (a.Wv - 2 + TP + a.Wv - 1) / a.Wv;          // output rows a tile can touch
         t.IR = (orows - 1) * sh + std::max(0, H - Ho * sh) + 2 * dh + 1;
         if (t.IR > 256) continue;
@@ -543,25 +611,35 @@ bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, in
         cps = std::min(cps, 4 * (16384 / (OP_REGS * 32)) / nwarps);
         if (cps < 1) continue;
         const long tiles = (MV + TP - 1) / TP;
-        const long rounds = (tiles + (long)sms * cps - 1) / ((long)sms * cps);
-        const long cost = rounds * cps * (TP + 16);   // + a per-tile overhead: ties go to larger tiles
+        const long ctas = tiles * cs;
+        const long rounds = (ctas + (long)sms * cps - 1) / ((long)sms * cps);
+        // time model: every CTA is a latency chain of its chunks (cost per chunk grows with the
+        // pixels per compute warp and with the CTAs sharing the SM) plus a fixed prologue /
+        // epilogue (the channel split adds the DSMEM reduction)
+        const int kper = cs == 2 ? std::max(t.ksplit, a.nch - t.ksplit) : a.nch;
+        const double per_chunk = (TP + 16) / 80.0 * (0.55 + 0.15 * std::min<long>(cps, (ctas + sms - 1) / sms));
+        const double cost = rounds * (kper * per_chunk + 4.0 + (cs == 2 ? 0.7 : 0.0));
         if (cost < best) {
             best = cost;
-            a = t;
-            p->tiles = (int)tiles;
+            best_t = t;
+            p->tiles = (int)ctas;
             p->cps = cps;
             p->smem = sm;
             found = true;
         }
     }
+    };
+    search(force_tp, force_split);
+    if (!found && (force_tp || force_split)) search(0, 0);   // a table entry that no longer fits
+    if (found) a = best_t;
     return found;
 }
 
 template <int ES>
 cudaError_t launch_op(const OpPlan& p, const CUtensorMap& xmap, cudaStream_t stream) {
     if (getenv("DEFCON_DEBUG"))
-        fprintf(stderr, "defcon onepass: TP=%d tiles=%d cps=%d XS=%d IR=%d IC=%d smem=%zu tmem=%d\n", p.a.TP,
-                p.tiles, p.cps, p.a.XS, p.a.IR, p.a.IC, p.smem, p.a.tmem_cols);
+        fprintf(stderr, "defcon onepass: TP=%d ctas=%d csplit=%d cps=%d XS=%d IR=%d IC=%d smem=%zu tmem=%d\n",
+                p.a.TP, p.tiles, p.a.csplit, p.cps, p.a.XS, p.a.IR, p.a.IC, p.smem, p.a.tmem_cols);
     const bool s1 = p.a.sw == 1 && p.a.dw == 1;
     auto kern = s1 ? offset_branch_onepass_kernel<ES, true> : offset_branch_onepass_kernel<ES, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
@@ -569,7 +647,22 @@ cudaError_t launch_op(const OpPlan& p, const CUtensorMap& xmap, cudaStream_t str
     const int nblk = p.a.TP / 16;
     // compute warps 0..nblk-1 (half 0), 4..3+nblk (half 1); issuer + loader: 3, 7 or 8, 9
     const int threads = 32 * (nblk < 4 ? 8 : 10);
-    return launch_pdl(kern, dim3(p.tiles), dim3(threads), p.smem, stream, xmap, p.a);
+    if (p.a.csplit != 2) return launch_pdl(kern, dim3(p.tiles), dim3(threads), p.smem, stream, xmap, p.a);
+    cudaLaunchConfig_t cfg = {};   // 2-CTA clusters (the channel split) + PDL
+    cfg.gridDim = dim3(p.tiles);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = p.smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 2;
+    return cudaLaunchKernelEx(&cfg, kern, xmap, p.a);
 }
 
 }  // namespace
