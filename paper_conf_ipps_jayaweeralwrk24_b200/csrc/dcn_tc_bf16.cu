@@ -783,12 +783,19 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
             Smp::store(L[p], stage + dst_lo[p], stage + dst_hi[p]);
             if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
         }
+#ifdef DEFCON_PROBE_NO_FENCE   // dev probe (WRONG results): no proxy fence, relaxed arrive -- the
+                               // cost of ordering the A stores before the MMA
+        __syncwarp();
+        if (lane == 0)
+            asm volatile("mbarrier.arrive.relaxed.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&full_a[s])) : "memory");
+#else
         fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) {
             if (PAIR) mbar_arrive_cluster(&full_a[s], 0);   // the pair's MMA issuer is rank 0
             else mbar_arrive(&full_a[s]);
         }
+#endif
         if (t == 0) KT(2, q);
         if (t == 224) KT(7, q);   // the last producer warp
 
