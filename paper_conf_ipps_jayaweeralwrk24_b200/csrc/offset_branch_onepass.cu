@@ -84,6 +84,8 @@ struct OpArgs {
     int XS;                 // x stages in flight
     int x_stage;            // bytes per x stage (1024-aligned)
     int tmem_cols, a_col;   // TMEM allocation and first A column
+    unsigned long long wv_mul, howv_mul;   // n / Wv, n / (Ho*Wv) as (n * mul) >> (32 + shr)
+    int wv_shr, howv_shr;
     int csplit;             // 1, or 2: a 2-CTA cluster per tile, each CTA half of the chunks
     int ksplit;             // csplit 2: rank 0 takes chunks [0, ksplit), rank 1 [ksplit, nch)
     int red_pitch;          // csplit 2: floats per row of the reduction buffer (OCN + 4)
@@ -149,6 +151,16 @@ __global__ void __launch_bounds__(256) op_pack_kernel(const float* __restrict__ 
 // (x window by TMA + the chunk's packed parameters by bulk copy) once the chunk's last MMAs,
 // which follow both halves' reads of the stage, have completed.
 constexpr int OP_REGS = 64;            // registers per thread (__maxnreg__)
+// n / d for 0 <= n < 2^32 by a multiply and a shift (m = ceil(2^(32+s) / d), s = ceil(log2 d))
+__device__ __forceinline__ int op_div(int n, unsigned long long mul, int shr) {
+    return (int)(((unsigned long long)(unsigned)n * mul) >> (32 + shr));
+}
+static void op_div_init(int d, unsigned long long* mul, int* shr) {
+    int s = 0;
+    while ((1ll << s) < d) ++s;
+    *shr = s;
+    *mul = ((1ull << (32 + s)) + (unsigned long long)d - 1) / (unsigned long long)d;
+}
 template <int ES, bool S1>
 __global__ void __maxnreg__(OP_REGS)
     offset_branch_onepass_kernel(const __grid_constant__ CUtensorMap xmap, const OpArgs a) {
@@ -220,7 +232,7 @@ __global__ void __maxnreg__(OP_REGS)
     OPTL(2);
 
     const int HoWv = a.Ho * a.Wv;
-    const int n0 = v0 / HoWv, ho0 = (v0 - n0 * HoWv) / a.Wv;
+    const int n0 = op_div(v0, a.howv_mul, a.howv_shr), ho0 = op_div(v0 - n0 * HoWv, a.wv_mul, a.wv_shr);
     const int Y0 = n0 * a.H + ho0 * a.sh - a.ph;              // window origin (stacked rows)
 
     if (warp == loader_warp) {
@@ -295,9 +307,9 @@ __global__ void __maxnreg__(OP_REGS)
         const int vp = v0 + 2 * q;                             // virtual pixel of the left one
         const bool pix_ok = sb < nsub && vp < a.MV;
         const int vpc = pix_ok ? vp : v0;
-        const int n = vpc / HoWv;
+        const int n = op_div(vpc, a.howv_mul, a.howv_shr);
         const int rem = vpc - n * HoWv;
-        const int ho = rem / a.Wv, wo = rem - ho * a.Wv;       // wo even
+        const int ho = op_div(rem, a.wv_mul, a.wv_shr), wo = rem - ho * a.Wv;   // wo even
         row_ok[sb] = 0;
 #pragma unroll
         for (int i = 0; i < 3; ++i) {
@@ -461,7 +473,7 @@ __global__ void __maxnreg__(OP_REGS)
     if (a.csplit == 2) mbar_wait_cluster(red_full, 0u);   // rank 1's partial is in red
     const int vl = min(v0 + TP, a.MV) - 1;
     auto real_m = [&](int v, bool up) {   // m of virtual pixel v (dead column: next / previous real)
-        const int r = v / a.Wv, c = v - r * a.Wv;
+        const int r = op_div(v, a.wv_mul, a.wv_shr), c = v - r * a.Wv;
         if (c >= a.Wo) return up ? (r + 1) * a.Wo : r * a.Wo + a.Wo - 1;
         return r * a.Wo + c;
     };
@@ -472,7 +484,7 @@ __global__ void __maxnreg__(OP_REGS)
     {
         const int li = lane & 15, bb = qd + 4 * (lane >> 4);
         const int v = v0 + 2 * (8 * bb + (li & 7)) + (li >> 3);   // virtual pixel of lane 32*qd + lane
-        const int rr = v / a.Wv, cc = v - rr * a.Wv;
+        const int rr = op_div(v, a.wv_mul, a.wv_shr), cc = v - rr * a.Wv;
         const bool ok = bb < nblk && v < a.MV && cc < a.Wo;
         const int dm = rr * a.Wo + cc - mf;                   // real-pixel index within the tile
         const int ngrp = a.OCN >> 4;                           // 16-column groups
@@ -496,20 +508,20 @@ __global__ void __maxnreg__(OP_REGS)
     tc_fence_before();
     named_bar_sync(3, NC);   // staged; TMEM no longer read
     OPTL(30);
-    if (warp == 0) {
-        tc_fence_after();
-        if (tcols == 128) tmem_dealloc<128>(tmem);
-        else if (tcols == 256) tmem_dealloc<256>(tmem);
-        else tmem_dealloc<512>(tmem);
-    }
-    OPTL(31);
-    {
+    {   // the stores first (fire and forget), the TMEM release after them
         const long go = (long)mf * a.n_off;
         for (int e = ctid; e < nreal * a.n_off; e += NC) st_offset1(a.offset, go + e, off_s[e], a.out_f16);
         if (a.n_msk) {
             const long gm = (long)mf * a.n_msk;
             for (int e = ctid; e < nreal * a.n_msk; e += NC) st_offset1(a.mask, gm + e, msk_s[e], a.out_f16);
         }
+    }
+    OPTL(31);
+    if (warp == 0) {
+        tc_fence_after();
+        if (tcols == 128) tmem_dealloc<128>(tmem);
+        else if (tcols == 256) tmem_dealloc<256>(tmem);
+        else tmem_dealloc<512>(tmem);
     }
     OPTL(22);
 }
@@ -557,6 +569,8 @@ bool make_op_plan(int N, int H, int W, int C, int Ho, int Wo, int sh, int sw, in
     const long MV = (long)N * Ho * a.Wv;
     if (a.OCN > 256 || C % 8 != 0 || MV >= (1L << 31)) return false;
     a.MV = (int)MV;
+    op_div_init(a.Wv, &a.wv_mul, &a.wv_shr);
+    op_div_init(Ho * a.Wv, &a.howv_mul, &a.howv_shr);
     a.nch = (C + OP_KC - 1) / OP_KC;
     a.IC = (a.Wv - 1) * sw + 2 * dw + 1;
     if (a.IC > 256) return false;                 // TMA box limit: wide images keep the two-pass path
