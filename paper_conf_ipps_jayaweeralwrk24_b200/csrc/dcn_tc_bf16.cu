@@ -48,11 +48,15 @@ struct Elem {
     static constexpr int A_STAGE = A_PLANE * PLANES;
 };
 constexpr int META_ENTRY = 32;   // int4 corner offsets + float4 weights
-constexpr int NPW = 8;           // producer warps
-constexpr int EPI_WARP0 = 8;     // 4 epilogue warps: TMEM lane quarters 0..3
-constexpr int TMA_WARP = 12;
-constexpr int MMA_WARP = 13;
-constexpr int NUM_THREADS = 14 * 32;
+#ifndef DEFCON_NPW
+#define DEFCON_NPW 8
+#endif
+constexpr int NPW = DEFCON_NPW;  // producer warps (8 or 16)
+constexpr int EPI_WARP0 = NPW;   // 4 epilogue warps: TMEM lane quarters 0..3
+constexpr int TMA_WARP = NPW + 4;
+constexpr int MMA_WARP = NPW + 5;
+constexpr int NUM_THREADS = (NPW + 6) * 32;
+constexpr int FEPI_WARPS = 8;    // producer warps that run the CTA's last epilogue
 constexpr int NPT = NPW * 32;
 constexpr int TPR = 4;               // producer threads per 128-byte A row (32 bytes each)
 constexpr int ROWS = BM * TPR / NPT; // A rows per producer thread
@@ -239,30 +243,31 @@ __device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& 
     *reinterpret_cast<float4*>(e + 16) = wt;
 }
 
-// The whole (tile, group) table, built by the NPT = 2*BM producer threads: thread t owns
-// row t/2 and taps (t&1), (t&1)+2, ...  The row's pixel decomposition is done once; the
+// The whole (tile, group) table, built by the NPT = TPM * BM producer threads: thread t owns
+// row t / TPM and taps t % TPM, + TPM, ...  The row's pixel decomposition is done once; the
 // offset/mask loads of a pass are all issued before any arithmetic (one round trip per
 // pass).  Rows of warp w use the format of that warp's sampler.
-static_assert(NPT == 2 * BM, "metadata build assumes two producer threads per tile row");
+constexpr int TPM = NPT / BM;    // producer threads per tile row in the metadata build
+static_assert(NPT % BM == 0, "metadata build assumes whole producer threads per tile row");
 #ifndef DEFCON_META_PASS
 #define DEFCON_META_PASS 3
 #endif
 template <int NTEX>
 __device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t) {
     constexpr int PASS = DEFCON_META_PASS;   // taps in flight per thread (register budget)
-    const int row = t >> 1;
+    const int row = t / TPM;
     const RowPos rp = row_pos(a, m0 + row);
     const bool tex_row = ((row % (NPW * RPW)) / RPW) < NTEX;
     const long pix = (long)(m0 + row) * a.G + g;
     uint8_t* rmeta = meta + row * a.KK * META_ENTRY;
-    int tap = t & 1;
+    int tap = t % TPM;
     int i = tap / a.Kw, j = tap - (tap / a.Kw) * a.Kw;
 #pragma unroll 1
     for (; tap < a.KK;) {
         MetaIn in[PASS];
 #pragma unroll
         for (int k = 0; k < PASS; ++k) {
-            const int tk = tap + 2 * k;
+            const int tk = tap + TPM * k;
             in[k].d = make_float2(0.f, 0.f);
             in[k].mk = 0.f;
             if (rp.ok && tk < a.KK) {
@@ -276,8 +281,8 @@ __device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g,
 #pragma unroll
         for (int k = 0; k < PASS; ++k) {
             if (tap < a.KK) store_meta_entry(a, rp, i, j, in[k], rmeta + tap * META_ENTRY, tex_row);
-            tap += 2;
-            j += 2;
+            tap += TPM;
+            j += TPM;
             while (j >= a.Kw) { j -= a.Kw; ++i; }
         }
     }
@@ -918,7 +923,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         // Its store scratch reuses the A stages other producer threads wrote: ordered already
         // through full_a -> MMA -> tmem_full, a barrier the race checker can see makes it explicit.
         named_bar_sync(1, NPT);
-        if (nseg > 0) {
+        if (nseg > 0 && warp < FEPI_WARPS) {
             const int o = nseg - 1;
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
             const int buf = o % Cfg::NBUF;
@@ -927,11 +932,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const int qd = warp & 3;
             const int r = qd * 32 + lane;
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * Cfg::ACC_STRIDE);
-            constexpr int SLICE = BLOCK_N / (NPW / 4);
+            constexpr int SLICE = BLOCK_N / (FEPI_WARPS / 4);
             if (t == 0) TL(12);
             // idle pipeline buffers: A stages hold the per-warp store scratch, B stages the
             // staged stream-K partials
-            epilogue_segment<BLOCK_N, SLICE, PAIR, F32>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 1, NPT,
+            epilogue_segment<BLOCK_N, SLICE, PAIR, F32>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 4,
+                                                  FEPI_WARPS * 32,
                                                   t == 0, fix_flag + 1, T, nct, a.bias_in_smem ? bias_s : nullptr,
                                                   sA + warp * EPI_W, sB,
                                              (size_t)STAGES * Cfg::B_STAGE_BYTES, t);
