@@ -210,10 +210,13 @@ int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, in
  * to the device, runs step 1 and step 2, copies y back to y_host and synchronises
  * `stream` before returning.  Parameters dw_* / pw_* / weight / bias are device
  * pointers (resident model weights), as in the two calls above.  Images are independent
- * (P:58 is per output pixel), so the batch is cut into min(N, 2) image ranges
- * (DEFCON_HOST_CHUNKS overrides) that flow H2D -> step 1 -> step 2 -> D2H on two
- * internal streams ordered after the caller's prior work on `stream`: the copies of
- * one range overlap the kernels of the other.  The internal streams / events are
+ * (P:58 is per output pixel), so the batch is cut into min(N, 4) image ranges
+ * (DEFCON_HOST_CHUNKS overrides, at most 16) that flow H2D -> step 1 -> step 2 -> D2H,
+ * ordered after the caller's prior work on `stream`: the host-to-device and the
+ * device-to-host copies each run on an internal stream of their own, back to back in
+ * range order, the kernels of a range on one of two internal compute streams once its
+ * copy has landed (per-range events), so the copy engines of both directions stay busy
+ * while earlier ranges compute.  The internal streams / events are
  * created once per process on first use; concurrent calls are serialised.  Only
  * DEFCON_SAMPLER_LDG is accepted (UNSUPPORTED otherwise: the entry owns no texture plan).
  * Every per-chunk device region is 256-byte aligned whatever the per-image sizes.  If an

@@ -319,11 +319,12 @@ static size_t align_up(size_t v) { return (v + 255) & ~size_t(255); }
 constexpr int HOST_PIPE_STREAMS = 2;
 
 static int host_chunks(int N) {
-    int k = N < 2 ? N : 2;
+    int k = N < 4 ? N : 4;
     if (const char* env = getenv("DEFCON_HOST_CHUNKS")) {
         const int v = atoi(env);
         if (v > 0) k = v < N ? v : N;
     }
+    k = k < 16 ? k : 16;   // HOST_MAX_CHUNKS
     return k > 0 ? k : 1;
 }
 
@@ -391,12 +392,17 @@ int defcon_layer_workspace_size(int N, int H, int W, int Cin, int dtype, int Cou
     return DEFCON_OK;
 }
 
-// Two internal streams and their completion events, created once per process on first use
-// (the only resources the host entry point keeps); calls are serialised by a mutex.
+// Internal streams and events, created once per process on first use (the only resources the
+// host entry point keeps); calls are serialised by a mutex.  Copies have streams of their own
+// (one host-to-device, one device-to-host, each in chunk order) so the copy engines stream
+// back to back while the compute streams work on earlier chunks; per-chunk events link them.
+constexpr int HOST_MAX_CHUNKS = 16;
 struct HostPipe {
     int dev = -1;
-    cudaStream_t s[HOST_PIPE_STREAMS] = {};
-    cudaEvent_t start = nullptr, done[HOST_PIPE_STREAMS] = {};
+    cudaStream_t s[HOST_PIPE_STREAMS] = {};   // compute
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t start = nullptr, done[HOST_PIPE_STREAMS] = {}, h2d_done = nullptr, d2h_done = nullptr;
+    cudaEvent_t in[HOST_MAX_CHUNKS] = {}, out[HOST_MAX_CHUNKS] = {};   // chunk k landed / computed
 };
 static std::mutex g_pipe_mu;
 static HostPipe g_pipe;
@@ -413,6 +419,14 @@ static cudaError_t host_pipe_ready() {
         if ((e = cudaEventCreateWithFlags(&p.done[i], cudaEventDisableTiming)) != cudaSuccess) return e;
     }
     if ((e = cudaEventCreateWithFlags(&p.start, cudaEventDisableTiming)) != cudaSuccess) return e;
+    if ((e = cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking)) != cudaSuccess) return e;
+    if ((e = cudaStreamCreateWithFlags(&p.d2h, cudaStreamNonBlocking)) != cudaSuccess) return e;
+    if ((e = cudaEventCreateWithFlags(&p.h2d_done, cudaEventDisableTiming)) != cudaSuccess) return e;
+    if ((e = cudaEventCreateWithFlags(&p.d2h_done, cudaEventDisableTiming)) != cudaSuccess) return e;
+    for (int k = 0; k < HOST_MAX_CHUNKS; ++k) {
+        if ((e = cudaEventCreateWithFlags(&p.in[k], cudaEventDisableTiming)) != cudaSuccess) return e;
+        if ((e = cudaEventCreateWithFlags(&p.out[k], cudaEventDisableTiming)) != cudaSuccess) return e;
+    }
     g_pipe = p;   // a previous device's objects are left to process teardown
     return cudaSuccess;
 }
@@ -447,47 +461,77 @@ int defcon_layer_forward_host(const void* x_host, int N, int H, int W, int Cin, 
     if ((e = cudaEventRecord(g_pipe.start, st)) != cudaSuccess) return cuda_fail(e, "event record");
     for (int i = 0; i < HOST_PIPE_STREAMS; ++i)
         if ((e = cudaStreamWaitEvent(g_pipe.s[i], g_pipe.start, 0)) != cudaSuccess) return cuda_fail(e, "event wait");
+    if ((e = cudaStreamWaitEvent(g_pipe.h2d, g_pipe.start, 0)) != cudaSuccess) return cuda_fail(e, "event wait");
+    if ((e = cudaStreamWaitEvent(g_pipe.d2h, g_pipe.start, 0)) != cudaSuccess) return cuda_fail(e, "event wait");
     // Any failure after the first enqueue: drain the internal streams before returning, so no
     // copy still reads x_host / writes y_host once the caller sees the error.
     auto bail = [&](int status) {
         for (int i = 0; i < HOST_PIPE_STREAMS; ++i) cudaStreamSynchronize(g_pipe.s[i]);
+        cudaStreamSynchronize(g_pipe.h2d);
+        cudaStreamSynchronize(g_pipe.d2h);
         return status;
     };
-    bool cleared[HOST_PIPE_STREAMS] = {};
+    // per-range device regions
+    struct Range {
+        uint8_t *x, *y;
+        float *off, *msk;
+        int n0, nc;
+    } rg[HOST_MAX_CHUNKS];
+    for (int k = 0; k < c.nchunk; ++k) {
+        Range& r = rg[k];
+        r.n0 = k * c.per;
+        r.nc = std::min(c.per, N - r.n0);
+        const ChunkCarve cc = chunk_carve(g, dtype, Cout, modulated, r.nc);
+        r.x = cur;
+        r.y = r.x + cc.x;
+        r.off = reinterpret_cast<float*>(r.y + cc.y);
+        r.msk = modulated ? reinterpret_cast<float*>(r.y + cc.y + cc.off) : nullptr;
+        cur += cc.total();
+    }
+    // the caller's workspace carries no zero-fill guarantee: clear step 2's tile counters once
+    // per compute stream (self-cleaning after every launch)
+    for (int si = 0; si < HOST_PIPE_STREAMS && si < c.nchunk; ++si)
+        if (c.ws && c.ctr_bytes) {
+            e = cudaMemsetAsync(wsbase + si * (c.ws + c.tws) + c.ctr_off, 0, c.ctr_bytes, g_pipe.s[si]);
+            if (e != cudaSuccess) return bail(cuda_fail(e, "workspace clear"));
+        }
+    // every host-to-device copy first, back to back on the copy stream
+    for (int k = 0; k < c.nchunk; ++k) {
+        e = cudaMemcpyAsync(rg[k].x, static_cast<const uint8_t*>(x_host) + rg[k].n0 * x_img, rg[k].nc * x_img,
+                            cudaMemcpyHostToDevice, g_pipe.h2d);
+        if (e == cudaSuccess) e = cudaEventRecord(g_pipe.in[k], g_pipe.h2d);
+        if (e != cudaSuccess) return bail(cuda_fail(e, "H2D copy of x"));
+    }
     for (int k = 0; k < c.nchunk; ++k) {
         const int si = k % HOST_PIPE_STREAMS;
         cudaStream_t s = g_pipe.s[si];
-        const int n0 = k * c.per, nc = std::min(c.per, N - n0);
-        const ChunkCarve cc = chunk_carve(g, dtype, Cout, modulated, nc);
-        uint8_t* xk = cur;
-        uint8_t* yk = xk + cc.x;
-        float* offd = reinterpret_cast<float*>(yk + cc.y);
-        float* mskd = modulated ? reinterpret_cast<float*>(yk + cc.y + cc.off) : nullptr;
-        cur += cc.total();
+        const Range& r = rg[k];
         uint8_t* wsd = c.ws ? wsbase + si * (c.ws + c.tws) : nullptr;
         void* twsd = wsbase + si * (c.ws + c.tws) + c.ws;
-        e = cudaMemcpyAsync(xk, static_cast<const uint8_t*>(x_host) + n0 * x_img, nc * x_img,
-                            cudaMemcpyHostToDevice, s);
-        if (e != cudaSuccess) return bail(cuda_fail(e, "H2D copy of x"));
-        rc = defcon_offset_dw_conv(xk, nc, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
-                                   offd, mskd, twsd, c.tws, s);
+        e = cudaStreamWaitEvent(s, g_pipe.in[k], 0);   // compute after the range's copy
+        if (e != cudaSuccess) return bail(cuda_fail(e, "event wait"));
+        rc = defcon_offset_dw_conv(r.x, r.nc, H, W, Cin, dtype, dw_w, dw_scale, dw_shift, pw_w, pw_b, K, cv,
+                                   r.off, r.msk, twsd, c.tws, s);
         if (rc) return bail(rc);
-        if (wsd && c.ctr_bytes && !cleared[si]) {   // the caller's workspace carries no zero-fill
-            cleared[si] = true;      // guarantee: clear step 2's tile counters once (self-cleaning after)
-            e = cudaMemsetAsync(wsd + c.ctr_off, 0, c.ctr_bytes, s);
-            if (e != cudaSuccess) return bail(cuda_fail(e, "workspace clear"));
-        }
-        rc = defcon_dcn_forward(xk, nc, H, W, Cin, offd, mskd, weight, bias, Cout, K, K, cv, dtype,
-                                sampler, fp32_mode, yk, wsd, c.ws, nullptr, s);
+        rc = defcon_dcn_forward(r.x, r.nc, H, W, Cin, r.off, r.msk, weight, bias, Cout, K, K, cv, dtype,
+                                sampler, fp32_mode, r.y, wsd, c.ws, nullptr, s);
         if (rc) return bail(rc);
-        e = cudaMemcpyAsync(static_cast<uint8_t*>(y_host) + n0 * y_img, yk, nc * y_img,
-                            cudaMemcpyDeviceToHost, s);
+        e = cudaEventRecord(g_pipe.out[k], s);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(g_pipe.d2h, g_pipe.out[k], 0);   // copy after the compute
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(static_cast<uint8_t*>(y_host) + r.n0 * y_img, r.y, r.nc * y_img,
+                                cudaMemcpyDeviceToHost, g_pipe.d2h);
         if (e != cudaSuccess) return bail(cuda_fail(e, "D2H copy of y"));
     }
     for (int i = 0; i < HOST_PIPE_STREAMS; ++i) {
         if ((e = cudaEventRecord(g_pipe.done[i], g_pipe.s[i])) != cudaSuccess) return bail(cuda_fail(e, "event record"));
         if ((e = cudaStreamWaitEvent(st, g_pipe.done[i], 0)) != cudaSuccess) return bail(cuda_fail(e, "event wait"));
     }
+    if ((e = cudaEventRecord(g_pipe.h2d_done, g_pipe.h2d)) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(st, g_pipe.h2d_done, 0)) != cudaSuccess ||
+        (e = cudaEventRecord(g_pipe.d2h_done, g_pipe.d2h)) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(st, g_pipe.d2h_done, 0)) != cudaSuccess)
+        return bail(cuda_fail(e, "event record / wait"));
     e = cudaStreamSynchronize(st);
     if (e != cudaSuccess) return bail(cuda_fail(e, "stream synchronize"));
     return DEFCON_OK;

@@ -20,7 +20,7 @@ P = {k: torch.from_numpy(v).to(dev) for k, v in inputs.gen_offset_branch(c).item
 wd, bd = torch.from_numpy(w).to(dev, torch.bfloat16), torch.from_numpy(b).to(dev)
 xh = torch.from_numpy(x).to(torch.bfloat16).pin_memory()
 yh = torch.empty((c.N, c.Ho, c.Wo, c.Cout), dtype=torch.bfloat16).pin_memory()
-for k in (1, 2, 4, 8, 16):
+for k in (1, 2, 4, 6, 8, 16):
     os.environ["DEFCON_HOST_CHUNKS"] = str(k)
     ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout), dtype=torch.uint8, device=dev)
     call = lambda: d.defcon_layer_forward_host(xh, P, wd, bd, yh, ws)
@@ -53,7 +53,7 @@ print(f"bare H2D + D2H (serial, one stream): {a.elapsed_time(e) / 20 * 1e3:.1f} 
 
 if len(sys.argv) > 1 and sys.argv[1] == "trace":
     from torch.profiler import ProfilerActivity, profile
-    for k in (1, 4):
+    for k in (2, 4):
         os.environ["DEFCON_HOST_CHUNKS"] = str(k)
         ws = torch.empty(d.defcon_layer_workspace_size(c.N, c.H, c.W, c.Cin, c.Cout), dtype=torch.uint8, device=dev)
         d.defcon_layer_forward_host(xh, P, wd, bd, yh, ws)
