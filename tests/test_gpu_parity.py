@@ -393,6 +393,30 @@ def test_offset_branch_parity(oracle_mod, d, dev, c):
     assert 0.5 < float(np.std(ro)) < 4.0
 
 
+@pytest.mark.parametrize("tp,split", [(64, 1), (128, 1), (48, 2), (128, 2)])
+@pytest.mark.parametrize("c", [small("op_c96", Cin=96, N=2, H=23, W=19),                 # 3 chunks: 2 + 1 split
+                               configs.C4_G4.replace(N=2),                                 # OC 108 -> 112 columns
+                               small("op_s2_f32", dtype="f32", stride=2, Cin=64, H=25, W=21)],
+                         ids=lambda c: c.name)
+def test_offset_branch_tiles_and_channel_split(oracle_mod, d, dev, monkeypatch, c, tp, split):
+    """Every tile size / channel-split combination the tuning table can select (DEFCON_OP_TP /
+    DEFCON_OP_CSPLIT force them): one-pass kernel with all 128 TMEM lanes, and the 2-CTA
+    cluster whose rank 1 hands its half-of-the-channels accumulator to rank 0 through
+    distributed shared memory."""
+    monkeypatch.setenv("DEFCON_OP_TP", str(tp))
+    monkeypatch.setenv("DEFCON_OP_CSPLIT", str(split))
+    x = inputs.gen_x(c)
+    P, Pd = gen_branch_dev(c, dev)
+    off, msk = d.defcon_offset_dw_conv(to_dev(x, TDT[c.dtype], dev), Pd["dw_w"], Pd["dw_scale"], Pd["dw_shift"],
+                                       Pd["pw_w"], Pd["pw_b"], K=c.K, stride=c.stride, pad=c.pad, dil=c.dil,
+                                       offset_groups=c.G, with_mask=c.modulated)
+    torch.cuda.synchronize()
+    ro, rm = oracle_mod.offset_branch(x, P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"], P["pw_b"], K=c.K,
+                                      G=c.G, with_mask=c.modulated, stride=c.stride, pad=c.pad, dil=c.dil)
+    assert normwise(off.cpu().numpy(), ro) < 1e-5
+    assert np.max(np.abs(msk.cpu().numpy() - rm)) < 1e-5
+
+
 @pytest.mark.parametrize("chunks", [1, 2])
 def test_layer_chain_and_host_entry(oracle_mod, d, dev, monkeypatch, chunks):
     """Whole hot path (step 1 -> step 2) on C3 shapes (N reduced), device and host entry.
