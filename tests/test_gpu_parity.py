@@ -303,6 +303,27 @@ def test_dcn_3xtf32_stream_k_and_workspace_reuse(oracle_mod, d, dev, monkeypatch
     assert int(ctrs.count_nonzero()) == 0
 
 
+@pytest.mark.parametrize("env", [{"DEFCON_BLOCK_N": "128"}, {"DEFCON_BLOCK_N": "512"},
+                                 {"DEFCON_BLOCK_N": "256", "DEFCON_DCN_PAIR": "1", "DEFCON_MAX_CTAS": "132"},
+                                 {"DEFCON_BLOCK_N": "256", "DEFCON_MAX_CTAS": "96"}],
+                         ids=lambda e: "-".join(f"{k.split('_')[-1]}{v}" for k, v in e.items()))
+@pytest.mark.parametrize("c", [small("sched_c256", Cout=256, Cin=64, H=21, W=23),
+                               small("sched_c512_g2", Cout=512, Cin=128, G=2, N=1, H=18, W=17)],
+                         ids=lambda c: c.name)
+def test_dcn_schedule_overrides(oracle_mod, d, dev, monkeypatch, c, env):
+    """Every schedule the tuning table can select (BLOCK_N below / above Cout, CTA pairs on a
+    capped grid) computes the same layer: oracle parity and ulp-level agreement with the
+    default schedule (the workspace is sized for the schedule in force)."""
+    L = inputs.gen_layer(c)
+    y0 = run_dcn(d, dev, c, L)
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    y = run_dcn(d, dev, c, L)
+    ref = oracle_mod.dcn_forward(L["x"], L["offset"], L["weight"], L["bias"], mask=L["mask"], G=c.G)
+    assert normwise(y, ref) < REG["bf16"]
+    assert ulp_close(y, y0, np.max(np.abs(ref)))
+
+
 def test_dcn_deterministic(d, dev):
     c = small("det")
     L = inputs.gen_layer(c)
