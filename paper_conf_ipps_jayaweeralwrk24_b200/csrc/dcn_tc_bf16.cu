@@ -805,9 +805,11 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         if (t == 224) KT(7, q);   // the last producer warp
 
         if (has_next && !prefetch) {          // offset group changes: new table
+#ifndef DEFCON_PROBE_NO_REBUILD   // dev probe (WRONG results for G > 1): keep the first table
             named_bar_sync(1, NPT);
             build_meta_table<NTEX>(a, m0, ng, meta, t);
             named_bar_sync(1, NPT);
+#endif
             g = ng;
 #pragma unroll
             for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
