@@ -77,6 +77,21 @@ DEFCON_DEVICE void mbar_wait(uint64_t* bar, uint32_t parity) {
     }
 }
 
+// Spinning variant (mbarrier.test_wait, never suspends): for the single MMA-issuing thread,
+// whose wake-up latency after a suspended try_wait is exposed as a tensor-pipe bubble.
+DEFCON_DEVICE void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(ok)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    }
+}
+
 // ------------------------------------------------------------------ bounded deformation
 // P:182 (section III-A-c), reading R12: the offset d of a tap at regular displacement r from the
 // centre tap, restricted so that r + d stays in [-h, h] (the P x P window, h = (P-1)/2).
@@ -360,6 +375,33 @@ DEFCON_DEVICE uint32_t ld_shared_u32(uint32_t addr) {
     uint32_t v;
     asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
     return v;
+}
+
+DEFCON_DEVICE uint2 ld_shared_v2(uint32_t addr) {
+    uint2 r;
+    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "r"(addr));
+    return r;
+}
+
+// d = x * w + c with x the bf16 in half XH of `x`, w the bf16 in half WH of `w` and c, d fp32:
+// the bf16 x bf16 product is exact in fp32, one rounding for the sum (sm_100 mixed-precision
+// fma.rn.f32.bf16 -> SASS FHFMA.BF16; no bf16 -> fp32 unpack instruction needed).
+template <int XH, int WH>
+DEFCON_DEVICE float fma_bf16h(uint32_t x, uint32_t w, float c) {
+    float d;
+    if constexpr (XH == 0 && WH == 0)
+        asm("{.reg .b16 x0, x1, w0, w1;\n\tmov.b32 {x0, x1}, %1;\n\tmov.b32 {w0, w1}, %2;\n\t"
+            "fma.rn.f32.bf16 %0, x0, w0, %3;}" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+    else if constexpr (XH == 1 && WH == 0)
+        asm("{.reg .b16 x0, x1, w0, w1;\n\tmov.b32 {x0, x1}, %1;\n\tmov.b32 {w0, w1}, %2;\n\t"
+            "fma.rn.f32.bf16 %0, x1, w0, %3;}" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+    else if constexpr (XH == 0 && WH == 1)
+        asm("{.reg .b16 x0, x1, w0, w1;\n\tmov.b32 {x0, x1}, %1;\n\tmov.b32 {w0, w1}, %2;\n\t"
+            "fma.rn.f32.bf16 %0, x0, w1, %3;}" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+    else
+        asm("{.reg .b16 x0, x1, w0, w1;\n\tmov.b32 {x0, x1}, %1;\n\tmov.b32 {w0, w1}, %2;\n\t"
+            "fma.rn.f32.bf16 %0, x1, w1, %3;}" : "=f"(d) : "r"(x), "r"(w), "f"(c));
+    return d;
 }
 
 DEFCON_DEVICE uint4 ld_shared_v4(uint32_t addr) {

@@ -47,7 +47,10 @@ struct Elem {
     static constexpr int PLANES = F32 ? 2 : 1;       // operand planes (tf32 hi / lo)
     static constexpr int A_STAGE = A_PLANE * PLANES;
 };
-constexpr int META_ENTRY = 32;   // int4 corner offsets + float4 weights
+constexpr int META_ENTRY = 32;   // int4 corner offsets + float4 weights (bf16 x: 2 bf16 pairs)
+#ifndef DEFCON_BF16_WEIGHTS
+#define DEFCON_BF16_WEIGHTS 1        // bf16 x: bf16 corner weights, FHFMA.BF16 lerp (R20)
+#endif
 #ifndef DEFCON_NPW
 #define DEFCON_NPW 8
 #endif
@@ -63,7 +66,7 @@ constexpr int ROWS = BM * TPR / NPT; // A rows per producer thread
 constexpr int RPW = 32 / TPR;        // rows per warp per pass
 
 #ifdef DEFCON_PROBE_KTRACE   // dev probe: per-k-iteration event clock64 stamps of CTA `KTRACE_CTA`
-__device__ long long g_kt[8][64];
+__device__ long long g_kt[12][64];
 #ifndef KTRACE_CTA
 #define KTRACE_CTA 5
 #endif
@@ -240,6 +243,12 @@ __device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& 
         }
     }
     *reinterpret_cast<uint4*>(e) = off;
+#if DEFCON_BF16_WEIGHTS
+    if (a.es == 2) {   // bf16 x: the 4 weights as bf16 pairs, consumed by FHFMA.BF16 (lerp_store_row)
+        *reinterpret_cast<uint2*>(e + 16) = make_uint2(pack_bf16x2(wt.x, wt.y), pack_bf16x2(wt.z, wt.w));
+        return;
+    }
+#endif
     *reinterpret_cast<float4*>(e + 16) = wt;
 }
 
@@ -309,6 +318,53 @@ struct RowLoad {
     U8x32 v[4];
     float4 w;
 };
+// bf16 x: the same, weights as two bf16 pairs (w0, w1), (w2, w3).
+struct RowLoadB {
+    U8x32 v[4];
+    uint2 w;
+};
+
+__device__ __forceinline__ void issue_row_b(RowLoadB& L, const void* xbase, uint32_t meta_addr) {
+    const uint4 o = ld_shared_v4(meta_addr);
+    L.w = ld_shared_v2(meta_addr + 16);
+    L.v[0] = ldg_nc_v8(add_u32(xbase, o.x));
+    L.v[1] = ldg_nc_v8(add_u32(xbase, o.y));
+    L.v[2] = ldg_nc_v8(add_u32(xbase, o.z));
+    L.v[3] = ldg_nc_v8(add_u32(xbase, o.w));
+}
+
+// Eq.3 for 16 bf16 channels with bf16 weights: sum_q w_q * corner_q as mixed-precision FMAs
+// (exact bf16 x bf16 products accumulated in fp32, FHFMA.BF16 -- the corners are used as
+// stored, no unpack), RNE to bf16, into the two 16-byte swizzled slots of this thread's part
+// of the A row.  Reading R20: the only rounding beyond the fp32 lerp is the weights' to bf16.
+__device__ __forceinline__ void lerp_store_row_b(const RowLoadB& L, uint32_t dst_lo, uint32_t dst_hi) {
+    float acc[16];
+    const uint32_t w01 = L.w.x, w23 = L.w.y;
+#pragma unroll
+    for (int h = 0; h < 8; ++h) {
+        acc[2 * h] = fma_bf16h<0, 0>(L.v[0].w[h], w01, 0.f);
+        acc[2 * h + 1] = fma_bf16h<1, 0>(L.v[0].w[h], w01, 0.f);
+    }
+#pragma unroll
+    for (int h = 0; h < 8; ++h) {
+        acc[2 * h] = fma_bf16h<0, 1>(L.v[1].w[h], w01, acc[2 * h]);
+        acc[2 * h + 1] = fma_bf16h<1, 1>(L.v[1].w[h], w01, acc[2 * h + 1]);
+    }
+#pragma unroll
+    for (int h = 0; h < 8; ++h) {
+        acc[2 * h] = fma_bf16h<0, 0>(L.v[2].w[h], w23, acc[2 * h]);
+        acc[2 * h + 1] = fma_bf16h<1, 0>(L.v[2].w[h], w23, acc[2 * h + 1]);
+    }
+#pragma unroll
+    for (int h = 0; h < 8; ++h) {
+        acc[2 * h] = fma_bf16h<0, 1>(L.v[3].w[h], w23, acc[2 * h]);
+        acc[2 * h + 1] = fma_bf16h<1, 1>(L.v[3].w[h], w23, acc[2 * h + 1]);
+    }
+    st_shared_v4(dst_lo, pack_bf16x2(acc[0], acc[1]), pack_bf16x2(acc[2], acc[3]), pack_bf16x2(acc[4], acc[5]),
+                 pack_bf16x2(acc[6], acc[7]));
+    st_shared_v4(dst_hi, pack_bf16x2(acc[8], acc[9]), pack_bf16x2(acc[10], acc[11]),
+                 pack_bf16x2(acc[12], acc[13]), pack_bf16x2(acc[14], acc[15]));
+}
 
 __device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr) {
     const uint4 o = ld_shared_v4(meta_addr);
@@ -385,6 +441,16 @@ template <bool TEX>
 struct Sampler;
 template <>
 struct Sampler<false> {
+#if DEFCON_BF16_WEIGHTS
+    using Load = RowLoadB;
+    static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
+                                                 uint32_t meta) {
+        issue_row_b(L, xb, meta);
+    }
+    static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
+        lerp_store_row_b(L, lo, hi);
+    }
+#else
     using Load = RowLoad;
     static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
                                                  uint32_t meta) {
@@ -393,6 +459,7 @@ struct Sampler<false> {
     static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
         lerp_store_row(L, lo, hi);
     }
+#endif
 };
 template <>
 struct Sampler<true> {
@@ -786,6 +853,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
 #pragma unroll
         for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
             Smp::store(L[p], stage + dst_lo[p], stage + dst_hi[p]);
+            if (t == 0) KT(8 + p, q);
             if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
         }
 #ifdef DEFCON_PROBE_NO_FENCE   // dev probe (WRONG results): no proxy fence, relaxed arrive -- the
@@ -795,6 +863,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
             asm volatile("mbarrier.arrive.relaxed.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&full_a[s])) : "memory");
 #else
         fence_proxy_async_smem();
+        if (t == 0) KT(10, q);
         __syncwarp();
         if (lane == 0) {
             if (PAIR) mbar_arrive_cluster(&full_a[s], 0);   // the pair's MMA issuer is rank 0
@@ -1059,6 +1128,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     if (PAIR) mma_commit_pair(&empty[s], 0x3);
                     else mma_commit(&empty[s]);
                     KT(6, q);
+#ifdef DEFCON_PROBE_MMA_SERIAL   // dev probe: wait for this k-iteration's MMAs to complete (serialises)
+                    mbar_wait_spin(&empty[s], ph);
+                    KT(11, q);
+#endif
                 }
                 if (PAIR) mma_commit_pair(&tmem_full[buf], 0x3);
                 else mma_commit(&tmem_full[buf]);
