@@ -47,10 +47,14 @@ struct Elem {
     static constexpr int PLANES = F32 ? 2 : 1;       // operand planes (tf32 hi / lo)
     static constexpr int A_STAGE = A_PLANE * PLANES;
 };
-constexpr int META_ENTRY = 32;   // int4 corner offsets + float4 weights (bf16 x: 2 bf16 pairs)
-#ifndef DEFCON_BF16_WEIGHTS
-#define DEFCON_BF16_WEIGHTS 1        // bf16 x: bf16 corner weights, FHFMA.BF16 lerp (R20)
-#endif
+// Per-(row, tap) sampling metadata entry.  bf16 x: 16 bytes {byte offset of the top-left
+// corner | 1 when the right-hand corners are a pixel further, byte offset of the bottom-left
+// corner, bf16 weights (w0, w1), (w2, w3)} (invalid corners alias a valid in-bounds one and have
+// weight 0); texture rows: float4 {u, v, mask, -}; fp32 x: 32 bytes {4 corner offsets, 4 fp32
+// weights}.
+template <bool F32>
+__host__ __device__ constexpr int meta_entry() { return F32 ? 32 : 16; }
+constexpr int META_ENTRY = 32;   // the largest entry (shape-support checks)
 #ifndef DEFCON_NPW
 #define DEFCON_NPW 8
 #endif
@@ -66,7 +70,8 @@ constexpr int ROWS = BM * TPR / NPT; // A rows per producer thread
 constexpr int RPW = 32 / TPR;        // rows per warp per pass
 
 #ifdef DEFCON_PROBE_KTRACE   // dev probe: per-k-iteration event clock64 stamps of CTA `KTRACE_CTA`
-__device__ long long g_kt[12][64];
+__device__ long long g_kt[24][64];
+__device__ int g_kt_q;
 #ifndef KTRACE_CTA
 #define KTRACE_CTA 5
 #endif
@@ -110,6 +115,7 @@ struct TcArgs {
     unsigned long long tex;          // DEFCON_SAMPLER_TEX: stacked-image texture object, else 0
     int bias_in_smem;      // Cout <= BIAS_SMEM_MAX: bias (or zeros) staged in shared memory
     int pair;              // 1: CTA pairs (cta_group::2, M = 256 per MMA), tiles of 2 x BM rows
+    int stage_meta;        // 1: the next metadata table's offsets / mask are cp.async-staged in smem
 };
 
 constexpr int BIAS_SMEM_MAX = 1024;
@@ -192,8 +198,16 @@ __device__ __forceinline__ RowPos row_pos(const TcArgs& a, int m) {
     return p;
 }
 
-__device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& rp, int i, int j, const MetaIn& in,
-                                                 uint8_t* e, bool tex_row) {
+// One metadata entry (see meta_entry) for tap (i, j) of row rp, computed without branches so
+// that a thread's entries are independent dependency chains the scheduler can interleave.
+// Corners outside the image get weight 0 and an in-bounds address (R8).
+struct MetaVal {
+    uint4 lo, hi;   // hi: fp32 weights of the 32-byte format
+};
+
+template <bool COMPACT>
+__device__ __forceinline__ MetaVal meta_value(const TcArgs& a, const RowPos& rp, int i, int j, const MetaIn& in,
+                                              bool tex_row) {
     float2 d = in.d;
     if (a.bound_h >= 0.f) {   // bounded deformation (R12)
         const int Kh = a.KK / a.Kw;
@@ -201,99 +215,168 @@ __device__ __forceinline__ void store_meta_entry(const TcArgs& a, const RowPos& 
         d.y = bound_offset(d.y, (j - 0.5f * (a.Kw - 1)) * a.dw, a.bound_h);
     }
     const float mk = in.mk;
+    const float py0 = (float)(rp.yb + i * a.dh) + d.x;
+    const float px0 = (float)(rp.xb + j * a.dw) + d.y;
+    const bool fin = rp.ok && py0 == py0 && px0 == px0;
+    MetaVal r;
     if (tex_row) {
         // texture sampler: unnormalised texel coordinates (texel centres at +0.5, R7) in the
         // stacked-image texture (image n occupies rows n*(H+1) .. n*(H+1)+H-1, row
         // n*(H+1)+H is zero) and the mask.  Clamping to [-1, H] x [-1, W] keeps samples
         // beyond the image on zero texels.
-        float4 c = make_float4(-4.f, -4.f, 0.f, 0.f);
-        if (rp.ok) {
-            const float py = (float)(rp.yb + i * a.dh) + d.x;
-            const float px = (float)(rp.xb + j * a.dw) + d.y;
-            if (px == px && py == py) {
-                c.x = fminf(fmaxf(px, -1.0f), (float)a.W) + 0.5f;
-                c.y = (float)(rp.n * (a.H + 1)) + fminf(fmaxf(py, -1.0f), (float)a.H) + 0.5f;
-                c.z = mk;
+        const float u = fminf(fmaxf(px0, -1.0f), (float)a.W) + 0.5f;
+        const float v = (float)(rp.n * (a.H + 1)) + fminf(fmaxf(py0, -1.0f), (float)a.H) + 0.5f;
+        r.lo = make_uint4(__float_as_uint(fin ? u : -4.f), __float_as_uint(fin ? v : -4.f),
+                          __float_as_uint(fin ? mk : 0.f), 0u);
+        r.hi = make_uint4(0u, 0u, 0u, 0u);
+        return r;
+    }
+    // Anything beyond one pixel outside samples only zeros; clamping keeps the int conversion
+    // defined for huge offsets (non-finite ones are mapped to a fully outside point).
+    const float py = fin ? fminf(fmaxf(py0, -2.0f), (float)a.H + 1.0f) : -2.0f;
+    const float px = fin ? fminf(fmaxf(px0, -2.0f), (float)a.W + 1.0f) : -2.0f;
+    const int y0 = __float2int_rd(py), x0 = __float2int_rd(px);
+    const float ly = py - (float)y0, lx = px - (float)x0;
+    const bool vy0 = (unsigned)y0 < (unsigned)a.H, vy1 = (unsigned)(y0 + 1) < (unsigned)a.H;
+    const bool vx0 = (unsigned)x0 < (unsigned)a.W, vx1 = (unsigned)(x0 + 1) < (unsigned)a.W;
+    const float w0 = (vy0 && vx0) ? (1.f - ly) * (1.f - lx) * mk : 0.f;
+    const float w1 = (vy0 && vx1) ? (1.f - ly) * lx * mk : 0.f;
+    const float w2 = (vy1 && vx0) ? ly * (1.f - lx) * mk : 0.f;
+    const float w3 = (vy1 && vx1) ? ly * lx * mk : 0.f;
+    const uint32_t base = (uint32_t)(rp.n * a.H);
+    const uint32_t pb = (uint32_t)(a.Cin * a.es);   // bytes per pixel
+    const uint32_t rowb = (uint32_t)a.W * pb;
+    if constexpr (COMPACT) {   // one valid column / row stands in for an invalid one (weight 0)
+        const int ya = vy0 ? y0 : (vy1 ? y0 + 1 : 0);
+        const int xa = vx0 ? x0 : (vx1 ? x0 + 1 : 0);
+        const uint32_t o = (base + (uint32_t)ya) * rowb + (uint32_t)xa * pb;
+        r.lo = make_uint4(o | ((vx0 && vx1) ? 1u : 0u), (vy0 && vy1) ? o + rowb : o, pack_bf16x2(w0, w1),
+                          pack_bf16x2(w2, w3));
+        r.hi = make_uint4(0u, 0u, 0u, 0u);
+    } else {
+        const uint32_t o00 = (base + (uint32_t)y0) * rowb + (uint32_t)x0 * pb;
+        r.lo = make_uint4((vy0 && vx0) ? o00 : 0u, (vy0 && vx1) ? o00 + pb : 0u, (vy1 && vx0) ? o00 + rowb : 0u,
+                          (vy1 && vx1) ? o00 + rowb + pb : 0u);
+        r.hi = make_uint4(__float_as_uint(w0), __float_as_uint(w1), __float_as_uint(w2), __float_as_uint(w3));
+    }
+    return r;
+}
+
+// Staging of the next table's inputs: every producer thread cp.async-copies the offsets / mask
+// of exactly the (row, tap) entries it will build (row t / TPM, taps t % TPM + TPM k) into its
+// own 64-byte slot -- 5 offset pairs at +0, 5 masks at +40 -- while the current table is in use,
+// so a table build reads shared memory instead of waiting on two L2 / DRAM round trips.
+constexpr int STG_TAPS = 5;
+constexpr int STG_BYTES = 64;
+
+__device__ __forceinline__ void cp_async_4(uint32_t dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_8(uint32_t dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src) : "memory");
+}
+
+// Issue the copies for table (m0, g) (m0 < 0: none).  One commit group per table.
+__device__ __forceinline__ void stage_meta_inputs(const TcArgs& a, int m0, int g, uint32_t stg, int t) {
+    const int TPMl = NPT / BM;
+    const int m = m0 + t / TPMl;
+    if (m0 >= 0 && m < a.M) {
+        const long pix = (long)m * a.G + g;
+#pragma unroll
+        for (int k = 0; k < STG_TAPS; ++k) {
+            const int tk = t % TPMl + TPMl * k;
+            if (tk < a.KK) {
+                const long i = pix * a.KK + tk;
+                if (a.off_f16) {
+                    cp_async_4(stg + 8 * k, reinterpret_cast<const uint16_t*>(a.offset) + 2 * i);
+                    if (a.mask) cp_async_4(stg + 40 + 4 * k, reinterpret_cast<const uint16_t*>(a.mask) + (i & ~1l));
+                } else {
+                    cp_async_8(stg + 8 * k, a.offset + 2 * i);
+                    if (a.mask) cp_async_4(stg + 40 + 4 * k, a.mask + i);
+                }
             }
         }
-        *reinterpret_cast<float4*>(e) = c;
-        return;
     }
-    uint4 off = make_uint4(0u, 0u, 0u, 0u);
-    float4 wt = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (rp.ok) {
-        float py = (float)(rp.yb + i * a.dh) + d.x;
-        float px = (float)(rp.xb + j * a.dw) + d.y;
-        // Anything beyond one pixel outside samples only zeros; clamping keeps the
-        // int conversion defined for huge / non-finite offsets.
-        py = fminf(fmaxf(py, -2.0f), (float)a.H + 1.0f);
-        px = fminf(fmaxf(px, -2.0f), (float)a.W + 1.0f);
-        if (py == py && px == px) {
-            const float fy = floorf(py), fx = floorf(px);
-            const float ly = py - fy, lx = px - fx;
-            const int y0 = (int)fy, x0 = (int)fx;
-            const bool vy0 = (y0 >= 0) && (y0 < a.H), vy1 = (y0 + 1 >= 0) && (y0 + 1 < a.H);
-            const bool vx0 = (x0 >= 0) && (x0 < a.W), vx1 = (x0 + 1 >= 0) && (x0 + 1 < a.W);
-            const uint32_t base = (uint32_t)(rp.n * a.H);
-            const uint32_t rowb = (uint32_t)(a.Cin * a.es);   // bytes per pixel
-            if (vy0 && vx0) { off.x = ((base + y0) * a.W + x0) * rowb;         wt.x = (1.f - ly) * (1.f - lx) * mk; }
-            if (vy0 && vx1) { off.y = ((base + y0) * a.W + x0 + 1) * rowb;     wt.y = (1.f - ly) * lx * mk; }
-            if (vy1 && vx0) { off.z = ((base + y0 + 1) * a.W + x0) * rowb;     wt.z = ly * (1.f - lx) * mk; }
-            if (vy1 && vx1) { off.w = ((base + y0 + 1) * a.W + x0 + 1) * rowb; wt.w = ly * lx * mk; }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+__device__ __forceinline__ MetaIn staged_input(const TcArgs& a, uint32_t stg, int k, long i) {
+    MetaIn in;
+    if (a.off_f16) {
+        const uint32_t w = ld_shared_u32(stg + 8 * k);
+        in.d = make_float2(__half2float(__ushort_as_half((unsigned short)(w & 0xFFFFu))),
+                           __half2float(__ushort_as_half((unsigned short)(w >> 16))));
+        if (a.mask) {
+            const uint32_t mw = ld_shared_u32(stg + 40 + 4 * k);
+            in.mk = __half2float(__ushort_as_half((unsigned short)((i & 1) ? (mw >> 16) : (mw & 0xFFFFu))));
+        } else {
+            in.mk = 1.0f;
         }
+    } else {
+        const uint2 w = make_uint2(ld_shared_u32(stg + 8 * k), ld_shared_u32(stg + 8 * k + 4));
+        in.d = make_float2(__uint_as_float(w.x), __uint_as_float(w.y));
+        in.mk = a.mask ? __uint_as_float(ld_shared_u32(stg + 40 + 4 * k)) : 1.0f;
     }
-    *reinterpret_cast<uint4*>(e) = off;
-#if DEFCON_BF16_WEIGHTS
-    if (a.es == 2) {   // bf16 x: the 4 weights as bf16 pairs, consumed by FHFMA.BF16 (lerp_store_row)
-        *reinterpret_cast<uint2*>(e + 16) = make_uint2(pack_bf16x2(wt.x, wt.y), pack_bf16x2(wt.z, wt.w));
-        return;
-    }
-#endif
-    *reinterpret_cast<float4*>(e + 16) = wt;
+    return in;
 }
 
 // The whole (tile, group) table, built by the NPT = TPM * BM producer threads: thread t owns
-// row t / TPM and taps t % TPM, + TPM, ...  The row's pixel decomposition is done once; the
-// offset/mask loads of a pass are all issued before any arithmetic (one round trip per
-// pass).  Rows of warp w use the format of that warp's sampler.
+// row t / TPM and taps t % TPM, + TPM, ... in rounds of STG_TAPS entries: all inputs of a round
+// are fetched (shared-memory staging or global loads) before any arithmetic, and the entries
+// are computed as independent chains before any is stored.  Rows of warp w use the format of
+// that warp's sampler.
 constexpr int TPM = NPT / BM;    // producer threads per tile row in the metadata build
 static_assert(NPT % BM == 0, "metadata build assumes whole producer threads per tile row");
-#ifndef DEFCON_META_PASS
-#define DEFCON_META_PASS 3
-#endif
-template <int NTEX>
-__device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t) {
-    constexpr int PASS = DEFCON_META_PASS;   // taps in flight per thread (register budget)
+template <int NTEX, int ME>
+__device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t,
+                                                 uint32_t stg = 0u) {
     const int row = t / TPM;
     const RowPos rp = row_pos(a, m0 + row);
     const bool tex_row = ((row % (NPW * RPW)) / RPW) < NTEX;
     const long pix = (long)(m0 + row) * a.G + g;
-    uint8_t* rmeta = meta + row * a.KK * META_ENTRY;
-    int tap = t % TPM;
-    int i = tap / a.Kw, j = tap - (tap / a.Kw) * a.Kw;
+    uint8_t* rmeta = meta + row * a.KK * ME;
+    if (t == 0) KT(16, g_kt_q);
+    if (stg) asm volatile("cp.async.wait_all;" ::: "memory");   // this thread's staged copies
+    if (t == 0) KT(17, g_kt_q);
+    const long ibase = pix * a.KK;
+    int i0 = (t % TPM) / a.Kw, j0 = (t % TPM) - ((t % TPM) / a.Kw) * a.Kw;
 #pragma unroll 1
-    for (; tap < a.KK;) {
-        MetaIn in[PASS];
+    for (int tb = t % TPM; tb < a.KK; tb += TPM * STG_TAPS) {
+        // inputs: every load unconditional (tap index clamped, rows past M read row 0's
+        // pixel), validity applied afterwards -- no branches between the independent entries
+        MetaIn in[STG_TAPS];
 #pragma unroll
-        for (int k = 0; k < PASS; ++k) {
-            const int tk = tap + TPM * k;
-            in[k].d = make_float2(0.f, 0.f);
-            in[k].mk = 0.f;
-            if (rp.ok && tk < a.KK) {
-                in[k].d = ld_offset2(a.offset, (pix * a.KK + tk) * 2, a.off_f16);
-                in[k].mk = a.mask ? ld_mask1(a.mask, pix * a.KK + tk, a.off_f16) : 1.0f;
+        for (int k = 0; k < STG_TAPS; ++k) {
+            const int tk = min(tb + TPM * k, a.KK - 1);
+            if (stg) {   // staged (only when every tap fits one round)
+                in[k] = staged_input(a, stg, k, ibase + tk);
+            } else {
+                in[k].d = ld_offset2(a.offset, (ibase + tk) * 2, a.off_f16);
+                in[k].mk = a.mask ? ld_mask1(a.mask, ibase + tk, a.off_f16) : 1.0f;
             }
         }
-#ifdef DEFCON_PROBE_TL_META
-        if (t == 0) TL(tap < 2 ? 6 : 7);
-#endif
+        MetaVal v[STG_TAPS];
+        int i = i0, j = j0;
 #pragma unroll
-        for (int k = 0; k < PASS; ++k) {
-            if (tap < a.KK) store_meta_entry(a, rp, i, j, in[k], rmeta + tap * META_ENTRY, tex_row);
-            tap += TPM;
+        for (int k = 0; k < STG_TAPS; ++k) {
+            v[k] = meta_value<ME == 16>(a, rp, i, j, in[k], tex_row);
             j += TPM;
-            while (j >= a.Kw) { j -= a.Kw; ++i; }
+            while (j >= a.Kw) {   // once per step for Kw >= TPM
+                j -= a.Kw;
+                ++i;
+            }
         }
+        i0 = i;
+        j0 = j;
+#pragma unroll
+        for (int k = 0; k < STG_TAPS; ++k) {
+            const int tk = tb + TPM * k;
+            if (tk < a.KK) {
+                *reinterpret_cast<uint4*>(rmeta + tk * ME) = v[k].lo;
+                if (ME == 32 && !tex_row) *reinterpret_cast<uint4*>(rmeta + tk * ME + 16) = v[k].hi;
+            }
+        }
+        if (t == 0) KT(18, g_kt_q);
     }
 }
 
@@ -324,13 +407,25 @@ struct RowLoadB {
     uint2 w;
 };
 
-__device__ __forceinline__ void issue_row_b(RowLoadB& L, const void* xbase, uint32_t meta_addr) {
-    const uint4 o = ld_shared_v4(meta_addr);
-    L.w = ld_shared_v2(meta_addr + 16);
-    L.v[0] = ldg_nc_v8(add_u32(xbase, o.x));
-    L.v[1] = ldg_nc_v8(add_u32(xbase, o.y));
-    L.v[2] = ldg_nc_v8(add_u32(xbase, o.z));
-    L.v[3] = ldg_nc_v8(add_u32(xbase, o.w));
+// One 16-byte compact entry (store_meta_entry): corners 1 / 3 are corners 0 / 2 plus one pixel
+// (pb bytes) when the entry's flag bit is set, else the same (weight-0) address.
+__device__ __forceinline__ void issue_row_b(RowLoadB& L, const void* xbase, uint32_t meta_addr, uint32_t pb) {
+    const uint4 e = ld_shared_v4(meta_addr);
+    L.w = make_uint2(e.z, e.w);
+    const uint32_t dx = (e.x & 1u) * pb;
+    const uint32_t o0 = e.x & ~1u;
+#ifdef DEFCON_PROBE_SAME_ADDR   // dev probe: every gather hits the same line (L1-resident)
+    L.v[0] = ldg_nc_v8(xbase);
+    L.v[1] = ldg_nc_v8(xbase);
+    L.v[2] = ldg_nc_v8(xbase);
+    L.v[3] = ldg_nc_v8(xbase);
+    (void)dx; (void)o0;
+#else
+    L.v[0] = ldg_nc_v8(add_u32(xbase, o0));
+    L.v[1] = ldg_nc_v8(add_u32(xbase, o0 + dx));
+    L.v[2] = ldg_nc_v8(add_u32(xbase, e.y));
+    L.v[3] = ldg_nc_v8(add_u32(xbase, e.y + dx));
+#endif
 }
 
 // Eq.3 for 16 bf16 channels with bf16 weights: sum_q w_q * corner_q as mixed-precision FMAs
@@ -338,6 +433,14 @@ __device__ __forceinline__ void issue_row_b(RowLoadB& L, const void* xbase, uint
 // stored, no unpack), RNE to bf16, into the two 16-byte swizzled slots of this thread's part
 // of the A row.  Reading R20: the only rounding beyond the fp32 lerp is the weights' to bf16.
 __device__ __forceinline__ void lerp_store_row_b(const RowLoadB& L, uint32_t dst_lo, uint32_t dst_hi) {
+#ifdef DEFCON_PROBE_NO_MATH   // dev probe: no lerp, the 4 corners xor-ed (keeps every load live)
+    uint32_t o[8];
+#pragma unroll
+    for (int h = 0; h < 8; ++h) o[h] = L.v[0].w[h] ^ L.v[1].w[h] ^ L.v[2].w[h] ^ L.v[3].w[h] ^ L.w.x;
+    st_shared_v4(dst_lo, o[0], o[1], o[2], o[3]);
+    st_shared_v4(dst_hi, o[4], o[5], o[6], o[7]);
+    return;
+#endif
     float acc[16];
     const uint32_t w01 = L.w.x, w23 = L.w.y;
 #pragma unroll
@@ -366,50 +469,16 @@ __device__ __forceinline__ void lerp_store_row_b(const RowLoadB& L, uint32_t dst
                  pack_bf16x2(acc[12], acc[13]), pack_bf16x2(acc[14], acc[15]));
 }
 
+// fp32 x: the 4 corner vectors and fp32 weights of one 32-byte entry.
 __device__ __forceinline__ void issue_row(RowLoad& L, const void* xbase, uint32_t meta_addr) {
     const uint4 o = ld_shared_v4(meta_addr);
     const uint4 wb = ld_shared_v4(meta_addr + 16);
     L.w = make_float4(__uint_as_float(wb.x), __uint_as_float(wb.y), __uint_as_float(wb.z),
                       __uint_as_float(wb.w));
-#ifdef DEFCON_PROBE_SAME_ADDR   // dev probe: every gather hits the same line (L1-resident)
-    L.v[0] = ldg_nc_v8(add_u32(xbase, o.x & 0u));
-    L.v[1] = ldg_nc_v8(add_u32(xbase, o.y & 0u));
-    L.v[2] = ldg_nc_v8(add_u32(xbase, o.z & 0u));
-    L.v[3] = ldg_nc_v8(add_u32(xbase, o.w & 0u));
-#else
     L.v[0] = ldg_nc_v8(add_u32(xbase, o.x));
     L.v[1] = ldg_nc_v8(add_u32(xbase, o.y));
     L.v[2] = ldg_nc_v8(add_u32(xbase, o.z));
     L.v[3] = ldg_nc_v8(add_u32(xbase, o.w));
-#endif
-}
-
-// Eq.3 for 16 channels: sum_q w_q * corner_q, fp32 (packed FFMA2), RNE to bf16, into the
-// two 16-byte swizzled slots of this thread's part of the A row.
-__device__ __forceinline__ void lerp_store_row(const RowLoad& L, uint32_t dst_lo, uint32_t dst_hi) {
-#ifdef DEFCON_PROBE_NO_MATH   // dev probe: no lerp, the 4 corners xor-ed (keeps every load live)
-    uint32_t o[8];
-#pragma unroll
-    for (int h = 0; h < 8; ++h) o[h] = L.v[0].w[h] ^ L.v[1].w[h] ^ L.v[2].w[h] ^ L.v[3].w[h] ^ __float_as_uint(L.w.x);
-    st_shared_v4(dst_lo, o[0], o[1], o[2], o[3]);
-    st_shared_v4(dst_hi, o[4], o[5], o[6], o[7]);
-    return;
-#endif
-    uint64_t acc[8];
-    const float wq[4] = {L.w.x, L.w.y, L.w.z, L.w.w};
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const uint64_t w2 = f32x2_pack(wq[q], wq[q]);
-#pragma unroll
-        for (int h = 0; h < 8; ++h) {
-            const uint64_t c = bf16x2_to_f32x2(L.v[q].w[h]);
-            acc[h] = q == 0 ? f32x2_mul(c, w2) : f32x2_fma(c, w2, acc[h]);
-        }
-    }
-    st_shared_v4(dst_lo, f32x2_to_bf16x2(acc[0]), f32x2_to_bf16x2(acc[1]), f32x2_to_bf16x2(acc[2]),
-                 f32x2_to_bf16x2(acc[3]));
-    st_shared_v4(dst_hi, f32x2_to_bf16x2(acc[4]), f32x2_to_bf16x2(acc[5]), f32x2_to_bf16x2(acc[6]),
-                 f32x2_to_bf16x2(acc[7]));
 }
 
 // Texture-sampler counterpart of RowLoad: 16 channels = 4 texels of 4 channels, already
@@ -441,31 +510,20 @@ template <bool TEX>
 struct Sampler;
 template <>
 struct Sampler<false> {
-#if DEFCON_BF16_WEIGHTS
     using Load = RowLoadB;
     static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
-                                                 uint32_t meta) {
-        issue_row_b(L, xb, meta);
+                                                 uint32_t meta, uint32_t pb) {
+        issue_row_b(L, xb, meta, pb);
     }
     static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
         lerp_store_row_b(L, lo, hi);
     }
-#else
-    using Load = RowLoad;
-    static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
-                                                 uint32_t meta) {
-        issue_row(L, xb, meta);
-    }
-    static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
-        lerp_store_row(L, lo, hi);
-    }
-#endif
 };
 template <>
 struct Sampler<true> {
     using Load = TexLoad;
     static __device__ __forceinline__ void issue(Load& L, const uint8_t*, unsigned long long tex, int layer,
-                                                 uint32_t meta) {
+                                                 uint32_t meta, uint32_t) {
         issue_row_tex(L, (cudaTextureObject_t)tex, layer, meta);
     }
     static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
@@ -507,7 +565,7 @@ __device__ __forceinline__ void lerp_store_row_f32(const RowLoad& L, uint32_t d0
 struct SamplerF32 {
     using Load = RowLoad;
     static __device__ __forceinline__ void issue(Load& L, const uint8_t* xb, unsigned long long, int,
-                                                 uint32_t meta) {
+                                                 uint32_t meta, uint32_t) {
         issue_row(L, xb, meta);
     }
     static __device__ __forceinline__ void store(const Load& L, uint32_t lo, uint32_t hi) {
@@ -814,19 +872,42 @@ template <bool TEXW, int STAGES, int NTEX, bool PAIR, bool F32>
 __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
                                                 const uint32_t (&dst_lo)[ROWS], const uint32_t (&dst_hi)[ROWS],
                                                 const uint32_t (&mrow)[ROWS], uint32_t a_s, uint64_t* empty,
-                                                uint64_t* full_a, int t, int sub, int lane, int next_m0) {
+                                                uint64_t* full_a, int t, int sub, int lane, int next_m0,
+                                                int next_g, uint32_t stg, int& staged_m0, int& staged_g) {
     using Smp = typename std::conditional<F32, SamplerF32, Sampler<TEXW>>::type;
     using E = Elem<F32>;
+    constexpr int ME = meta_entry<F32>();
+    const uint32_t pb = (uint32_t)(a.Cin * a.es);   // bytes per x pixel
     const int m0 = tile_m0<PAIR>(a, sg.tile);
     int chunk = sg.kb / a.KK;
     int tap = sg.kb - chunk * a.KK;
     int g = (chunk * E::CPI) / a.Cg;
+    const int g_last = (((sg.ke - 1) / a.KK) * E::CPI) / a.Cg;   // the segment's last offset group
+    // The table after (m0, gc): the segment's next group, else the next segment's first.
+    auto stage_after = [&](int gc) {
+        if (!stg) return;
+        staged_m0 = gc < g_last ? m0 : next_m0;
+        staged_g = gc < g_last ? gc + 1 : next_g;
+        stage_meta_inputs(a, staged_m0, staged_g, stg, t);
+    };
+#ifdef DEFCON_PROBE_KTRACE
+    if (t == 0) g_kt_q = q;
+#endif
+    if (t == 0) KT(12, q);
     named_bar_sync(1, NPT);          // previous table no longer read
 #ifdef DEFCON_PROBE_TL_META
     if (t == 0) TL(9);
 #endif
-    build_meta_table<NTEX>(a, m0, g, meta, t);
+    if (t == 0) KT(13, q);
+#ifdef DEFCON_PROBE_BUILD_TWICE   // dev probe: a second, warm build of the same table
+    build_meta_table<NTEX, ME>(a, m0, g, meta, t, 0u);
+    if (t == 0) KT(23, q);
+#endif
+    build_meta_table<NTEX, ME>(a, m0, g, meta, t, (stg && staged_m0 == m0 && staged_g == g) ? stg : 0u);
+    stage_after(g);
+    if (t == 0) KT(14, q);
     named_bar_sync(1, NPT);
+    if (t == 0) KT(15, q);
     prefetch_meta_l2(a, next_m0, t);
     if (t == 0) TL(10 + (q ? 1 : 0));     // metadata table ready (first / later segment)
     // position of this thread's 16 channels: byte pointer (LDG) / texture layer (TEX)
@@ -834,7 +915,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     int layer = chunk * (BK / 4) + sub * 4;
     typename Smp::Load L[ROWS];
 #pragma unroll
-    for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], xb, a.tex, layer, mrow[p] + tap * META_ENTRY);
+    for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], xb, a.tex, layer, mrow[p] + tap * ME, pb);
     for (int kt = sg.kb; kt < sg.ke; ++kt, ++q) {
         int ntap = tap + 1, nchunk = chunk;
         if (ntap == a.KK) { ntap = 0; ++nchunk; }
@@ -854,7 +935,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
             Smp::store(L[p], stage + dst_lo[p], stage + dst_hi[p]);
             if (t == 0) KT(8 + p, q);
-            if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
+            if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * ME, pb);
         }
 #ifdef DEFCON_PROBE_NO_FENCE   // dev probe (WRONG results): no proxy fence, relaxed arrive -- the
                                // cost of ordering the A stores before the MMA
@@ -876,12 +957,13 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         if (has_next && !prefetch) {          // offset group changes: new table
 #ifndef DEFCON_PROBE_NO_REBUILD   // dev probe (WRONG results for G > 1): keep the first table
             named_bar_sync(1, NPT);
-            build_meta_table<NTEX>(a, m0, ng, meta, t);
+            build_meta_table<NTEX, ME>(a, m0, ng, meta, t, (stg && staged_m0 == m0 && staged_g == ng) ? stg : 0u);
+            stage_after(ng);
             named_bar_sync(1, NPT);
 #endif
             g = ng;
 #pragma unroll
-            for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * META_ENTRY);
+            for (int p = 0; p < ROWS; ++p) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * ME, pb);
         }
         layer = nlayer;
         tap = ntap;
@@ -906,7 +988,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     uint8_t* sB = smem + STAGES * Cfg::A_STAGE_BYTES;
     uint8_t* epi_scratch = sB + STAGES * Cfg::B_STAGE_BYTES;   // 4 epilogue warps x EPI_W
     uint8_t* meta = epi_scratch + 4 * EPI_W;
-    uint64_t* bars = reinterpret_cast<uint64_t*>(meta + BM * a.KK * META_ENTRY);
+    uint8_t* stg_area = meta + BM * a.KK * meta_entry<F32>();   // NPT x STG_BYTES when a.stage_meta
+    uint64_t* bars = reinterpret_cast<uint64_t*>(stg_area + (a.stage_meta ? NPT * STG_BYTES : 0));
     uint64_t* full_a = bars;
     uint64_t* full_b = bars + STAGES;
     uint64_t* empty = bars + 2 * STAGES;
@@ -973,20 +1056,35 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const int row = (t / TPR) + p * (NPT / TPR);
             dst_lo[p] = row * 128 + (((2 * sub) ^ (row & 7)) << 4);
             dst_hi[p] = row * 128 + (((2 * sub + 1) ^ (row & 7)) << 4);
-            mrow[p] = meta_s + row * a.KK * META_ENTRY;
+            mrow[p] = meta_s + row * a.KK * meta_entry<F32>();
         }
         int q = 0;                           // running k-iteration (stage) counter
+        const uint32_t stg = a.stage_meta ? smem_u32(stg_area) + t * STG_BYTES : 0u;
+        auto seg_group = [&](const Segment& sx) { return ((sx.kb / a.KK) * Elem<F32>::CPI) / a.Cg; };
+        int staged_m0 = -1, staged_g = -1;   // the table whose inputs sit in this thread's staging slot
+        if (stg && nseg > 0) {               // the first table: one round trip
+            const Segment s0 = segment_j(a, it_begin, it_end, seg_order(0, nseg));
+            staged_m0 = tile_m0<PAIR>(a, s0.tile);
+            staged_g = seg_group(s0);
+            stage_meta_inputs(a, staged_m0, staged_g, stg, t);
+        }
         for (int o = 0; o < nseg; ++o) {
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
-            const int next_m0 = o + 1 < nseg
-                ? tile_m0<PAIR>(a, segment_j(a, it_begin, it_end, seg_order(o + 1, nseg)).tile) : -1;
+            int next_m0 = -1, next_g = 0;
+            if (o + 1 < nseg) {
+                const Segment sn = segment_j(a, it_begin, it_end, seg_order(o + 1, nseg));
+                next_m0 = tile_m0<PAIR>(a, sn.tile);
+                next_g = seg_group(sn);
+            }
             if (t == 0 && o < 4) TL(2 + 2 * o);
             if (warp < NTEX)
                 produce_segment<true, STAGES, NTEX, PAIR, F32>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty,
-                                                               full_a, t, sub, lane, next_m0);
+                                                               full_a, t, sub, lane, next_m0, next_g, stg,
+                                                               staged_m0, staged_g);
             else
                 produce_segment<false, STAGES, NTEX, PAIR, F32>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty,
-                                                                full_a, t, sub, lane, next_m0);
+                                                                full_a, t, sub, lane, next_m0, next_g, stg,
+                                                                staged_m0, staged_g);
             if (t == 0 && o < 4) TL(3 + 2 * o);
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
@@ -1299,8 +1397,8 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     if (PAIR && g_pair_units == 0) {   // how many pairs fit at once (one CTA per SM)
         auto kp = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>;
         const size_t smem_q = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
-                              (size_t)BM * g.KK * META_ENTRY + bias_smem_offset(STAGES, Cfg::NBUF) +
-                              (size_t)BIAS_SMEM_MAX * 4;
+                              (size_t)BM * g.KK * meta_entry<false>() + (size_t)NPT * STG_BYTES +
+                              bias_smem_offset(STAGES, Cfg::NBUF) + (size_t)BIAS_SMEM_MAX * 4;
         cudaFuncSetAttribute(kp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_q);
         cudaLaunchConfig_t qc = {};
         qc.gridDim = dim3(num_sms());
@@ -1400,9 +1498,15 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
 
     a.bias_in_smem = g.Cout <= BIAS_SMEM_MAX ? 1 : 0;
     a.pair = PAIR ? 1 : 0;
+    // metadata staging (bf16 x, up to 10 taps): NPT x 64 bytes of shared memory
+#ifndef DEFCON_META_STAGE
+#define DEFCON_META_STAGE 0   // measured slower at C3 / C4 / C4 G4 (the 16 KB come out of L1)
+#endif
+    a.stage_meta = (DEFCON_META_STAGE && !F32 && g.KK <= (NPT / BM) * STG_TAPS) ? 1 : 0;
     // Stream-K tile counters are NOT reset here: the workspace is zero-filled once by its
     // owner and every launch leaves it zeroed (the finisher of each split tile resets it).
-    const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_W + (size_t)BM * g.KK * META_ENTRY +
+    const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_W + (size_t)BM * g.KK * meta_entry<F32>() +
+                        (a.stage_meta ? (size_t)NPT * STG_BYTES : 0) +
                         bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0);
     auto kern = F32 ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false, F32>
                 : PAIR ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>

@@ -718,9 +718,11 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
     a.packed = static_cast<const uint8_t*>(ws);
     // PDL launch: its launch overlaps the previous kernel; it waits for that kernel before writing
     // (measured A/B on one box: bench step 75.5 -> 74.8 us, host entry 0.70 -> 0.56 ms)
+#ifndef DEFCON_PROBE_NO_PACK   // dev probe (stale parameters unless packed before): the pack kernel's cost
     cudaError_t e = launch_pdl(op_pack_kernel, dim3(a.nch, (a.OCN * OP_KC + 255) / 256), dim3(256), 0, stream, dw_w,
                                dw_scale, dw_shift, pw_w, C, a.OC, a.OCN, static_cast<uint8_t*>(ws));
     if (e != cudaSuccess) return e;
+#endif
     PFN_encodeTiled encode = get_encode_tiled();
     if (!encode) return cudaErrorNotSupported;
     // x as a 3-D tensor [N*H][W][C] (C innermost); box = 32 channels x IC columns x IR rows

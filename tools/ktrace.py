@@ -21,11 +21,15 @@ name = sys.argv[1] if len(sys.argv) > 1 else "yolact_r101_c4_v2"
 c = configs.SINGLE_LAYER[name]
 lib = d.load_library()
 us, tf = time_cfg(c, "ldg", reps=20)
-buf = np.zeros((12, 64), dtype=np.int64)
+buf = np.zeros((24, 64), dtype=np.int64)
 lib.defcon_debug_ktrace(buf.ctypes.data_as(ctypes.c_void_p))
 n = int((buf[6] > 0).sum())
 b = buf[:, :n] - buf[3, 0]
 print(f"{name}: {us:.2f} us; {n} k-iterations traced (cycles relative to the first MMA wait)")
+for q in range(n):
+    if buf[12, q]:
+        print(f"segment start at q={q}: sync1 {b[12,q]} -> {b[13,q]}, build -> {b[14,q]}, sync2 -> {b[15,q]}; "
+              f"build: enter {b[16,q]} waited {b[17,q]} round done {b[18,q]}; (probe: first build done {b[23,q]})")
 print("MMA serial probe: m:done-m:gotB per q:", [int(b[11,q]-b[5,q]) for q in range(n)] if buf[11].any() else "n/a")
 print("  q   p:emptyW  p:got  row0  row1  fence  p0:arr  pLast:arr  m:waitA  m:gotA  m:gotB  m:commit  | MMA period  A-wait  B-wait")
 for q in range(n):
