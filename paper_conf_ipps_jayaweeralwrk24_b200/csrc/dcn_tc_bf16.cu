@@ -115,7 +115,6 @@ struct TcArgs {
     unsigned long long tex;          // DEFCON_SAMPLER_TEX: stacked-image texture object, else 0
     int bias_in_smem;      // Cout <= BIAS_SMEM_MAX: bias (or zeros) staged in shared memory
     int pair;              // 1: CTA pairs (cta_group::2, M = 256 per MMA), tiles of 2 x BM rows
-    int stage_meta;        // 1: the next metadata table's offsets / mask are cp.async-staged in smem
 };
 
 constexpr int BIAS_SMEM_MAX = 1024;
@@ -262,82 +261,23 @@ __device__ __forceinline__ MetaVal meta_value(const TcArgs& a, const RowPos& rp,
     return r;
 }
 
-// Staging of the next table's inputs: every producer thread cp.async-copies the offsets / mask
-// of exactly the (row, tap) entries it will build (row t / TPM, taps t % TPM + TPM k) into its
-// own 64-byte slot -- 5 offset pairs at +0, 5 masks at +40 -- while the current table is in use,
-// so a table build reads shared memory instead of waiting on two L2 / DRAM round trips.
-constexpr int STG_TAPS = 5;
-constexpr int STG_BYTES = 64;
-
-__device__ __forceinline__ void cp_async_4(uint32_t dst, const void* src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_8(uint32_t dst, const void* src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src) : "memory");
-}
-
-// Issue the copies for table (m0, g) (m0 < 0: none).  One commit group per table.
-__device__ __forceinline__ void stage_meta_inputs(const TcArgs& a, int m0, int g, uint32_t stg, int t) {
-    const int TPMl = NPT / BM;
-    const int m = m0 + t / TPMl;
-    if (m0 >= 0 && m < a.M) {
-        const long pix = (long)m * a.G + g;
-#pragma unroll
-        for (int k = 0; k < STG_TAPS; ++k) {
-            const int tk = t % TPMl + TPMl * k;
-            if (tk < a.KK) {
-                const long i = pix * a.KK + tk;
-                if (a.off_f16) {
-                    cp_async_4(stg + 8 * k, reinterpret_cast<const uint16_t*>(a.offset) + 2 * i);
-                    if (a.mask) cp_async_4(stg + 40 + 4 * k, reinterpret_cast<const uint16_t*>(a.mask) + (i & ~1l));
-                } else {
-                    cp_async_8(stg + 8 * k, a.offset + 2 * i);
-                    if (a.mask) cp_async_4(stg + 40 + 4 * k, a.mask + i);
-                }
-            }
-        }
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-}
-
-__device__ __forceinline__ MetaIn staged_input(const TcArgs& a, uint32_t stg, int k, long i) {
-    MetaIn in;
-    if (a.off_f16) {
-        const uint32_t w = ld_shared_u32(stg + 8 * k);
-        in.d = make_float2(__half2float(__ushort_as_half((unsigned short)(w & 0xFFFFu))),
-                           __half2float(__ushort_as_half((unsigned short)(w >> 16))));
-        if (a.mask) {
-            const uint32_t mw = ld_shared_u32(stg + 40 + 4 * k);
-            in.mk = __half2float(__ushort_as_half((unsigned short)((i & 1) ? (mw >> 16) : (mw & 0xFFFFu))));
-        } else {
-            in.mk = 1.0f;
-        }
-    } else {
-        const uint2 w = make_uint2(ld_shared_u32(stg + 8 * k), ld_shared_u32(stg + 8 * k + 4));
-        in.d = make_float2(__uint_as_float(w.x), __uint_as_float(w.y));
-        in.mk = a.mask ? __uint_as_float(ld_shared_u32(stg + 40 + 4 * k)) : 1.0f;
-    }
-    return in;
-}
+constexpr int STG_TAPS = 5;   // entries per thread per round of the table build
 
 // The whole (tile, group) table, built by the NPT = TPM * BM producer threads: thread t owns
 // row t / TPM and taps t % TPM, + TPM, ... in rounds of STG_TAPS entries: all inputs of a round
-// are fetched (shared-memory staging or global loads) before any arithmetic, and the entries
+// are loaded before any arithmetic, and the entries
 // are computed as independent chains before any is stored.  Rows of warp w use the format of
 // that warp's sampler.
 constexpr int TPM = NPT / BM;    // producer threads per tile row in the metadata build
 static_assert(NPT % BM == 0, "metadata build assumes whole producer threads per tile row");
 template <int NTEX, int ME>
-__device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t,
-                                                 uint32_t stg = 0u) {
+__device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g, uint8_t* meta, int t) {
     const int row = t / TPM;
     const RowPos rp = row_pos(a, m0 + row);
     const bool tex_row = ((row % (NPW * RPW)) / RPW) < NTEX;
     const long pix = (long)(m0 + row) * a.G + g;
     uint8_t* rmeta = meta + row * a.KK * ME;
     if (t == 0) KT(16, g_kt_q);
-    if (stg) asm volatile("cp.async.wait_all;" ::: "memory");   // this thread's staged copies
-    if (t == 0) KT(17, g_kt_q);
     const long ibase = pix * a.KK;
     int i0 = (t % TPM) / a.Kw, j0 = (t % TPM) - ((t % TPM) / a.Kw) * a.Kw;
 #pragma unroll 1
@@ -348,12 +288,8 @@ __device__ __forceinline__ void build_meta_table(const TcArgs& a, int m0, int g,
 #pragma unroll
         for (int k = 0; k < STG_TAPS; ++k) {
             const int tk = min(tb + TPM * k, a.KK - 1);
-            if (stg) {   // staged (only when every tap fits one round)
-                in[k] = staged_input(a, stg, k, ibase + tk);
-            } else {
-                in[k].d = ld_offset2(a.offset, (ibase + tk) * 2, a.off_f16);
-                in[k].mk = a.mask ? ld_mask1(a.mask, ibase + tk, a.off_f16) : 1.0f;
-            }
+            in[k].d = ld_offset2(a.offset, (ibase + tk) * 2, a.off_f16);
+            in[k].mk = a.mask ? ld_mask1(a.mask, ibase + tk, a.off_f16) : 1.0f;
         }
         MetaVal v[STG_TAPS];
         int i = i0, j = j0;
@@ -872,8 +808,7 @@ template <bool TEXW, int STAGES, int NTEX, bool PAIR, bool F32>
 __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& sg, int& q, uint8_t* meta,
                                                 const uint32_t (&dst_lo)[ROWS], const uint32_t (&dst_hi)[ROWS],
                                                 const uint32_t (&mrow)[ROWS], uint32_t a_s, uint64_t* empty,
-                                                uint64_t* full_a, int t, int sub, int lane, int next_m0,
-                                                int next_g, uint32_t stg, int& staged_m0, int& staged_g) {
+                                                uint64_t* full_a, int t, int sub, int lane, int next_m0) {
     using Smp = typename std::conditional<F32, SamplerF32, Sampler<TEXW>>::type;
     using E = Elem<F32>;
     constexpr int ME = meta_entry<F32>();
@@ -882,14 +817,6 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     int chunk = sg.kb / a.KK;
     int tap = sg.kb - chunk * a.KK;
     int g = (chunk * E::CPI) / a.Cg;
-    const int g_last = (((sg.ke - 1) / a.KK) * E::CPI) / a.Cg;   // the segment's last offset group
-    // The table after (m0, gc): the segment's next group, else the next segment's first.
-    auto stage_after = [&](int gc) {
-        if (!stg) return;
-        staged_m0 = gc < g_last ? m0 : next_m0;
-        staged_g = gc < g_last ? gc + 1 : next_g;
-        stage_meta_inputs(a, staged_m0, staged_g, stg, t);
-    };
 #ifdef DEFCON_PROBE_KTRACE
     if (t == 0) g_kt_q = q;
 #endif
@@ -903,8 +830,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
     build_meta_table<NTEX, ME>(a, m0, g, meta, t, 0u);
     if (t == 0) KT(23, q);
 #endif
-    build_meta_table<NTEX, ME>(a, m0, g, meta, t, (stg && staged_m0 == m0 && staged_g == g) ? stg : 0u);
-    stage_after(g);
+    build_meta_table<NTEX, ME>(a, m0, g, meta, t);
     if (t == 0) KT(14, q);
     named_bar_sync(1, NPT);
     if (t == 0) KT(15, q);
@@ -957,8 +883,7 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         if (has_next && !prefetch) {          // offset group changes: new table
 #ifndef DEFCON_PROBE_NO_REBUILD   // dev probe (WRONG results for G > 1): keep the first table
             named_bar_sync(1, NPT);
-            build_meta_table<NTEX, ME>(a, m0, ng, meta, t, (stg && staged_m0 == m0 && staged_g == ng) ? stg : 0u);
-            stage_after(ng);
+            build_meta_table<NTEX, ME>(a, m0, ng, meta, t);
             named_bar_sync(1, NPT);
 #endif
             g = ng;
@@ -988,8 +913,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     uint8_t* sB = smem + STAGES * Cfg::A_STAGE_BYTES;
     uint8_t* epi_scratch = sB + STAGES * Cfg::B_STAGE_BYTES;   // 4 epilogue warps x EPI_W
     uint8_t* meta = epi_scratch + 4 * EPI_W;
-    uint8_t* stg_area = meta + BM * a.KK * meta_entry<F32>();   // NPT x STG_BYTES when a.stage_meta
-    uint64_t* bars = reinterpret_cast<uint64_t*>(stg_area + (a.stage_meta ? NPT * STG_BYTES : 0));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(meta + BM * a.KK * meta_entry<F32>());
     uint64_t* full_a = bars;
     uint64_t* full_b = bars + STAGES;
     uint64_t* empty = bars + 2 * STAGES;
@@ -1059,32 +983,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             mrow[p] = meta_s + row * a.KK * meta_entry<F32>();
         }
         int q = 0;                           // running k-iteration (stage) counter
-        const uint32_t stg = a.stage_meta ? smem_u32(stg_area) + t * STG_BYTES : 0u;
-        auto seg_group = [&](const Segment& sx) { return ((sx.kb / a.KK) * Elem<F32>::CPI) / a.Cg; };
-        int staged_m0 = -1, staged_g = -1;   // the table whose inputs sit in this thread's staging slot
-        if (stg && nseg > 0) {               // the first table: one round trip
-            const Segment s0 = segment_j(a, it_begin, it_end, seg_order(0, nseg));
-            staged_m0 = tile_m0<PAIR>(a, s0.tile);
-            staged_g = seg_group(s0);
-            stage_meta_inputs(a, staged_m0, staged_g, stg, t);
-        }
         for (int o = 0; o < nseg; ++o) {
             const Segment sg = segment_j(a, it_begin, it_end, seg_order(o, nseg));
-            int next_m0 = -1, next_g = 0;
-            if (o + 1 < nseg) {
-                const Segment sn = segment_j(a, it_begin, it_end, seg_order(o + 1, nseg));
-                next_m0 = tile_m0<PAIR>(a, sn.tile);
-                next_g = seg_group(sn);
-            }
+            const int next_m0 = o + 1 < nseg
+                ? tile_m0<PAIR>(a, segment_j(a, it_begin, it_end, seg_order(o + 1, nseg)).tile) : -1;
             if (t == 0 && o < 4) TL(2 + 2 * o);
             if (warp < NTEX)
                 produce_segment<true, STAGES, NTEX, PAIR, F32>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty,
-                                                               full_a, t, sub, lane, next_m0, next_g, stg,
-                                                               staged_m0, staged_g);
+                                                               full_a, t, sub, lane, next_m0);
             else
                 produce_segment<false, STAGES, NTEX, PAIR, F32>(a, sg, q, meta, dst_lo, dst_hi, mrow, a_s, empty,
-                                                                full_a, t, sub, lane, next_m0, next_g, stg,
-                                                                staged_m0, staged_g);
+                                                                full_a, t, sub, lane, next_m0);
             if (t == 0 && o < 4) TL(3 + 2 * o);
         }
         // The producers (4 lane quarters x NPW/4 column slices) run the last processed
@@ -1397,8 +1306,8 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     if (PAIR && g_pair_units == 0) {   // how many pairs fit at once (one CTA per SM)
         auto kp = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>;
         const size_t smem_q = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
-                              (size_t)BM * g.KK * meta_entry<false>() + (size_t)NPT * STG_BYTES +
-                              bias_smem_offset(STAGES, Cfg::NBUF) + (size_t)BIAS_SMEM_MAX * 4;
+                              (size_t)BM * g.KK * meta_entry<false>() + bias_smem_offset(STAGES, Cfg::NBUF) +
+                              (size_t)BIAS_SMEM_MAX * 4;
         cudaFuncSetAttribute(kp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_q);
         cudaLaunchConfig_t qc = {};
         qc.gridDim = dim3(num_sms());
@@ -1498,15 +1407,9 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
 
     a.bias_in_smem = g.Cout <= BIAS_SMEM_MAX ? 1 : 0;
     a.pair = PAIR ? 1 : 0;
-    // metadata staging (bf16 x, up to 10 taps): NPT x 64 bytes of shared memory
-#ifndef DEFCON_META_STAGE
-#define DEFCON_META_STAGE 0   // measured slower at C3 / C4 / C4 G4 (the 16 KB come out of L1)
-#endif
-    a.stage_meta = (DEFCON_META_STAGE && !F32 && g.KK <= (NPT / BM) * STG_TAPS) ? 1 : 0;
     // Stream-K tile counters are NOT reset here: the workspace is zero-filled once by its
     // owner and every launch leaves it zeroed (the finisher of each split tile resets it).
     const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_W + (size_t)BM * g.KK * meta_entry<F32>() +
-                        (a.stage_meta ? (size_t)NPT * STG_BYTES : 0) +
                         bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0);
     auto kern = F32 ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false, F32>
                 : PAIR ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>
@@ -1592,7 +1495,7 @@ cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, siz
     if (bn == 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
     if (bn == 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 #ifndef DEFCON_STAGES_256
-#define DEFCON_STAGES_256 2
+#define DEFCON_STAGES_256 3   // 2 -> 3 once the compact table freed 18 KB: C4 43.4 -> 42.0 us
 #endif
 #ifndef DEFCON_STAGES_PAIR
 #define DEFCON_STAGES_PAIR 4
