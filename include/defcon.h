@@ -136,6 +136,28 @@ int defcon_offset_workspace_size(int N, int H, int W, int C, int K, defcon_conv_
                                  size_t* bytes);
 
 /*
+ * Step 1 with parameters packed once (inference: the branch weights are constants).
+ * defcon_offset_pack_params writes dw_w / dw_scale / dw_shift / pw_w (same layouts as
+ * defcon_offset_dw_conv, OC = offset_groups*K*K*(modulated ? 3 : 2)) as the per-32-channel
+ * blocks the one-pass kernel streams (W2 as tf32 hi / lo in the tensor-core operand image, dw
+ * taps and folded BN) into `packed` (defcon_offset_packed_size() bytes, caller-owned device
+ * memory, 16-byte aligned); it is asynchronous on `stream`.  defcon_offset_dw_conv_packed then
+ * computes exactly what defcon_offset_dw_conv computes from those parameters (bit-identical
+ * results) without re-packing them per call; `packed` is only read, so one buffer serves
+ * concurrent calls.  modulated must match (mask != NULL).
+ * Errors: as defcon_offset_dw_conv; UNSUPPORTED for shapes that run the two-launch branch
+ * (input rows wider than the one-pass kernel's TMA box; use defcon_offset_dw_conv there);
+ * LIMIT if packed_bytes is too small.
+ */
+int defcon_offset_packed_size(int C, int K, int offset_groups, int modulated, size_t* bytes);
+int defcon_offset_pack_params(int C, int K, int offset_groups, int modulated, const float* dw_w,
+                              const float* dw_scale, const float* dw_shift, const float* pw_w,
+                              void* packed, size_t packed_bytes, void* stream);
+int defcon_offset_dw_conv_packed(const void* x, int N, int H, int W, int C, int x_dtype,
+                                 const void* packed, size_t packed_bytes, const float* pw_b, int K,
+                                 defcon_conv_t cv, float* offset, float* mask, void* stream);
+
+/*
  * Step 2 -- deformable convolution forward, Eq.2 + Eq.3:
  *   y[n][ho][wo][co] = bias[co] + sum_{i<Kh, j<Kw, ci<Cin} weight[co][i][j][ci]
  *                      * m[n][ho][wo][g][k] * X(n, ci, p_y, p_x)

@@ -14,6 +14,8 @@ from ._binding import (  # noqa: F401
     defcon_layer_forward_host,
     defcon_layer_workspace_size,
     defcon_offset_dw_conv,
+    defcon_offset_dw_conv_packed,
+    defcon_offset_pack_params,
     defcon_offset_workspace_size,
     defcon_tex_filter_probe,
     load_library,

@@ -23,7 +23,8 @@ DEFCON_FP32_3XTF32, DEFCON_FP32_SIMT = 0, 1
 
 # Every symbol include/defcon.h declares (checked by tests/test_abi.py).
 EXPORTED = (
-    "defcon_offset_dw_conv", "defcon_offset_workspace_size", "defcon_dcn_forward",
+    "defcon_offset_dw_conv", "defcon_offset_workspace_size", "defcon_offset_packed_size",
+    "defcon_offset_pack_params", "defcon_offset_dw_conv_packed", "defcon_dcn_forward",
     "defcon_dcn_workspace_size", "defcon_deform_columns",
     "defcon_layer_forward_host", "defcon_layer_workspace_size", "defcon_tex_plan_create",
     "defcon_tex_plan_destroy", "defcon_tex_filter_probe", "defcon_status_string",
@@ -70,6 +71,9 @@ def load_library(path: str = None):
     lib.defcon_offset_dw_conv.argtypes = [vp, i, i, i, i, i, fp, fp, fp, fp, fp, i, conv, fp, fp, vp,
                                           sz, vp]
     lib.defcon_offset_workspace_size.argtypes = [i, i, i, i, i, conv, ctypes.POINTER(sz)]
+    lib.defcon_offset_packed_size.argtypes = [i, i, i, i, ctypes.POINTER(sz)]
+    lib.defcon_offset_pack_params.argtypes = [i, i, i, i, fp, fp, fp, fp, vp, sz, vp]
+    lib.defcon_offset_dw_conv_packed.argtypes = [vp, i, i, i, i, i, vp, sz, fp, i, conv, fp, fp, vp]
     lib.defcon_dcn_forward.argtypes = [vp, i, i, i, i, fp, fp, vp, fp, i, i, i, conv, i, i, i, vp, vp,
                                        sz, vp, vp]
     lib.defcon_dcn_workspace_size.argtypes = [i, i, i, i, i, i, i, conv, i, i, i,
@@ -207,6 +211,65 @@ def defcon_offset_dw_conv(x, dw_w, dw_scale, dw_shift, pw_w, pw_b=None, K=3, str
                                    workspace.numel() * workspace.element_size(),
                                    _stream_handle(stream))
     _check(rc, "defcon_offset_dw_conv")
+    return offset, mask
+
+
+def defcon_offset_pack_params(dw_w, dw_scale, dw_shift, pw_w, K=3, offset_groups=1, with_mask=True,
+                              packed=None, stream=None):
+    """Step 1's parameters packed once per set of weights (include/defcon.h,
+    defcon_offset_pack_params); returns the packed uint8 device tensor for
+    defcon_offset_dw_conv_packed."""
+    lib = load_library()
+    C = int(dw_w.shape[0])
+    G, KK = int(offset_groups), K * K
+    OC = G * KK * (3 if with_mask else 2)
+    _dev_tensor(dw_w, "dw_w", torch.float32, (C, 3, 3))
+    _dev_tensor(dw_scale, "dw_scale", torch.float32, (C,))
+    _dev_tensor(dw_shift, "dw_shift", torch.float32, (C,))
+    _dev_tensor(pw_w, "pw_w", torch.float32, (OC, C))
+    out = ctypes.c_size_t(0)
+    _check(lib.defcon_offset_packed_size(C, K, G, int(with_mask), ctypes.byref(out)), "defcon_offset_packed_size")
+    with _on(stream):
+        if packed is None:
+            packed = torch.empty(int(out.value), dtype=torch.uint8, device=dw_w.device)
+    _dev_tensor(packed, "packed")
+    rc = lib.defcon_offset_pack_params(C, K, G, int(with_mask), _ptr(dw_w), _ptr(dw_scale), _ptr(dw_shift),
+                                       _ptr(pw_w), _ptr(packed), packed.numel() * packed.element_size(),
+                                       _stream_handle(stream))
+    _check(rc, "defcon_offset_pack_params")
+    return packed
+
+
+def defcon_offset_dw_conv_packed(x, packed, pw_b=None, K=3, stride=1, pad=1, dil=1, offset_groups=1,
+                                 with_mask=True, offset=None, mask=None, stream=None,
+                                 offset_dtype=torch.float32):
+    """Step 1 from pre-packed parameters (defcon_offset_pack_params): the same results as
+    defcon_offset_dw_conv without the per-call parameter packing."""
+    lib = load_library()
+    _dev_tensor(x, "x")
+    if x.dtype not in _DTYPES:
+        raise ValueError("x must be float32 or bfloat16")
+    _dev_tensor(packed, "packed")
+    N, H, W, C = x.shape
+    cv = _conv(stride, pad, dil, offset_groups, 0, offset_dtype)
+    Ho, Wo = _out(H, 3, cv.stride_h, cv.pad_h, cv.dil_h), _out(W, 3, cv.stride_w, cv.pad_w, cv.dil_w)
+    G, KK = int(offset_groups), K * K
+    OC = G * KK * (3 if with_mask else 2)
+    _dev_tensor(pw_b, "pw_b", torch.float32, (OC,), allow_none=True)
+    with _on(stream):
+        if offset is None:
+            offset = torch.empty((N, Ho, Wo, G, KK, 2), device=x.device, dtype=offset_dtype)
+        if with_mask and mask is None:
+            mask = torch.empty((N, Ho, Wo, G, KK), device=x.device, dtype=offset_dtype)
+    _dev_tensor(offset, "offset", offset_dtype, (N, Ho, Wo, G, KK, 2))
+    if with_mask:
+        _dev_tensor(mask, "mask", offset_dtype, (N, Ho, Wo, G, KK))
+    else:
+        mask = None
+    rc = lib.defcon_offset_dw_conv_packed(_ptr(x), N, H, W, C, _DTYPES[x.dtype], _ptr(packed),
+                                          packed.numel() * packed.element_size(), _ptr(pw_b), K, cv,
+                                          _ptr(offset), _ptr(mask), _stream_handle(stream))
+    _check(rc, "defcon_offset_dw_conv_packed")
     return offset, mask
 
 

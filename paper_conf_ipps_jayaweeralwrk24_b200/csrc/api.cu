@@ -221,6 +221,67 @@ int defcon_offset_dw_conv(const void* x, int N, int H, int W, int C, int x_dtype
     return DEFCON_OK;
 }
 
+int defcon_offset_packed_size(int C, int K, int offset_groups, int modulated, size_t* bytes) {
+    g_detail[0] = 0;
+    if (!bytes) return fail(DEFCON_ERR_INVALID_ARG, "bytes is NULL");
+    if (C <= 0 || K <= 0 || offset_groups <= 0) return fail(DEFCON_ERR_INVALID_ARG, "sizes must be positive");
+    if (C % 8 != 0) return fail(DEFCON_ERR_UNSUPPORTED, "offset branch needs C %% 8 == 0 (C = %d)", C);
+    const int OC = offset_groups * K * K * (modulated ? 3 : 2);
+    if (OC > 256) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 256", OC);
+    *bytes = offset_branch_onepass_workspace(C, OC);
+    return DEFCON_OK;
+}
+
+int defcon_offset_pack_params(int C, int K, int offset_groups, int modulated, const float* dw_w,
+                              const float* dw_scale, const float* dw_shift, const float* pw_w, void* packed,
+                              size_t packed_bytes, void* stream) {
+    size_t need = 0;
+    int rc = defcon_offset_packed_size(C, K, offset_groups, modulated, &need);
+    if (rc) return rc;
+    if (!dw_w || !dw_scale || !dw_shift || !pw_w || !packed) return fail(DEFCON_ERR_INVALID_ARG, "NULL pointer");
+    const void* ptrs[] = {dw_w, dw_scale, dw_shift, pw_w, packed};
+    for (const void* p : ptrs)
+        if (!aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "pointer not 16-byte aligned");
+    if (packed_bytes < need) return fail(DEFCON_ERR_LIMIT, "packed buffer of %zu bytes < required %zu", packed_bytes, need);
+    const int OC = offset_groups * K * K * (modulated ? 3 : 2);
+    cudaError_t e = launch_offset_pack(dw_w, dw_scale, dw_shift, pw_w, C, OC, packed, static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "offset parameter pack launch");
+    return DEFCON_OK;
+}
+
+int defcon_offset_dw_conv_packed(const void* x, int N, int H, int W, int C, int x_dtype, const void* packed,
+                                 size_t packed_bytes, const float* pw_b, int K, defcon_conv_t cv, float* offset,
+                                 float* mask, void* stream) {
+    g_detail[0] = 0;
+    int Ho, Wo;
+    int rc = branch_geom(N, H, W, C, K, cv, &Ho, &Wo);
+    if (rc) return rc;
+    if (x_dtype != DEFCON_F32 && x_dtype != DEFCON_BF16) return fail(DEFCON_ERR_INVALID_ARG, "bad dtype");
+    if (!x || !packed || !offset) return fail(DEFCON_ERR_INVALID_ARG, "NULL tensor pointer");
+    const void* ptrs[] = {x, packed, pw_b, offset, mask};
+    for (const void* p : ptrs)
+        if (p && !aligned16(p)) return fail(DEFCON_ERR_MISALIGNED, "tensor pointer not 16-byte aligned");
+    const int G = cv.offset_groups;
+    const int OC = G * K * K * (mask ? 3 : 2);
+    if (OC > 256) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d > 256", OC);
+    if ((long)N * Ho * Wo * OC >= (1L << 31))
+        return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
+    if (!offset_branch_is_onepass(N, H, W, C, Ho, Wo, K, G, cv.stride_h, cv.stride_w, cv.pad_h, cv.pad_w, cv.dil_h,
+                                  cv.dil_w, x_dtype == DEFCON_BF16))
+        return fail(DEFCON_ERR_UNSUPPORTED, "this shape runs the two-launch branch: use defcon_offset_dw_conv");
+    if (packed_bytes < offset_branch_onepass_workspace(C, OC))
+        return fail(DEFCON_ERR_LIMIT, "packed buffer of %zu bytes < required %zu", packed_bytes,
+                    offset_branch_onepass_workspace(C, OC));
+    cudaError_t e = launch_offset_branch(x, x_dtype == DEFCON_BF16, N, H, W, C, nullptr, nullptr, nullptr, nullptr,
+                                         pw_b, K, G, mask != nullptr, cv.stride_h, cv.stride_w, cv.pad_h, cv.pad_w,
+                                         cv.dil_h, cv.dil_w, Ho, Wo, offset, mask,
+                                         static_cast<float*>(const_cast<void*>(packed)),
+                                         static_cast<cudaStream_t>(stream), cv.offset_dtype == DEFCON_F16, true);
+    if (e == cudaErrorInvalidValue) return fail(DEFCON_ERR_LIMIT, "offset branch OC = %d unsupported", OC);
+    if (e != cudaSuccess) return cuda_fail(e, "offset_branch launch");
+    return DEFCON_OK;
+}
+
 int defcon_dcn_workspace_size(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
                               defcon_conv_t cv, int dtype, int sampler, int fp32_mode,
                               size_t* bytes) {

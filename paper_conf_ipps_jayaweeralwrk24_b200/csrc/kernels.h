@@ -35,7 +35,10 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                  float* offset, float* mask, float* t_ws, cudaStream_t stream,
-                                 bool out_f16 = false);
+                                 bool out_f16 = false, bool prepacked = false);
+// true when step 1 runs as the one-pass kernel for this shape (its parameters can be pre-packed)
+bool offset_branch_is_onepass(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph,
+                              int pw, int dh, int dw, bool x_bf16);
 // workspace of defcon_offset_dw_conv: the one-pass kernel's packed parameters when it can run
 // this shape (decided for the widest branch, OC = 3*G*K*K), else the two-pass t buffers
 size_t offset_branch_workspace(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph,
@@ -50,7 +53,9 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
                                          const float* pw_w, const float* pw_b, int n_off, int n_msk,
                                          int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                          float* offset, float* mask, void* ws, cudaStream_t stream,
-                                         bool out_f16);
+                                         bool out_f16, bool prepacked = false);
+cudaError_t launch_offset_pack(const float* dw_w, const float* dw_scale, const float* dw_shift, const float* pw_w,
+                               int C, int OC, void* packed, cudaStream_t stream);
 // ---- sampling step alone: deformable columns [M][KK*Cin] (sampler.cu)
 cudaError_t launch_deform_columns(const DcnGeom& g, const void* x, const float* offset, const float* mask,
                                   bool bf16, void* cols, cudaStream_t stream);

@@ -521,12 +521,17 @@ size_t offset_branch_workspace(int N, int H, int W, int C, int Ho, int Wo, int K
     return two_pass_workspace(N * Ho * Wo, C);
 }
 
+bool offset_branch_is_onepass(int N, int H, int W, int C, int Ho, int Wo, int K, int G, int sh, int sw, int ph,
+                              int pw, int dh, int dw, bool x_bf16) {
+    return use_onepass(N, H, W, C, Ho, Wo, K, G, sh, sw, ph, pw, dh, dw, x_bf16);
+}
+
 cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W, int C,
                                  const float* dw_w, const float* dw_scale, const float* dw_shift,
                                  const float* pw_w, const float* pw_b, int K, int G, bool with_mask,
                                  int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                  float* offset, float* mask, float* t_ws, cudaStream_t stream,
-                                 bool out_f16) {
+                                 bool out_f16, bool prepacked) {
     BranchArgs a;
     a.out_f16 = out_f16 ? 1 : 0;
     a.x = x; a.dw_w = dw_w; a.dw_scale = dw_scale; a.dw_shift = dw_shift;
@@ -543,7 +548,8 @@ cudaError_t launch_offset_branch(const void* x, bool x_bf16, int N, int H, int W
     if (use_onepass(N, H, W, C, Ho, Wo, K, G, s_h, s_w, p_h, p_w, d_h, d_w, x_bf16))
         return launch_offset_branch_onepass(x, x_bf16, N, H, W, C, dw_w, dw_scale, dw_shift, pw_w, pw_b,
                                             a.n_off, a.n_msk, s_h, s_w, p_h, p_w, d_h, d_w, Ho, Wo, offset,
-                                            mask, t_ws, stream, out_f16);
+                                            mask, t_ws, stream, out_f16, prepacked);
+    if (prepacked) return cudaErrorNotSupported;   // pre-packed parameters serve the one-pass kernel only
     // 1x1 on tcgen05 from TMA-loaded hi / lo planes, or the mma.sync 3xTF32 kernel (t in one
     // plane)
     // The tcgen05 kernel runs one 128-pixel tile per CTA, two CTAs per SM, each CTA a latency

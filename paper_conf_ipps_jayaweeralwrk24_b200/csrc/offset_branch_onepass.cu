@@ -700,12 +700,21 @@ size_t offset_branch_onepass_workspace(int C, int OC) {
     return (size_t)((C + OP_KC - 1) / OP_KC) * op_block_bytes(OCN);
 }
 
+// The per-chunk parameter blocks (W2 hi / lo in the UMMA B image + dw / BN), OC outputs.
+cudaError_t launch_offset_pack(const float* dw_w, const float* dw_scale, const float* dw_shift, const float* pw_w,
+                               int C, int OC, void* packed, cudaStream_t stream) {
+    const int OCN = (OC + 15) & ~15;
+    const int nch = (C + OP_KC - 1) / OP_KC;
+    return launch_pdl(op_pack_kernel, dim3(nch, (OCN * OP_KC + 255) / 256), dim3(256), 0, stream, dw_w, dw_scale,
+                      dw_shift, pw_w, C, OC, OCN, static_cast<uint8_t*>(packed));
+}
+
 cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int H, int W, int C,
                                          const float* dw_w, const float* dw_scale, const float* dw_shift,
                                          const float* pw_w, const float* pw_b, int n_off, int n_msk,
                                          int s_h, int s_w, int p_h, int p_w, int d_h, int d_w, int Ho, int Wo,
                                          float* offset, float* mask, void* ws, cudaStream_t stream,
-                                         bool out_f16) {
+                                         bool out_f16, bool prepacked) {
     const int es = x_bf16 ? 2 : 4;
     OpPlan p;
     if (!make_op_plan(N, H, W, C, Ho, Wo, s_h, s_w, p_h, p_w, d_h, d_w, n_off + n_msk, es, &p))
@@ -718,11 +727,10 @@ cudaError_t launch_offset_branch_onepass(const void* x, bool x_bf16, int N, int 
     a.packed = static_cast<const uint8_t*>(ws);
     // PDL launch: its launch overlaps the previous kernel; it waits for that kernel before writing
     // (measured A/B on one box: bench step 75.5 -> 74.8 us, host entry 0.70 -> 0.56 ms)
-#ifndef DEFCON_PROBE_NO_PACK   // dev probe (stale parameters unless packed before): the pack kernel's cost
-    cudaError_t e = launch_pdl(op_pack_kernel, dim3(a.nch, (a.OCN * OP_KC + 255) / 256), dim3(256), 0, stream, dw_w,
-                               dw_scale, dw_shift, pw_w, C, a.OC, a.OCN, static_cast<uint8_t*>(ws));
-    if (e != cudaSuccess) return e;
-#endif
+    if (!prepacked) {   // else ws holds the blocks of defcon_offset_pack_params (packed once per weights)
+        cudaError_t e = launch_offset_pack(dw_w, dw_scale, dw_shift, pw_w, C, a.OC, ws, stream);
+        if (e != cudaSuccess) return e;
+    }
     PFN_encodeTiled encode = get_encode_tiled();
     if (!encode) return cudaErrorNotSupported;
     // x as a 3-D tensor [N*H][W][C] (C innermost); box = 32 channels x IC columns x IR rows

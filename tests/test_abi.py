@@ -110,6 +110,28 @@ def test_offset_branch_validation(lib):
     assert out.value in ((2 * 32 * 128 + 352 * 4 + 1023) // 1024 * 1024, (2 * 8 * 8 * 16 + 2 * 256 * 16) * 4)
 
 
+def test_offset_prepack_validation(lib):
+    """defcon_offset_packed_size / defcon_offset_pack_params / defcon_offset_dw_conv_packed reject
+    bad arguments before any launch (include/defcon.h)."""
+    V, sz = ctypes.c_void_p, ctypes.c_size_t(0)
+    assert lib.defcon_offset_packed_size(256, 3, 1, 1, ctypes.byref(sz)) == 0
+    # 8 chunks of 32 channels, one 1 KB-aligned block each (W2 hi / lo for 27 -> 32 rows + dw / BN)
+    assert sz.value == 8 * ((2 * 32 * 128 + 352 * 4 + 1023) // 1024 * 1024)
+    assert lib.defcon_offset_packed_size(12, 3, 1, 1, ctypes.byref(sz)) == 2            # C % 8
+    assert lib.defcon_offset_packed_size(256, 3, 64, 1, ctypes.byref(sz)) == 5          # OC > 256
+    assert lib.defcon_offset_packed_size(0, 3, 1, 1, ctypes.byref(sz)) == 1
+    P = [V(FAKE)] * 4
+    assert lib.defcon_offset_pack_params(256, 3, 1, 1, *P, V(FAKE), 16, None) == 5      # too small
+    assert lib.defcon_offset_pack_params(256, 3, 1, 1, *P, V(FAKE + 4), 1 << 30, None) == 3
+    assert lib.defcon_offset_pack_params(256, 3, 1, 1, V(0), *P[1:], V(FAKE), 1 << 30, None) == 1
+    args = [V(FAKE), 1, 8, 8, 16, 1, V(FAKE), 1 << 30, V(FAKE), 3]
+    assert lib.defcon_offset_dw_conv_packed(*args, _conv(), V(0), V(FAKE), None) == 1     # offset NULL
+    assert lib.defcon_offset_dw_conv_packed(*args, _conv(), V(FAKE + 4), V(FAKE), None) == 3
+    bad = list(args)
+    bad[5] = 7
+    assert lib.defcon_offset_dw_conv_packed(*bad, _conv(), V(FAKE), V(FAKE), None) == 1   # dtype
+
+
 def test_workspace_size_and_layer_size(lib):
     out = ctypes.c_size_t(99)
     # bf16 tensor-core path: stream-K counters + fp32 partial tiles

@@ -414,6 +414,42 @@ def test_offset_branch_parity(oracle_mod, d, dev, c):
     assert 0.5 < float(np.std(ro)) < 4.0
 
 
+@pytest.mark.parametrize("c", [configs.C4.replace(N=2), configs.C4_G4.replace(N=2),
+                               small("pk_v1_f32", dtype="f32", Cin=64, N=2, H=17, W=15, modulated=False),
+                               small("pk_s2_f16", Cin=96, N=2, H=25, W=21, stride=2)],
+                         ids=lambda c: c.name)
+def test_offset_branch_prepacked(oracle_mod, d, dev, c):
+    """defcon_offset_pack_params + defcon_offset_dw_conv_packed (include/defcon.h): bit-identical
+    to the per-call path (the same packed blocks feed the same kernel), one packed buffer reused
+    by several calls, and binary16 outputs (R13); two-launch shapes are refused (UNSUPPORTED)."""
+    x = to_dev(inputs.gen_x(c), TDT[c.dtype], dev)
+    P, Pd = gen_branch_dev(c, dev)
+    kw = dict(K=c.K, stride=c.stride, pad=c.pad, dil=c.dil, offset_groups=c.G, with_mask=c.modulated)
+    ref_o, ref_m = d.defcon_offset_dw_conv(x, Pd["dw_w"], Pd["dw_scale"], Pd["dw_shift"], Pd["pw_w"], Pd["pw_b"], **kw)
+    packed = d.defcon_offset_pack_params(Pd["dw_w"], Pd["dw_scale"], Pd["dw_shift"], Pd["pw_w"], K=c.K,
+                                         offset_groups=c.G, with_mask=c.modulated)
+    for _ in range(2):
+        o, m = d.defcon_offset_dw_conv_packed(x, packed, Pd["pw_b"], **kw)
+        torch.cuda.synchronize()
+        assert torch.equal(o, ref_o)
+        if c.modulated:
+            assert torch.equal(m, ref_m)
+    o16, m16 = d.defcon_offset_dw_conv_packed(x, packed, Pd["pw_b"], offset_dtype=torch.float16, **kw)
+    torch.cuda.synchronize()
+    assert torch.equal(o16, ref_o.to(torch.float16))
+    ro, _ = oracle_mod.offset_branch(x.float().cpu().numpy(), P["dw_w"], P["dw_scale"], P["dw_shift"], P["pw_w"],
+                                     P["pw_b"], K=c.K, G=c.G, with_mask=c.modulated, stride=c.stride, pad=c.pad,
+                                     dil=c.dil)
+    assert normwise(o.cpu().numpy(), ro) < 1e-5
+    wide = small("pk_wide", Cin=16, N=1, H=16, W=300)
+    xw = to_dev(inputs.gen_x(wide), torch.bfloat16, dev)
+    Pw, Pwd = gen_branch_dev(wide, dev)
+    pk = d.defcon_offset_pack_params(Pwd["dw_w"], Pwd["dw_scale"], Pwd["dw_shift"], Pwd["pw_w"])
+    with pytest.raises(d.DefconError) as ei:
+        d.defcon_offset_dw_conv_packed(xw, pk, Pwd["pw_b"])
+    assert ei.value.status == 2
+
+
 @pytest.mark.parametrize("tp,split", [(64, 1), (128, 1), (48, 2), (128, 2)])
 @pytest.mark.parametrize("c", [small("op_c96", Cin=96, N=2, H=23, W=19),                 # 3 chunks: 2 + 1 split
                                configs.C4_G4.replace(N=2),                                 # OC 108 -> 112 columns
