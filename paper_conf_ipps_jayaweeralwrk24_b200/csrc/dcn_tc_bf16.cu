@@ -1493,7 +1493,10 @@ cudaError_t launch_dcn_tc_bf16(const DcnGeom& g, const DcnPtrs& p, void* ws, siz
                                const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
     const int bn = tc_block_n(g);
     if (bn == 64) return launch_impl<64, 6>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
-    if (bn == 128) return launch_impl<128, 4>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
+#ifndef DEFCON_STAGES_128
+#define DEFCON_STAGES_128 3   // 4 -> 3: C3 37.3 -> 36.5 us (more L1 for the gathers)
+#endif
+    if (bn == 128) return launch_impl<128, DEFCON_STAGES_128>(g, p, ws, ws_bytes, tex, hybrid, stream, detail);
 #ifndef DEFCON_STAGES_256
 #define DEFCON_STAGES_256 3   // 2 -> 3 once the compact table freed 18 KB: C4 43.4 -> 42.0 us
 #endif
