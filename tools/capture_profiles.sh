@@ -11,7 +11,7 @@ python bench.py > gpurun_out/${R}_bench.json 2> gpurun_out/${R}_bench.err
 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv \
     --log-file gpurun_out/${R}_launches.csv python bench.py --steps 4 --warmup 3 --no-cpu-baseline > /dev/null 2>&1
 # one full capture per hot-path kernel, same command
-ncu --set full --clock-control none --import-source on -k regex:"dcn_fwd|offset_branch_onepass|op_pack" -s 3 -c 3 \
+ncu --set full --clock-control none --import-source on -k regex:"dcn_fwd|offset_branch_onepass" -s 4 -c 2 \
     -o gpurun_out/${R}_full python bench.py --steps 4 --warmup 3 --no-cpu-baseline > /dev/null 2>&1
 ncu -i gpurun_out/${R}_full.ncu-rep --page details --csv > gpurun_out/${R}_full_details.csv 2>/dev/null
 ncu -i gpurun_out/${R}_full.ncu-rep --page raw --csv > gpurun_out/${R}_full_raw.csv 2>/dev/null
