@@ -5,7 +5,7 @@ fp32 3xTF32, the TEX sampler, bounded deformation, the columns kernel, and both 
 paths (one-pass; two-launch for wide rows).  Each case is checked loosely against the oracle
 (the parity suite holds the tight gates).
 
-  compute-sanitizer --tool memcheck python tools/sanitize_cases.py
+  compute-sanitizer --tool memcheck python tests/tools/sanitize_cases.py
 """
 import os
 import sys
@@ -13,7 +13,7 @@ import sys
 import numpy as np
 import torch
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 import oracle  # noqa: E402  (test infrastructure: the checker)
 from defcon_workloads import configs, inputs  # noqa: E402
