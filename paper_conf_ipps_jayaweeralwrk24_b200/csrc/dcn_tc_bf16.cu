@@ -59,6 +59,9 @@ constexpr int META_ENTRY = 32;   // the largest entry (shape-support checks)
 #define DEFCON_NPW 8
 #endif
 constexpr int NPW = DEFCON_NPW;  // producer warps (8 or 16)
+#ifndef DEFCON_LATE_LAST
+#define DEFCON_LATE_LAST 0   // 1: the last row's next gathers after the full_a arrive, 2: all rows (DESIGN 12b)
+#endif
 constexpr int EPI_WARP0 = NPW;   // 4 epilogue warps: TMEM lane quarters 0..3
 constexpr int TMA_WARP = NPW + 4;
 constexpr int MMA_WARP = NPW + 5;
@@ -861,7 +864,10 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
         for (int p = 0; p < ROWS; ++p) {    // rolling prefetch of the next k-iteration
             Smp::store(L[p], stage + dst_lo[p], stage + dst_hi[p]);
             if (t == 0) KT(8 + p, q);
-            if (prefetch) Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * ME, pb);
+            // the last row's gathers go out after the arrive: the proxy fence below lowers to
+            // MEMBAR.ALL.CTA, which waits for this thread's outstanding loads
+            if (prefetch && (DEFCON_LATE_LAST == 0 || (DEFCON_LATE_LAST == 1 && p + 1 < ROWS)))
+                Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * ME, pb);
         }
 #ifdef DEFCON_PROBE_NO_FENCE   // dev probe (WRONG results): no proxy fence, relaxed arrive -- the
                                // cost of ordering the A stores before the MMA
@@ -879,6 +885,11 @@ __device__ __forceinline__ void produce_segment(const TcArgs& a, const Segment& 
 #endif
         if (t == 0) KT(2, q);
         if (t == 224) KT(7, q);   // the last producer warp
+        if (DEFCON_LATE_LAST && prefetch) {
+#pragma unroll
+            for (int p = DEFCON_LATE_LAST == 1 ? ROWS - 1 : 0; p < ROWS; ++p)
+                Smp::issue(L[p], nxb, a.tex, nlayer, mrow[p] + ntap * ME, pb);
+        }
 
         if (has_next && !prefetch) {          // offset group changes: new table
 #ifndef DEFCON_PROBE_NO_REBUILD   // dev probe (WRONG results for G > 1): keep the first table
