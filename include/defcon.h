@@ -190,8 +190,9 @@ int defcon_offset_dw_conv_packed(const void* x, int N, int H, int W, int C, int 
  *            prologue may overlap the previous kernel on `stream`, never its data.
  * Errors: INVALID_ARG for non-positive sizes, Ho/Wo <= 0, G not dividing Cin, bad enums,
  *   NULL required pointers; UNSUPPORTED for (Cin/G) % 8 != 0 (bf16) or % 4 != 0 (fp32),
- *   or a Cout not multiple of 16 on the tensor-core paths; LIMIT when N*H*W*Cin >= 2^31
- *   or the workspace is too small; MISALIGNED for pointers not 16-byte aligned, or x not
+ *   or a Cout not multiple of 16 on the tensor-core paths; LIMIT when N*H*W*Cin >= 2^31,
+ *   x spans >= 4 GiB (the samplers use 32-bit byte offsets) or the workspace is too small;
+ *   MISALIGNED for pointers not 16-byte aligned, or x not
  *   32-byte aligned on the bf16 tensor-core path.
  */
 int defcon_dcn_forward(const void* x, int N, int H, int W, int Cin,

@@ -89,6 +89,9 @@ static int make_geom(int N, int H, int W, int Cin, int Cout, int Kh, int Kw,
     if ((long)N * H * W * Cin >= (1L << 31) || M * Cout >= (1L << 31) ||
         M * g->G * g->KK * 2 >= (1L << 31) || (long)Cout * g->KK * Cin >= (1L << 31))
         return fail(DEFCON_ERR_LIMIT, "tensor too large for 32-bit element indexing");
+    // the samplers address x by 32-bit byte offsets from its base (sampling metadata)
+    if ((long)N * H * W * Cin * (dtype == DEFCON_BF16 ? 2 : 4) >= (1L << 32))
+        return fail(DEFCON_ERR_LIMIT, "x larger than 4 GiB (32-bit byte offsets)");
     g->M = (int)M;
     const int vec = dtype == DEFCON_BF16 ? 8 : 4;
     if (g->Cg % vec != 0)

@@ -110,6 +110,18 @@ def test_offset_branch_validation(lib):
     assert out.value in ((2 * 32 * 128 + 352 * 4 + 1023) // 1024 * 1024, (2 * 8 * 8 * 16 + 2 * 256 * 16) * 4)
 
 
+def test_dcn_forward_x_byte_limit(lib):
+    """fp32 x of 2^30 elements (4 GiB) passes the element-count limit but not the samplers'
+    32-bit byte offsets: LIMIT before any launch; the same shape in bf16 (2 GiB) is accepted by
+    the size query."""
+    out = ctypes.c_size_t(0)
+    # N=1, H=W=1024, Cin=1024, Cout=16, K=1 (pad 0): x = 2^30 elements
+    assert lib.defcon_dcn_workspace_size(1, 1024, 1024, 1024, 16, 1, 1, _conv(pad_h=0, pad_w=0), 0, 0, 0,
+                                         ctypes.byref(out)) == 5
+    assert lib.defcon_dcn_workspace_size(1, 1024, 1024, 1024, 16, 1, 1, _conv(pad_h=0, pad_w=0), 1, 0, 0,
+                                         ctypes.byref(out)) == 0
+
+
 def test_offset_prepack_validation(lib):
     """defcon_offset_packed_size / defcon_offset_pack_params / defcon_offset_dw_conv_packed reject
     bad arguments before any launch (include/defcon.h)."""
