@@ -926,7 +926,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     uint8_t* meta = epi_scratch + 4 * EPI_W;
     uint64_t* bars = reinterpret_cast<uint64_t*>(meta + BM * a.KK * meta_entry<F32>());
     uint64_t* full_a = bars;
-    uint64_t* full_b = bars + STAGES;
+    // single CTAs: the producers' arrivals and the weight TMA's transaction bytes complete ONE
+    // barrier per stage (NPW + 1 arrivals), so the MMA issuer waits once per k-iteration
+#ifndef DEFCON_SPLIT_FULL
+    constexpr bool MERGED = !PAIR;
+#else
+    constexpr bool MERGED = false;
+#endif
+    uint64_t* full_b = MERGED ? bars : bars + STAGES;
     uint64_t* empty = bars + 2 * STAGES;
     uint64_t* tmem_full = bars + 3 * STAGES;
     uint64_t* tmem_empty = tmem_full + Cfg::NBUF;
@@ -949,8 +956,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
     if (warp == TMA_WARP && lane == 0) {
         for (int s = 0; s < STAGES; ++s) {
-            mbar_init(&full_a[s], PAIR ? 2 * NPW : NPW);   // pair: both CTAs' producers
-            mbar_init(&full_b[s], 1);
+            mbar_init(&full_a[s], PAIR ? 2 * NPW : MERGED ? NPW + 1 : NPW);   // pair: both CTAs' producers
+            if (!MERGED) mbar_init(&full_b[s], 1);
             mbar_init(&empty[s], 1);
         }
         for (int b = 0; b < Cfg::NBUF; ++b) {
@@ -1112,7 +1119,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         KT(3, q);
                         mbar_wait(&full_a[s], ph);
                         KT(4, q);
-                        mbar_wait(&full_b[s], ph);
+                        if (!MERGED) mbar_wait(&full_b[s], ph);
                         KT(5, q);
                     }
                     tc_fence_after();
@@ -1142,7 +1149,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                                 mma_bf16_ss(d_base + h * Cfg::UMMA_N, adesc, bdesc, idesc, acc);
                             }
                         }
+                        if (kk == 0) KT(16, q);
                     }
+                    KT(17, q);
                     if (PAIR) mma_commit_pair(&empty[s], 0x3);
                     else mma_commit(&empty[s]);
                     KT(6, q);

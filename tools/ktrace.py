@@ -30,6 +30,8 @@ for q in range(n):
     if buf[12, q]:
         print(f"segment start at q={q}: sync1 {b[12,q]} -> {b[13,q]}, build -> {b[14,q]}, sync2 -> {b[15,q]}; "
               f"build: enter {b[16,q]} waited {b[17,q]} round done {b[18,q]}; (probe: first build done {b[23,q]})")
+print("MMA warp per q: gotB->1st MMA issued, ->last issued, ->commit done, commit->next waitA:",
+      [(int(b[16,q]-b[5,q]), int(b[17,q]-b[5,q]), int(b[6,q]-b[5,q]), int(b[3,q+1]-b[6,q]) if q + 1 < n else 0) for q in range(min(n, 12))])
 print("MMA serial probe: m:done-m:gotB per q:", [int(b[11,q]-b[5,q]) for q in range(n)] if buf[11].any() else "n/a")
 print("  q   p:emptyW  p:got  row0  row1  fence  p0:arr  pLast:arr  m:waitA  m:gotA  m:gotB  m:commit  | MMA period  A-wait  B-wait")
 for q in range(n):
