@@ -1030,13 +1030,29 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const uint32_t tacc = tmem_base + ((uint32_t)(qd * 32) << 16) + (uint32_t)(buf * Cfg::ACC_STRIDE);
             constexpr int SLICE = BLOCK_N / (FEPI_WARPS / 4);
             if (t == 0) TL(12);
-            // idle pipeline buffers: A stages hold the per-warp store scratch, B stages the
-            // staged stream-K partials
+            // idle pipeline buffers: the per-warp store scratch and the staged stream-K partials.
+            // Single CTAs: warps 0-3 take the epilogue warps' scratch (free once those have
+            // released the accumulator of the CTA's previous segment), warps 4-7 the start of
+            // the A stages, and the partials get everything behind that (A + B stages, one pass
+            // at BLOCK_N = 256); pairs: A stages for the scratch, B stages for the partials.
+            uint8_t* fscr = sA + warp * EPI_W;
+            uint8_t* fstg = sB;
+            size_t fstg_bytes = (size_t)STAGES * Cfg::B_STAGE_BYTES;
+#ifndef DEFCON_FINAL_STAGE_B_ONLY
+            if (!PAIR && STAGES * Cfg::A_STAGE_BYTES >= 4 * EPI_W) {
+                if (nseg >= 2) {
+                    const int op = nseg - 2;
+                    mbar_wait(&tmem_empty[op % Cfg::NBUF], (uint32_t)(op / Cfg::NBUF) & 1u);
+                }
+                fscr = warp < 4 ? epi_scratch + warp * EPI_W : sA + (warp - 4) * EPI_W;
+                fstg = sA + 4 * EPI_W;
+                fstg_bytes = (size_t)STAGES * Cfg::A_STAGE_BYTES - 4 * EPI_W + (size_t)STAGES * Cfg::B_STAGE_BYTES;
+            }
+#endif
             epilogue_segment<BLOCK_N, SLICE, PAIR, F32>(a, &ymap, sg, tacc, r, (warp >> 2) * SLICE, 4,
                                                   FEPI_WARPS * 32,
                                                   t == 0, fix_flag + 1, T, nct, a.bias_in_smem ? bias_s : nullptr,
-                                                  sA + warp * EPI_W, sB,
-                                             (size_t)STAGES * Cfg::B_STAGE_BYTES, t);
+                                                  fscr, fstg, fstg_bytes, t);
             if (t == 0) TL(13);
         }
     } else if (warp < EPI_WARP0 + 4) {
