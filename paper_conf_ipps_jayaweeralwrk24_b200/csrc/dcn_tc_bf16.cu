@@ -1446,7 +1446,11 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
     // Stream-K tile counters are NOT reset here: the workspace is zero-filled once by its
     // owner and every launch leaves it zeroed (the finisher of each split tile resets it).
     const size_t smem = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_W + (size_t)BM * g.KK * meta_entry<F32>() +
-                        bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0);
+                        bias_smem_offset(STAGES, Cfg::NBUF) + (a.bias_in_smem ? (size_t)g.Cout * 4 : 0)
+#ifdef DEFCON_PROBE_SMEM_PAD   // dev probe: unused shared memory (the L1 it costs the gathers)
+                        + DEFCON_PROBE_SMEM_PAD
+#endif
+        ;
     auto kern = F32 ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false, F32>
                 : PAIR ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>
                 : !tex ? dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, false, false>
