@@ -557,15 +557,21 @@ __device__ __forceinline__ int ld_acquire_gpu(const int* p) {
 constexpr int CS = 32;
 constexpr int EPI_SCRATCH_PER_WARP = 2 * 2048;   // bf16: two 2 KB buffers (32 rows x 64 B)
 // fp32 y: two 4 KB buffers per warp (32 rows x 128 B, 128-byte swizzle)
-template <bool F32>
-__host__ __device__ constexpr int epi_scratch_per_warp() { return F32 ? 2 * 4096 : EPI_SCRATCH_PER_WARP; }
+// BLOCK_N = 512 (bf16): one 2 KB buffer per warp -- its 2-stage pipeline then stays under the
+// shared-memory carveout step that would leave the gathers no L1 (C5 66.5 -> 64.9 us; DESIGN
+// 12b item 15)
+template <bool F32, int BLOCK_N = 256>
+__host__ __device__ constexpr int epi_scratch_per_warp() {
+    return F32 ? 2 * 4096 : BLOCK_N >= 512 ? EPI_SCRATCH_PER_WARP / 2 : EPI_SCRATCH_PER_WARP;
+}
 
+template <int NB = 2>   // 2 KB scratch buffers per warp
 __device__ __forceinline__ void store_group_tma(const CUtensorMap* ymap, uint8_t* scratch, int gi,
                                                 const uint32_t (&pk)[CS / 2], int col, int row0,
                                                 int lane) {
-    uint8_t* buf = scratch + (gi & 1) * 2048;
-    if (gi >= 2) {                         // the store that used this buffer has read it
-        if (lane == 0) bulk_wait_read<1>();
+    uint8_t* buf = scratch + (gi % NB) * 2048;
+    if (gi >= NB) {                        // the store that used this buffer has read it
+        if (lane == 0) bulk_wait_read<NB - 1>();
         __syncwarp();
     }
     const uint32_t base = smem_u32(buf) + lane * 64;
@@ -709,7 +715,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
             uint32_t pk[CS / 2];
 #pragma unroll
             for (int u = 0; u < CS / 2; ++u) pk[u] = pack_bf16x2(acc[2 * u], acc[2 * u + 1]);
-            store_group_tma(ymap, scratch, gi, pk, n0 + c, row0, lane);
+            store_group_tma<BLOCK_N >= 512 ? 1 : 2>(ymap, scratch, gi, pk, n0 + c, row0, lane);
         }
     };
     auto drain = [&]() {
@@ -915,7 +921,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     dcn_fwd_bf16_tc_kernel(const __grid_constant__ CUtensorMap wmap, const __grid_constant__ CUtensorMap wmap_lo,
                            const __grid_constant__ CUtensorMap ymap, const TcArgs a) {
     using Cfg = TcCfg<BLOCK_N, PAIR, F32>;
-    constexpr int EPI_W = epi_scratch_per_warp<F32>();
+    constexpr int EPI_W = epi_scratch_per_warp<F32, BLOCK_N>();
 
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -1338,7 +1344,7 @@ cudaError_t launch_impl(const DcnGeom& g, const DcnPtrs& p, void* ws, size_t ws_
                         const TexPlan* tex, bool hybrid, cudaStream_t stream, const char** detail) {
     using Cfg = TcCfg<BLOCK_N, PAIR, F32>;
     using E = Elem<F32>;
-    constexpr int EPI_W = epi_scratch_per_warp<F32>();
+    constexpr int EPI_W = epi_scratch_per_warp<F32, BLOCK_N>();
     if (PAIR && g_pair_units == 0) {   // how many pairs fit at once (one CTA per SM)
         auto kp = dcn_fwd_bf16_tc_kernel<BLOCK_N, STAGES, 0, PAIR, false>;
         const size_t smem_q = 1024 + (size_t)STAGES * Cfg::STAGE_BYTES + 4 * EPI_SCRATCH_PER_WARP +
