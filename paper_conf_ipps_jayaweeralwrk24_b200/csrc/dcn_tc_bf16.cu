@@ -555,6 +555,9 @@ __device__ __forceinline__ int ld_acquire_gpu(const int* p) {
 // swizzled layout (conflict-free) and stored by one TMA bulk-tensor store (rows >= M and
 // columns >= Cout are clipped by the TMA unit).  Two buffers alternate per warp.
 constexpr int CS = 32;
+#ifndef DEFCON_F32_EPI_NB
+#define DEFCON_F32_EPI_NB 1   // fp32 y: one 4 KB scratch buffer per warp (the 3xTF32 kernel under the carveout cliff)
+#endif
 constexpr int EPI_SCRATCH_PER_WARP = 2 * 2048;   // bf16: two 2 KB buffers (32 rows x 64 B)
 // fp32 y: two 4 KB buffers per warp (32 rows x 128 B, 128-byte swizzle)
 // BLOCK_N = 512 (bf16): one 2 KB buffer per warp -- its 2-stage pipeline then stays under the
@@ -562,7 +565,7 @@ constexpr int EPI_SCRATCH_PER_WARP = 2 * 2048;   // bf16: two 2 KB buffers (32 r
 // 12b item 15)
 template <bool F32, int BLOCK_N = 256>
 __host__ __device__ constexpr int epi_scratch_per_warp() {
-    return F32 ? 2 * 4096 : BLOCK_N >= 512 ? EPI_SCRATCH_PER_WARP / 2 : EPI_SCRATCH_PER_WARP;
+    return F32 ? DEFCON_F32_EPI_NB * 4096 : BLOCK_N >= 512 ? EPI_SCRATCH_PER_WARP / 2 : EPI_SCRATCH_PER_WARP;
 }
 
 template <int NB = 2>   // 2 KB scratch buffers per warp
@@ -589,11 +592,12 @@ __device__ __forceinline__ void store_group_tma(const CUtensorMap* ymap, uint8_t
 
 // fp32 y: 32 columns of this lane's row (128 B) into a 4 KB buffer in the 128-byte swizzled
 // layout (16-byte unit c of row r at c ^ (r % 8)), stored by one 32 x 32 TMA box.
+template <int NB = 2>   // 4 KB scratch buffers per warp
 __device__ __forceinline__ void store_group_tma_f32(const CUtensorMap* ymap, uint8_t* scratch, int gi,
                                                     const float (&v)[CS], int col, int row0, int lane) {
-    uint8_t* buf = scratch + (gi & 1) * 4096;
-    if (gi >= 2) {
-        if (lane == 0) bulk_wait_read<1>();
+    uint8_t* buf = scratch + (gi % NB) * 4096;
+    if (gi >= NB) {
+        if (lane == 0) bulk_wait_read<NB - 1>();
         __syncwarp();
     }
     const uint32_t base = smem_u32(buf) + lane * 128;
@@ -710,7 +714,7 @@ __device__ __forceinline__ void epilogue_segment(const TcArgs& a, const CUtensor
             acc[4 * u] += bb.x; acc[4 * u + 1] += bb.y; acc[4 * u + 2] += bb.z; acc[4 * u + 3] += bb.w;
         }
         if (F32) {
-            store_group_tma_f32(ymap, scratch, gi, acc, n0 + c, row0, lane);
+            store_group_tma_f32<DEFCON_F32_EPI_NB>(ymap, scratch, gi, acc, n0 + c, row0, lane);
         } else {
             uint32_t pk[CS / 2];
 #pragma unroll
